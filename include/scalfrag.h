@@ -1,0 +1,169 @@
+/*
+ * scalfrag.h - C ABI of the B200-native ScalFrag hot path: mode-n sparse MTTKRP.
+ *
+ * What is computed (§II-C, Eq. (4)):
+ *     M = X_(n) (A^(N) ⊙ ... ⊙ A^(n+1) ⊙ A^(n-1) ⊙ ... ⊙ A^(1))
+ * for an N-way COO tensor X (§II-D: entries M(i,j,k,val)),
+ * i.e. elementwise  Y(i,:) = sum_{e: i_n(e)=i} v_e * ⊙_{m≠n} A_m(i_m(e),:)
+ * (reading R1).  Y is OVERWRITTEN (Alg. 1 line 4, PAPER.md L111
+ * "M <- ..."), rows without nonzeros are 0, duplicate coordinates are summed.
+ *
+ * The calls follow the north star: sf_tensor_create (ingest, §8(a) A1; the
+ * paper's "pipelined to the device side"), sf_plan
+ * (matricize + chunk + features + launch selection, PAPER.md L189-199;
+ * §8(a) A2-A4) and sf_mttkrp (the kernel, §8(a) A5-A7).
+ *
+ * Conventions
+ *   - All functions are extern "C", take plain pointers and sizes, never throw,
+ *     and return an sf_status.  On failure no state changes; sf_last_error()
+ *     returns a thread-local detail string.
+ *   - 2 <= nmodes <= SF_MAX_MODES; 1 <= dims[m] <= 2^32-1; indices are 0-based
+ *     uint32; values fp32; factors fp32 row-major I_m x rank (ld = rank).
+ *   - Per-device nnz (per shard) must be < 2^32.  nnz = 0 is valid (Y = 0).
+ *   - A handle is bound to the CUDA device current at create time; it owns all
+ *     device arrays, plans and scratch.  Handles are not thread-safe; calls on
+ *     different handles are independent.
+ *   - Device pointers are CUDA device pointers (e.g. torch tensor .data_ptr()).
+ *     `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - Asynchronous kernel faults surface at the caller's next synchronization
+ *     (as in cuBLAS); the library itself synchronizes only where stated.
+ */
+#ifndef SCALFRAG_H
+#define SCALFRAG_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SF_MAX_MODES 8
+#define SF_HIST_BINS 40
+
+typedef struct sf_tensor_s* sf_tensor_t;
+
+typedef enum {
+  SF_OK = 0,
+  SF_ERR_INVALID_ARG = 1,        /* bad pointer / size / mode / rank */
+  SF_ERR_INDEX_OUT_OF_RANGE = 2, /* some inds[m][e] >= dims[m] */
+  SF_ERR_OUT_OF_MEMORY = 3,      /* cudaMalloc / pinned allocation failed */
+  SF_ERR_NOT_PLANNED = 4,        /* sf_mttkrp before sf_plan(mode, rank) */
+  SF_ERR_UNSUPPORTED = 5,        /* e.g. shard nnz >= 2^32 */
+  SF_ERR_CUDA = 6                /* a CUDA runtime call failed (detail in sf_last_error) */
+} sf_status;
+
+/* Kernel families. */
+typedef enum {
+  SF_KERNEL_AUTO = 0, /* let the selector choose (sf_set_launch only) */
+  SF_KERNEL_COO = 1,  /* nnz-parallel over the raw COO, one vector atomic per nonzero */
+  SF_KERNEL_FRAG = 2  /* sorted fragments: register segmented reduction, factor blocks
+                         staged in shared memory, atomics only at run/fragment edges */
+} sf_kernel_kind;
+
+/* Launch configuration ("combination of launch parameters"),
+ * extended for the fragment kernel. */
+typedef struct {
+  int32_t kernel;        /* sf_kernel_kind */
+  int32_t block_threads; /* threads per CTA, multiple of 32 in [64, 1024] */
+  int32_t ctas_per_sm;   /* FRAG: persistent grid = ctas_per_sm * #SMs (0 = max resident) */
+  int32_t chunk_nnz;     /* FRAG: C, nonzeros per chunk ("segment") */
+  uint32_t staged_mask;  /* FRAG: bit m set => factor m is staged in shared memory by
+                            blocks of block_rows[m] rows (a "tensor block") */
+  uint32_t block_rows[SF_MAX_MODES];
+} sf_launch_t;
+
+/* Tensor feature vector (reading R4). Integers are exact. */
+typedef struct {
+  uint64_t nnz;
+  uint64_t dim;               /* I_n */
+  uint64_t num_slices;        /* non-empty rows of mode n */
+  uint64_t num_fibers;        /* distinct (i_n, i_s) pairs, s = highest mode != n */
+  uint64_t max_nnz_per_slice;
+  uint64_t max_nnz_per_fiber;
+  uint64_t sum_sq_nnz_per_slice;
+  uint64_t slice_hist[SF_HIST_BINS]; /* slices with nnz in [2^b, 2^(b+1)) */
+  int32_t nmodes, mode, secondary, reserved;
+  double slice_ratio;         /* num_slices / I_n */
+  double fiber_ratio;         /* num_fibers / num_slices */
+  double avg_nnz_per_slice, avg_nnz_per_fiber, std_nnz_per_slice;
+} sf_features_t;
+
+typedef struct {
+  sf_features_t feat;   /* features of the whole tensor for this mode */
+  sf_launch_t launch;   /* the launch the plan uses */
+  uint64_t nnz_local;   /* nonzeros of this shard */
+  uint64_t num_tiles;   /* distinct tiles present */
+  uint64_t num_chunks;
+  uint64_t row_begin;   /* this shard touches rows [row_begin, row_end) of Y */
+  uint64_t row_end;
+  uint64_t device_bytes;
+  double plan_ms;       /* device time of the last sf_plan for this (mode, rank) */
+} sf_plan_info_t;
+
+/* ---- lifetime ---------------------------------------------------------- */
+
+/* Ingest (§8(a) A1).  Copies the COO tensor to the device and validates every
+ * index on the device (one synchronization).  inds: nmodes pointers, each to nnz
+ * uint32; vals: nnz floats.  Pointers may be host (pageable or pinned) or device;
+ * host data is uploaded in `segments` chunks through pinned staging buffers over
+ * `streams` CUDA streams, overlapping copies with the device-side range check
+ * (§IV-C; segments/streams <= 0 pick defaults 8/4).
+ * The caller keeps ownership of its buffers (deep copy). */
+sf_status sf_tensor_create(int nmodes, const uint64_t* dims, uint64_t nnz,
+                           const uint32_t* const* inds, const float* vals, sf_tensor_t* out);
+sf_status sf_tensor_create_ex(int nmodes, const uint64_t* dims, uint64_t nnz,
+                              const uint32_t* const* inds, const float* vals, int segments,
+                              int streams, sf_tensor_t* out);
+sf_status sf_tensor_destroy(sf_tensor_t t);
+
+/* Multi-GPU (§8(e)): restrict this handle to shard `rank` of `nranks`: for every mode
+ * it owns matricized positions [floor(rank*nnz/nranks), floor((rank+1)*nnz/nranks)).
+ * Drops existing plans.  Default 1/0. */
+sf_status sf_set_shard(sf_tensor_t t, int nranks, int rank);
+
+/* ---- planning (§8(a) A2-A4) -------------------------------------------- */
+
+/* Sort (matricized order, then tiles), build fragments/chunks, compute features and
+ * select the launch for (mode, rank).  Idempotent; synchronizes the device. */
+sf_status sf_plan(sf_tensor_t t, int mode, int rank);
+/* Override the selector (sweeps, Fig. 4) and re-plan. */
+sf_status sf_set_launch(sf_tensor_t t, int mode, int rank, const sf_launch_t* launch);
+/* Features only (no plan needed). Synchronizes. */
+sf_status sf_features(sf_tensor_t t, int mode, sf_features_t* out);
+sf_status sf_plan_info(sf_tensor_t t, int mode, int rank, sf_plan_info_t* out);
+/* Bit-exact export for tests: perm_host[k] = input position of the k-th nonzero in
+ * kernel order (nnz_local entries); chunks_host: 3*num_chunks uint64 (begin, end, tile).
+ * Either pointer may be NULL. Synchronizes. */
+sf_status sf_plan_export(sf_tensor_t t, int mode, int rank, uint64_t* perm_host,
+                         uint64_t* chunks_host);
+
+/* ---- the hot path (§8(a) A5-A7) ---------------------------------------- */
+
+/* Y = mode-`mode` MTTKRP.  factors: host array of nmodes DEVICE pointers (factors[mode]
+ * is ignored and may be NULL); out: device I_mode x rank fp32, overwritten (with a
+ * shard set, only rows [row_begin,row_end) are written; the rest are zeroed).
+ * Stream-ordered, returns after enqueue.  out must not alias a factor. */
+sf_status sf_mttkrp(sf_tensor_t t, int mode, const float* const* factors, int rank, float* out,
+                    void* stream);
+
+/* One-shot streamed path (the paper's pipeline; §8(a) A8 (ii)):
+ * host COO is uploaded in `segments` pieces over `streams` streams while the
+ * nnz-parallel kernel consumes finished segments; Y (device) is overwritten.
+ * No handle, no sort.  Synchronizes before returning. */
+sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
+                             const uint32_t* const* inds_host, const float* vals_host,
+                             const float* const* factors, int rank, int mode, float* out,
+                             int segments, int streams);
+
+/* ---- diagnostics -------------------------------------------------------- */
+const char* sf_status_string(sf_status s);
+const char* sf_last_error(void);
+/* Number of kernels this library has launched in this process (monotone). */
+uint64_t sf_kernel_launches(void);
+/* Library version string. */
+const char* sf_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SCALFRAG_H */

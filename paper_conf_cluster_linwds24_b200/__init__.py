@@ -1,0 +1,254 @@
+"""ScalFrag on B200: thin Python binding of libscalfrag.so (include/scalfrag.h).
+
+Argument marshalling only -- every step of the hot path (ingest, sort, tiles,
+features, selection, MTTKRP) runs inside the CUDA library.  There is no CPU
+fallback: if the extension is missing the import of ``lib()`` fails loudly.
+
+Arrays may be torch tensors (host, pinned or CUDA) or numpy arrays; index arrays
+are passed as their raw 32-bit pattern (uint32 semantics; torch.int32 tensors are
+accepted as long as every index < 2^31).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+from . import _build
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_lock = threading.Lock()
+_lib = None
+
+SF_MAX_MODES = 8
+SF_HIST_BINS = 40
+KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
+
+STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
+          3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",
+          6: "SF_ERR_CUDA"}
+
+
+class SfError(RuntimeError):
+    def __init__(self, status, detail):
+        self.status = status
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+
+
+class Launch(ctypes.Structure):
+    _fields_ = [("kernel", ctypes.c_int32), ("block_threads", ctypes.c_int32),
+                ("ctas_per_sm", ctypes.c_int32), ("chunk_nnz", ctypes.c_int32),
+                ("staged_mask", ctypes.c_uint32), ("block_rows", ctypes.c_uint32 * SF_MAX_MODES)]
+
+    def as_dict(self):
+        return {"kernel": {0: "auto", 1: "coo", 2: "frag"}.get(self.kernel, self.kernel),
+                "block_threads": self.block_threads, "ctas_per_sm": self.ctas_per_sm,
+                "chunk_nnz": self.chunk_nnz, "staged_mask": self.staged_mask,
+                "block_rows": list(self.block_rows)}
+
+    @classmethod
+    def make(cls, kernel=KERNEL_FRAG, block_threads=512, ctas_per_sm=0, chunk_nnz=1024,
+             staged=None):
+        """staged: {mode: block_rows}"""
+        l = cls()
+        l.kernel, l.block_threads, l.ctas_per_sm, l.chunk_nnz = kernel, block_threads, ctas_per_sm, chunk_nnz
+        mask = 0
+        for m, r in (staged or {}).items():
+            mask |= 1 << m
+            l.block_rows[m] = r
+        l.staged_mask = mask
+        return l
+
+
+class Features(ctypes.Structure):
+    _fields_ = [("nnz", ctypes.c_uint64), ("dim", ctypes.c_uint64), ("num_slices", ctypes.c_uint64),
+                ("num_fibers", ctypes.c_uint64), ("max_nnz_per_slice", ctypes.c_uint64),
+                ("max_nnz_per_fiber", ctypes.c_uint64), ("sum_sq_nnz_per_slice", ctypes.c_uint64),
+                ("slice_hist", ctypes.c_uint64 * SF_HIST_BINS), ("nmodes", ctypes.c_int32),
+                ("mode", ctypes.c_int32), ("secondary", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("slice_ratio", ctypes.c_double), ("fiber_ratio", ctypes.c_double),
+                ("avg_nnz_per_slice", ctypes.c_double), ("avg_nnz_per_fiber", ctypes.c_double),
+                ("std_nnz_per_slice", ctypes.c_double)]
+
+    def as_dict(self):
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("slice_hist", "reserved")}
+        d["slice_hist"] = list(self.slice_hist)
+        return d
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("feat", Features), ("launch", Launch), ("nnz_local", ctypes.c_uint64),
+                ("num_tiles", ctypes.c_uint64), ("num_chunks", ctypes.c_uint64),
+                ("row_begin", ctypes.c_uint64), ("row_end", ctypes.c_uint64),
+                ("device_bytes", ctypes.c_uint64), ("plan_ms", ctypes.c_double)]
+
+    def as_dict(self):
+        return {"features": self.feat.as_dict(), "launch": self.launch.as_dict(),
+                "nnz_local": self.nnz_local, "num_tiles": self.num_tiles,
+                "num_chunks": self.num_chunks, "row_begin": self.row_begin,
+                "row_end": self.row_end, "device_bytes": self.device_bytes,
+                "plan_ms": self.plan_ms}
+
+
+EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
+            "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
+            "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
+            "sf_kernel_launches", "sf_version"]
+
+
+def lib(build_if_missing: bool = True):
+    """Load libscalfrag.so (building it in-tree with nvcc if absent)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            so = _build.SO
+            if not os.path.exists(so):
+                if not build_if_missing:
+                    raise RuntimeError(f"{so} missing: run __graft_entry__.build()")
+                _build.build()
+            L = ctypes.CDLL(so)
+            P, I, U64 = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64
+            L.sf_tensor_create.argtypes = [I, P, U64, P, P, ctypes.POINTER(P)]
+            L.sf_tensor_create_ex.argtypes = [I, P, U64, P, P, I, I, ctypes.POINTER(P)]
+            L.sf_tensor_destroy.argtypes = [P]
+            L.sf_set_shard.argtypes = [P, I, I]
+            L.sf_plan.argtypes = [P, I, I]
+            L.sf_set_launch.argtypes = [P, I, I, ctypes.POINTER(Launch)]
+            L.sf_features.argtypes = [P, I, ctypes.POINTER(Features)]
+            L.sf_plan_info.argtypes = [P, I, I, ctypes.POINTER(PlanInfo)]
+            L.sf_plan_export.argtypes = [P, I, I, P, P]
+            L.sf_mttkrp.argtypes = [P, I, P, I, P, P]
+            L.sf_mttkrp_streamed.argtypes = [I, P, U64, P, P, P, I, I, P, I, I]
+            for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
+                       "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
+                       "sf_mttkrp", "sf_mttkrp_streamed"]:
+                getattr(L, fn).restype = ctypes.c_int
+            L.sf_status_string.argtypes = [I]
+            L.sf_status_string.restype = ctypes.c_char_p
+            L.sf_last_error.argtypes = []
+            L.sf_last_error.restype = ctypes.c_char_p
+            L.sf_kernel_launches.argtypes = []
+            L.sf_kernel_launches.restype = U64
+            L.sf_version.argtypes = []
+            L.sf_version.restype = ctypes.c_char_p
+            _lib = L
+    return _lib
+
+
+def _check(rc):
+    if rc != 0:
+        raise SfError(rc, lib().sf_last_error().decode())
+
+
+def _ptr(x):
+    if x is None:
+        return None
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if hasattr(x, "ctypes"):
+        return x.ctypes.data
+    if isinstance(x, int):
+        return x
+    raise TypeError(f"cannot take a pointer of {type(x)}")
+
+
+def _stream_handle(stream):
+    if stream is None:
+        try:
+            import torch
+            if torch.cuda.is_available():
+                return torch.cuda.current_stream().cuda_stream
+        except Exception:
+            pass
+        return 0
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def kernel_launches() -> int:
+    return int(lib().sf_kernel_launches())
+
+
+def version() -> str:
+    return lib().sf_version().decode()
+
+
+class Tensor:
+    """Handle of a device-resident COO tensor (sf_tensor_t)."""
+
+    def __init__(self, dims, inds, vals, segments=0, streams=0):
+        self.dims = tuple(int(d) for d in dims)
+        self.nmodes = len(self.dims)
+        self.nnz = int(len(vals))
+        d = (ctypes.c_uint64 * self.nmodes)(*self.dims)
+        ip = (ctypes.c_void_p * self.nmodes)(*[_ptr(a) for a in inds])
+        h = ctypes.c_void_p()
+        _check(lib().sf_tensor_create_ex(self.nmodes, d, self.nnz, ip, _ptr(vals), int(segments),
+                                         int(streams), ctypes.byref(h)))
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().sf_tensor_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def set_shard(self, nranks, rank):
+        _check(lib().sf_set_shard(self._h, int(nranks), int(rank)))
+
+    def plan(self, mode, rank):
+        _check(lib().sf_plan(self._h, int(mode), int(rank)))
+
+    def set_launch(self, mode, rank, launch: Launch):
+        _check(lib().sf_set_launch(self._h, int(mode), int(rank), ctypes.byref(launch)))
+
+    def features(self, mode) -> dict:
+        f = Features()
+        _check(lib().sf_features(self._h, int(mode), ctypes.byref(f)))
+        return f.as_dict()
+
+    def plan_info(self, mode, rank) -> dict:
+        p = PlanInfo()
+        _check(lib().sf_plan_info(self._h, int(mode), int(rank), ctypes.byref(p)))
+        return p.as_dict()
+
+    def plan_export(self, mode, rank):
+        import numpy as np
+        info = self.plan_info(mode, rank)
+        perm = np.empty(info["nnz_local"], np.uint64)
+        chunks = np.empty((info["num_chunks"], 3), np.uint64)
+        _check(lib().sf_plan_export(self._h, int(mode), int(rank), perm.ctypes.data if perm.size else None,
+                                    chunks.ctypes.data if chunks.size else None))
+        return perm, chunks
+
+    def mttkrp(self, mode, factors, out, rank=None, stream=None):
+        """out <- mode-`mode` MTTKRP (device tensors; stream-ordered)."""
+        rank = int(out.shape[1]) if rank is None else int(rank)
+        fp = (ctypes.c_void_p * self.nmodes)(*[_ptr(f) if (m != mode and f is not None) else None
+                                               for m, f in enumerate(factors)])
+        _check(lib().sf_mttkrp(self._h, int(mode), fp, rank, _ptr(out), _stream_handle(stream)))
+        return out
+
+
+def mttkrp_streamed(dims, inds, vals, factors, mode, out, segments=8, streams=4):
+    """One-shot streamed MTTKRP of a HOST COO tensor (the paper's pipeline, §IV-C)."""
+    N = len(dims)
+    d = (ctypes.c_uint64 * N)(*[int(x) for x in dims])
+    ip = (ctypes.c_void_p * N)(*[_ptr(a) for a in inds])
+    fp = (ctypes.c_void_p * N)(*[_ptr(f) if (m != mode and f is not None) else None
+                                 for m, f in enumerate(factors)])
+    _check(lib().sf_mttkrp_streamed(N, d, int(len(vals)), ip, _ptr(vals), fp, int(out.shape[1]), int(mode),
+                                    _ptr(out), int(segments), int(streams)))
+    return out

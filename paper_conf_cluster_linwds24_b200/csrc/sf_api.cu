@@ -1,0 +1,468 @@
+// sf_api.cu - the C ABI (include/scalfrag.h) and the ingest / stream pipeline.
+//
+// Ingest (§8(a) A1) and the stream pipeline (§8(a) A8) follow PAPER.md §IV-C
+// (L201-229): the COO tensor is cut into equal-nnz contiguous segments (reading R12),
+// each segment is transferred asynchronously on its own CUDA stream, and the device
+// works on finished segments while later ones are still in flight (here: the index
+// range check for the resident path, the nnz-parallel kernel for the one-shot
+// streamed path).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "sf_internal.h"
+
+namespace sf {
+
+std::atomic<uint64_t> g_launches{0};
+static thread_local std::string g_err;
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+void DevBuf::alloc(size_t b) {
+  release();
+  if (b == 0) b = 16;
+  void* q = nullptr;
+  cudaError_t e = cudaMalloc(&q, b);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    throw CudaError{e, "cudaMalloc"};
+  }
+  p = q;
+  bytes = b;
+}
+
+void DevBuf::release() {
+  if (p) cudaFree(p);
+  p = nullptr;
+  bytes = 0;
+}
+
+size_t Plan::device_bytes() const {
+  size_t b = val.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes;
+  for (int m = 0; m < SF_MAX_MODES; ++m) b += ind[m].bytes;
+  return b;
+}
+
+Tensor::~Tensor() {
+  for (auto& kv : plans) delete kv.second;
+  plans.clear();
+  if (stream) cudaStreamDestroy(stream);
+}
+
+template <class F>
+static sf_status guard(F&& f) {
+  try {
+    return f();
+  } catch (const CudaError& e) {
+    set_error(std::string(e.what) + ": " + cudaGetErrorString(e.err));
+    return (e.err == cudaErrorMemoryAllocation) ? SF_ERR_OUT_OF_MEMORY : SF_ERR_CUDA;
+  } catch (const StatusError& e) {
+    set_error(e.msg);
+    return e.st;
+  } catch (const std::bad_alloc&) {
+    set_error("host allocation failed");
+    return SF_ERR_OUT_OF_MEMORY;
+  } catch (...) {
+    set_error("unknown internal error");
+    return SF_ERR_CUDA;
+  }
+}
+
+static bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a{};
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+static bool is_pinned_ptr(const void* p) {
+  cudaPointerAttributes a{};
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost;
+}
+
+// Segmented, multi-stream upload of the (N+1) COO arrays into the tensor's device
+// arrays, with the range check of each segment enqueued behind its copy.
+static void upload(Tensor& t, const uint32_t* const* inds, const float* vals, int segments,
+                   int nstreams, int* d_flag) {
+  const int N = t.nmodes;
+  const uint64_t n = t.nnz;
+  if (segments <= 0) segments = 8;
+  if (nstreams <= 0) nstreams = 4;
+  segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, n)));
+  nstreams = std::max(1, std::min(nstreams, segments));
+  std::vector<cudaStream_t> st(nstreams);
+  for (auto& s : st) SF_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  bool pageable = false;
+  for (int m = 0; m < N && !pageable; ++m) pageable = !is_pinned_ptr(inds[m]);
+  if (!pageable) pageable = !is_pinned_ptr(vals);
+  const uint64_t seg_len = (n + segments - 1) / segments;
+  // pinned staging ring for pageable input: one slot per stream
+  std::vector<void*> stage(nstreams, nullptr);
+  std::vector<cudaEvent_t> done(nstreams, nullptr);
+  try {
+    if (pageable) {
+      for (int s = 0; s < nstreams; ++s) {
+        SF_CUDA(cudaMallocHost(&stage[s], (size_t)seg_len * 4 * (N + 1) + 64));
+        SF_CUDA(cudaEventCreateWithFlags(&done[s], cudaEventDisableTiming));
+      }
+    }
+    for (int k = 0; k < segments; ++k) {
+      const uint64_t a = (uint64_t)k * seg_len;
+      if (a >= n) break;
+      const uint64_t b = std::min(n, a + seg_len);
+      const uint64_t len = b - a;
+      const int s = k % nstreams;
+      uint32_t* dseg[SF_MAX_MODES];
+      for (int m = 0; m < N; ++m) dseg[m] = t.ind[m].as<uint32_t>() + a;
+      if (pageable) {
+        if (k >= nstreams) SF_CUDA(cudaEventSynchronize(done[s]));  // slot free again
+        char* h = static_cast<char*>(stage[s]);
+        for (int m = 0; m < N; ++m) {
+          memcpy(h + (size_t)m * len * 4, inds[m] + a, len * 4);
+          SF_CUDA(cudaMemcpyAsync(dseg[m], h + (size_t)m * len * 4, len * 4, cudaMemcpyHostToDevice, st[s]));
+        }
+        memcpy(h + (size_t)N * len * 4, vals + a, len * 4);
+        SF_CUDA(cudaMemcpyAsync(t.val.as<float>() + a, h + (size_t)N * len * 4, len * 4,
+                                cudaMemcpyHostToDevice, st[s]));
+        SF_CUDA(cudaEventRecord(done[s], st[s]));
+      } else {
+        for (int m = 0; m < N; ++m)
+          SF_CUDA(cudaMemcpyAsync(dseg[m], inds[m] + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+        SF_CUDA(cudaMemcpyAsync(t.val.as<float>() + a, vals + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+      }
+      validate_indices(N, t.dims, len, dseg, d_flag, st[s]);
+    }
+    for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
+  } catch (...) {
+    for (auto& s : st) cudaStreamSynchronize(s);
+    for (auto& s : st) cudaStreamDestroy(s);
+    for (auto& p : stage) if (p) cudaFreeHost(p);
+    for (auto& e : done) if (e) cudaEventDestroy(e);
+    throw;
+  }
+  for (auto& s : st) cudaStreamDestroy(s);
+  for (auto& p : stage) if (p) cudaFreeHost(p);
+  for (auto& e : done) if (e) cudaEventDestroy(e);
+}
+
+static Tensor* as_tensor(sf_tensor_t h) { return reinterpret_cast<Tensor*>(h); }
+
+static void check_mode_rank(const Tensor& t, int mode, int rank) {
+  if (mode < 0 || mode >= t.nmodes) throw StatusError{SF_ERR_INVALID_ARG, "mode out of range"};
+  if (rank < 1 || rank > 4096) throw StatusError{SF_ERR_INVALID_ARG, "rank out of range [1, 4096]"};
+}
+
+static Plan* get_plan(Tensor& t, int mode, int rank) {
+  auto it = t.plans.find({mode, rank});
+  return it == t.plans.end() ? nullptr : it->second;
+}
+
+static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override_launch) {
+  SF_CUDA(cudaSetDevice(t.device));
+  sf_features_t f;
+  compute_features(t, mode, &f);
+  const uint64_t lo = (uint64_t)(((unsigned __int128)t.rank * t.nnz) / t.nranks);
+  const uint64_t hi = (uint64_t)(((unsigned __int128)(t.rank + 1) * t.nnz) / t.nranks);
+  sf_launch_t l;
+  if (override_launch && override_launch->kernel != SF_KERNEL_AUTO) {
+    l = *override_launch;
+    normalize_launch(t, mode, rank, l);
+  } else {
+    l = select_launch(t, f, mode, rank, hi - lo);
+  }
+  if (l.kernel == SF_KERNEL_FRAG && frag_smem_bytes(t, mode, rank, l) > t.smem_optin)
+    throw StatusError{SF_ERR_INVALID_ARG, "launch needs more shared memory than the device has"};
+  Plan* p = new Plan();
+  try {
+    build_plan(t, *p, mode, rank, l);
+  } catch (...) {
+    delete p;
+    throw;
+  }
+  Plan* old = get_plan(t, mode, rank);
+  delete old;
+  t.plans[{mode, rank}] = p;
+}
+
+}  // namespace sf
+
+using namespace sf;
+
+extern "C" {
+
+sf_status sf_tensor_create_ex(int nmodes, const uint64_t* dims, uint64_t nnz,
+                              const uint32_t* const* inds, const float* vals, int segments,
+                              int streams, sf_tensor_t* out) {
+  return guard([&]() -> sf_status {
+    if (!out) throw StatusError{SF_ERR_INVALID_ARG, "out is NULL"};
+    *out = nullptr;
+    if (nmodes < 2 || nmodes > SF_MAX_MODES || !dims)
+      throw StatusError{SF_ERR_INVALID_ARG, "nmodes must be in [2, 8] and dims non-NULL"};
+    for (int m = 0; m < nmodes; ++m)
+      if (dims[m] < 1 || dims[m] > 0xFFFFFFFFull)
+        throw StatusError{SF_ERR_INVALID_ARG, "dims[m] must be in [1, 2^32-1]"};
+    if (nnz > 0 && (!inds || !vals)) throw StatusError{SF_ERR_INVALID_ARG, "inds/vals NULL"};
+    if (nnz > 0)
+      for (int m = 0; m < nmodes; ++m)
+        if (!inds[m]) throw StatusError{SF_ERR_INVALID_ARG, "inds[m] is NULL"};
+    Tensor* t = new Tensor();
+    try {
+      SF_CUDA(cudaGetDevice(&t->device));
+      SF_CUDA(cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, t->device));
+      int optin = 0;
+      SF_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, t->device));
+      t->smem_optin = (size_t)optin;
+      SF_CUDA(cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking));
+      t->nmodes = nmodes;
+      t->nnz = nnz;
+      for (int m = 0; m < nmodes; ++m) {
+        t->dims[m] = dims[m];
+        t->ind[m].alloc(nnz * 4 + kPadBytes);
+      }
+      t->val.alloc(nnz * 4 + kPadBytes);
+      DevBuf flag(16);
+      SF_CUDA(cudaMemsetAsync(flag.p, 0, 16, t->stream));
+      SF_CUDA(cudaStreamSynchronize(t->stream));
+      if (nnz > 0) {
+        bool dev = is_device_ptr(vals);
+        for (int m = 0; m < nmodes; ++m) dev = dev && is_device_ptr(inds[m]);
+        if (dev) {
+          for (int m = 0; m < nmodes; ++m)
+            SF_CUDA(cudaMemcpyAsync(t->ind[m].p, inds[m], nnz * 4, cudaMemcpyDeviceToDevice, t->stream));
+          SF_CUDA(cudaMemcpyAsync(t->val.p, vals, nnz * 4, cudaMemcpyDeviceToDevice, t->stream));
+          uint32_t* di[SF_MAX_MODES];
+          for (int m = 0; m < nmodes; ++m) di[m] = t->ind[m].as<uint32_t>();
+          validate_indices(nmodes, t->dims, nnz, di, flag.as<int>(), t->stream);
+        } else {
+          upload(*t, inds, vals, segments, streams, flag.as<int>());
+        }
+      }
+      int bad = 0;
+      SF_CUDA(cudaMemcpyAsync(&bad, flag.p, 4, cudaMemcpyDeviceToHost, t->stream));
+      SF_CUDA(cudaStreamSynchronize(t->stream));
+      if (bad) throw StatusError{SF_ERR_INDEX_OUT_OF_RANGE, "some index is >= its dimension"};
+    } catch (...) {
+      delete t;
+      throw;
+    }
+    *out = reinterpret_cast<sf_tensor_t>(t);
+    return SF_OK;
+  });
+}
+
+sf_status sf_tensor_create(int nmodes, const uint64_t* dims, uint64_t nnz,
+                           const uint32_t* const* inds, const float* vals, sf_tensor_t* out) {
+  return sf_tensor_create_ex(nmodes, dims, nnz, inds, vals, 0, 0, out);
+}
+
+sf_status sf_tensor_destroy(sf_tensor_t h) {
+  return guard([&]() -> sf_status {
+    if (!h) return SF_OK;
+    Tensor* t = as_tensor(h);
+    cudaSetDevice(t->device);
+    cudaStreamSynchronize(t->stream);
+    delete t;
+    return SF_OK;
+  });
+}
+
+sf_status sf_set_shard(sf_tensor_t h, int nranks, int rank) {
+  return guard([&]() -> sf_status {
+    if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
+    if (nranks < 1 || rank < 0 || rank >= nranks) throw StatusError{SF_ERR_INVALID_ARG, "bad shard"};
+    Tensor* t = as_tensor(h);
+    for (auto& kv : t->plans) delete kv.second;
+    t->plans.clear();
+    t->nranks = nranks;
+    t->rank = rank;
+    return SF_OK;
+  });
+}
+
+sf_status sf_plan(sf_tensor_t h, int mode, int rank) {
+  return guard([&]() -> sf_status {
+    if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    if (get_plan(*t, mode, rank)) return SF_OK;
+    make_plan(*t, mode, rank, nullptr);
+    return SF_OK;
+  });
+}
+
+sf_status sf_set_launch(sf_tensor_t h, int mode, int rank, const sf_launch_t* launch) {
+  return guard([&]() -> sf_status {
+    if (!h || !launch) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    make_plan(*t, mode, rank, launch);
+    return SF_OK;
+  });
+}
+
+sf_status sf_features(sf_tensor_t h, int mode, sf_features_t* out) {
+  return guard([&]() -> sf_status {
+    if (!h || !out) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, 1);
+    SF_CUDA(cudaSetDevice(t->device));
+    compute_features(*t, mode, out);
+    return SF_OK;
+  });
+}
+
+sf_status sf_plan_info(sf_tensor_t h, int mode, int rank, sf_plan_info_t* out) {
+  return guard([&]() -> sf_status {
+    if (!h || !out) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    Plan* p = get_plan(*t, mode, rank);
+    if (!p) throw StatusError{SF_ERR_NOT_PLANNED, "sf_plan(mode, rank) has not been called"};
+    memset(out, 0, sizeof(*out));
+    out->feat = p->feat;
+    out->launch = p->launch;
+    out->nnz_local = p->nnz_local;
+    out->num_tiles = p->num_tiles;
+    out->num_chunks = p->num_chunks;
+    out->row_begin = p->row_begin;
+    out->row_end = p->row_end;
+    out->device_bytes = p->device_bytes();
+    out->plan_ms = p->plan_ms;
+    return SF_OK;
+  });
+}
+
+sf_status sf_plan_export(sf_tensor_t h, int mode, int rank, uint64_t* perm_host, uint64_t* chunks_host) {
+  return guard([&]() -> sf_status {
+    if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    Plan* p = get_plan(*t, mode, rank);
+    if (!p) throw StatusError{SF_ERR_NOT_PLANNED, "sf_plan(mode, rank) has not been called"};
+    SF_CUDA(cudaSetDevice(t->device));
+    if (perm_host && p->nnz_local) {
+      std::vector<uint32_t> tmp(p->nnz_local);
+      SF_CUDA(cudaMemcpy(tmp.data(), p->perm.p, p->nnz_local * 4, cudaMemcpyDeviceToHost));
+      for (uint64_t k = 0; k < p->nnz_local; ++k) perm_host[k] = tmp[k];
+    }
+    if (chunks_host && p->num_chunks) {
+      std::vector<uint32_t> b(p->num_chunks + 1);
+      std::vector<uint64_t> tl(p->num_chunks);
+      SF_CUDA(cudaMemcpy(b.data(), p->chunk_begin.p, (p->num_chunks + 1) * 4, cudaMemcpyDeviceToHost));
+      SF_CUDA(cudaMemcpy(tl.data(), p->chunk_tile.p, p->num_chunks * 8, cudaMemcpyDeviceToHost));
+      for (uint64_t j = 0; j < p->num_chunks; ++j) {
+        chunks_host[3 * j] = b[j];
+        chunks_host[3 * j + 1] = b[j + 1];
+        chunks_host[3 * j + 2] = tl[j];
+      }
+    }
+    return SF_OK;
+  });
+}
+
+sf_status sf_mttkrp(sf_tensor_t h, int mode, const float* const* factors, int rank, float* out,
+                    void* stream) {
+  return guard([&]() -> sf_status {
+    if (!h || !factors || !out) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    Plan* p = get_plan(*t, mode, rank);
+    if (!p) throw StatusError{SF_ERR_NOT_PLANNED, "sf_plan(mode, rank) has not been called"};
+    for (int m = 0; m < t->nmodes; ++m)
+      if (m != mode && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
+    launch_mttkrp(*t, *p, factors, out, static_cast<cudaStream_t>(stream));
+    return SF_OK;
+  });
+}
+
+sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
+                             const uint32_t* const* inds_host, const float* vals_host,
+                             const float* const* factors, int rank, int mode, float* out,
+                             int segments, int streams) {
+  return guard([&]() -> sf_status {
+    if (nmodes < 2 || nmodes > SF_MAX_MODES || !dims || !factors || !out)
+      throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
+    if (mode < 0 || mode >= nmodes || rank < 1) throw StatusError{SF_ERR_INVALID_ARG, "bad mode/rank"};
+    if (nnz > 0 && (!inds_host || !vals_host)) throw StatusError{SF_ERR_INVALID_ARG, "NULL COO"};
+    for (int m = 0; m < nmodes; ++m)
+      if (m != mode && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
+    if (segments <= 0) segments = 8;
+    if (streams <= 0) streams = 4;
+    segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, nnz)));
+    streams = std::max(1, std::min(streams, segments));
+    const uint64_t seg_len = (nnz + segments - 1) / segments;
+    std::vector<cudaStream_t> st(streams);
+    for (auto& s : st) SF_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    std::vector<DevBuf> ring;
+    DevBuf flag(16);
+    cudaEvent_t zeroed = nullptr;
+    try {
+      ring.reserve(streams);
+      for (int s = 0; s < streams; ++s) ring.emplace_back((size_t)seg_len * 4 * (nmodes + 1) + 64);
+      SF_CUDA(cudaEventCreateWithFlags(&zeroed, cudaEventDisableTiming));
+      SF_CUDA(cudaMemsetAsync(flag.p, 0, 16, st[0]));
+      SF_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * dims[mode] * (size_t)rank, st[0]));
+      SF_CUDA(cudaEventRecord(zeroed, st[0]));
+      for (int s = 1; s < streams; ++s) SF_CUDA(cudaStreamWaitEvent(st[s], zeroed, 0));
+      for (int k = 0; k < segments; ++k) {
+        const uint64_t a = (uint64_t)k * seg_len;
+        if (a >= nnz) break;
+        const uint64_t len = std::min(nnz, a + seg_len) - a;
+        const int s = k % streams;
+        char* base = ring[s].as<char>();
+        uint32_t* di[SF_MAX_MODES];
+        for (int m = 0; m < nmodes; ++m) {
+          di[m] = reinterpret_cast<uint32_t*>(base + (size_t)m * seg_len * 4);
+          SF_CUDA(cudaMemcpyAsync(di[m], inds_host[m] + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+        }
+        float* dv = reinterpret_cast<float*>(base + (size_t)nmodes * seg_len * 4);
+        SF_CUDA(cudaMemcpyAsync(dv, vals_host + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+        validate_indices(nmodes, dims, len, di, flag.as<int>(), st[s]);
+        launch_coo(nmodes, dims, len, di, dv, factors, rank, mode, out, st[s]);
+      }
+      for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
+      int bad = 0;
+      SF_CUDA(cudaMemcpy(&bad, flag.p, 4, cudaMemcpyDeviceToHost));
+      for (auto& s : st) cudaStreamDestroy(s);
+      cudaEventDestroy(zeroed);
+      if (bad) throw StatusError{SF_ERR_INDEX_OUT_OF_RANGE, "some index is >= its dimension"};
+    } catch (...) {
+      for (auto& s : st) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
+      if (zeroed) cudaEventDestroy(zeroed);
+      throw;
+    }
+    return SF_OK;
+  });
+}
+
+const char* sf_status_string(sf_status s) {
+  switch (s) {
+    case SF_OK: return "SF_OK";
+    case SF_ERR_INVALID_ARG: return "SF_ERR_INVALID_ARG";
+    case SF_ERR_INDEX_OUT_OF_RANGE: return "SF_ERR_INDEX_OUT_OF_RANGE";
+    case SF_ERR_OUT_OF_MEMORY: return "SF_ERR_OUT_OF_MEMORY";
+    case SF_ERR_NOT_PLANNED: return "SF_ERR_NOT_PLANNED";
+    case SF_ERR_UNSUPPORTED: return "SF_ERR_UNSUPPORTED";
+    case SF_ERR_CUDA: return "SF_ERR_CUDA";
+    default: return "SF_ERR_UNKNOWN";
+  }
+}
+
+const char* sf_last_error(void) { return g_err.c_str(); }
+
+uint64_t sf_kernel_launches(void) { return g_launches.load(); }
+
+const char* sf_version(void) { return "scalfrag-b200 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,114 @@
+// sf_internal.h - internal types of libscalfrag (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <map>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "../../include/scalfrag.h"
+
+namespace sf {
+
+// Thread-local error detail + status plumbing.
+void set_error(const std::string& msg);
+extern std::atomic<uint64_t> g_launches;
+inline void count_launch(uint64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+struct CudaError {
+  cudaError_t err;
+  const char* what;
+};
+
+#define SF_CUDA(call)                                                      \
+  do {                                                                     \
+    cudaError_t _e = (call);                                               \
+    if (_e != cudaSuccess) throw ::sf::CudaError{_e, #call};               \
+  } while (0)
+
+struct StatusError {
+  sf_status st;
+  std::string msg;
+};
+
+// RAII device buffer.
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  DevBuf() = default;
+  explicit DevBuf(size_t b) { alloc(b); }
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : p(o.p), bytes(o.bytes) { o.p = nullptr; o.bytes = 0; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    if (this != &o) { release(); p = o.p; bytes = o.bytes; o.p = nullptr; o.bytes = 0; }
+    return *this;
+  }
+  ~DevBuf() { release(); }
+  void alloc(size_t b);
+  void release();
+  template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// Padding (bytes) added to every streamed array so 16-byte-aligned bulk copies of
+// an aligned superset of a chunk never read past the allocation.
+constexpr size_t kPadBytes = 64;
+
+struct Plan {
+  int mode = -1, rank = 0;
+  sf_launch_t launch{};
+  sf_features_t feat{};
+  uint64_t nnz_local = 0;
+  uint64_t num_tiles = 0, num_chunks = 0;
+  uint64_t row_begin = 0, row_end = 0;
+  double plan_ms = 0;
+  // kernel-order arrays (SoA): sorted indices of every mode + values + input position
+  DevBuf ind[SF_MAX_MODES];
+  DevBuf val;
+  DevBuf perm;          // uint32 input position per sorted slot
+  DevBuf chunk_begin;   // uint32[num_chunks + 1]
+  DevBuf chunk_tile;    // uint64[num_chunks]
+  size_t device_bytes() const;
+};
+
+struct Tensor {
+  int device = 0;
+  int nmodes = 0;
+  uint64_t dims[SF_MAX_MODES] = {};
+  uint64_t nnz = 0;
+  int nranks = 1, rank = 0;
+  int num_sms = 148;
+  size_t smem_optin = 227 * 1024;
+  DevBuf ind[SF_MAX_MODES];  // raw COO (input order)
+  DevBuf val;
+  bool have_features[SF_MAX_MODES] = {};
+  sf_features_t features[SF_MAX_MODES] = {};
+  std::map<std::pair<int, int>, Plan*> plans;  // (mode, rank) -> plan
+  cudaStream_t stream = nullptr;               // internal stream for planning
+  ~Tensor();
+};
+
+// ---- planning (sf_plan.cu) ----
+void compute_features(Tensor& t, int mode, sf_features_t* out);
+void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch);
+// ---- selection (sf_select.cpp) ----
+sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank,
+                          uint64_t nnz_local);
+void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l);
+size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l);
+// ---- kernels (sf_mttkrp.cu) ----
+void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
+                   cudaStream_t s);
+void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* const* inds,
+                const float* vals, const float* const* factors, int rank, int mode, float* out,
+                cudaStream_t s);
+int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem);
+bool frag_supported(int nmodes, int rank);
+void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
+                      uint32_t* const* inds, int* d_flag, cudaStream_t s);
+
+}  // namespace sf

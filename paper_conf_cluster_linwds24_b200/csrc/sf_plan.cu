@@ -1,0 +1,447 @@
+// sf_plan.cu - device-side preprocessing (§8(a) A2-A4): integer-exact.
+//
+// "ScalFrag first matricizes the input tensor and then chunks the
+// matricized tensor ... uses a trained model to select the best combination of
+// launch parameters based on the sparsity features of the matrixed tensor after
+// chunking."  Here, per (mode n, rank):
+//   1. matricized order: stable LSD radix sort of the key i_n * I_s + i_s with the
+//      input position as payload (s = highest mode != n; reading R10);
+//   2. features from run lengths of that order;
+//   3. shard cut [floor(p*nnz/P), floor((p+1)*nnz/P)) of that order (§8(e));
+//   4. tiles ("tensor blocks ... based on the resource constraints of hardware",
+//      PAPER.md L34): a second stable sort by tile id -> order (tile, i_n, i_s, pos);
+//   5. gather the kernel-order SoA arrays;
+//   6. chunks ("segments"): a new chunk at every tile start and every
+//      C nonzeros inside a tile.
+// All of it is integer work; tests compare it == against oracle/plan.py.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cstring>
+
+#include "sf_internal.h"
+
+namespace sf {
+
+static inline int bitlen(uint64_t x) {
+  int b = 0;
+  while (x) { ++b; x >>= 1; }
+  return b;
+}
+
+static inline int grid_for(uint64_t n, int threads = 256) {
+  return (int)std::max<uint64_t>(1, std::min<uint64_t>((n + threads - 1) / threads, 148ull * 32));
+}
+
+// ---------------------------------------------------------------------------
+__global__ void key_matricized_kernel(const uint32_t* __restrict__ in, const uint32_t* __restrict__ is,
+                                      uint64_t Is, uint64_t n, uint64_t* __restrict__ key,
+                                      uint32_t* __restrict__ pos) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    key[e] = (uint64_t)in[e] * Is + (uint64_t)is[e];
+    pos[e] = (uint32_t)e;
+  }
+}
+
+// Run-start positions for slices (i_n = key / Is) and fibers (key) in the sorted order.
+__global__ void run_start_kernel(const uint64_t* __restrict__ key, uint64_t Is, uint64_t n,
+                                 uint32_t* __restrict__ sstart, uint32_t* __restrict__ fstart,
+                                 unsigned long long* __restrict__ counts /*[2]*/) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long ns = 0, nf = 0;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    const uint64_t k = key[e];
+    bool fs = true, ss = true;
+    if (e > 0) {
+      const uint64_t kp = key[e - 1];
+      fs = (k != kp);
+      ss = (k / Is) != (kp / Is);
+    }
+    sstart[e] = ss ? (uint32_t)e : 0u;
+    fstart[e] = fs ? (uint32_t)e : 0u;
+    ns += ss;
+    nf += fs;
+  }
+  typedef cub::BlockReduce<unsigned long long, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long a = BR(tmp).Sum(ns);
+  __syncthreads();
+  unsigned long long b = BR(tmp).Sum(nf);
+  if (threadIdx.x == 0) {
+    atomicAdd(&counts[0], a);
+    atomicAdd(&counts[1], b);
+  }
+}
+
+struct FeatAcc {
+  unsigned long long max_slice, max_fiber, sum_sq;
+  unsigned long long hist[SF_HIST_BINS];
+};
+
+// At every run end: run length = e - start + 1.
+__global__ void run_end_kernel(const uint64_t* __restrict__ key, uint64_t Is, uint64_t n,
+                               const uint32_t* __restrict__ sstart, const uint32_t* __restrict__ fstart,
+                               FeatAcc* __restrict__ acc) {
+  __shared__ unsigned long long h[SF_HIST_BINS];
+  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long ms = 0, mf = 0, sq = 0;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    const uint64_t k = key[e];
+    bool fend = true, send = true;
+    if (e + 1 < n) {
+      const uint64_t kn = key[e + 1];
+      fend = (k != kn);
+      send = (k / Is) != (kn / Is);
+    }
+    if (fend) {
+      const unsigned long long len = e - fstart[e] + 1;
+      mf = max(mf, len);
+    }
+    if (send) {
+      const unsigned long long len = e - sstart[e] + 1;
+      ms = max(ms, len);
+      sq += len * len;
+      atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
+    }
+  }
+  typedef cub::BlockReduce<unsigned long long, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long a = BR(tmp).Reduce(ms, cub::Max());
+  __syncthreads();
+  unsigned long long b = BR(tmp).Reduce(mf, cub::Max());
+  __syncthreads();
+  unsigned long long c = BR(tmp).Sum(sq);
+  if (threadIdx.x == 0) {
+    atomicMax(&acc->max_slice, a);
+    atomicMax(&acc->max_fiber, b);
+    atomicAdd(&acc->sum_sq, c);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x)
+    if (h[i]) atomicAdd(&acc->hist[i], h[i]);
+}
+
+struct MaxOp {
+  __device__ __forceinline__ uint32_t operator()(uint32_t a, uint32_t b) const { return a > b ? a : b; }
+};
+
+// Matricized sort of the whole tensor for `mode`. Returns sorted keys + positions.
+static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_out) {
+  const uint64_t n = t.nnz;
+  int s = 0;
+  for (int m = 0; m < t.nmodes; ++m)
+    if (m != mode) s = m;
+  const uint64_t Is = t.dims[s];
+  DevBuf k0(n * 8 + 16), k1(n * 8 + 16), p0(n * 4 + 16), p1(n * 4 + 16);
+  key_matricized_kernel<<<grid_for(n), 256, 0, t.stream>>>(t.ind[mode].as<uint32_t>(),
+                                                         t.ind[s].as<uint32_t>(), Is, n,
+                                                         k0.as<uint64_t>(), p0.as<uint32_t>());
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+  const int end_bit = std::max(1, bitlen(t.dims[mode] * Is - 1));
+  cub::DoubleBuffer<uint64_t> dk(k0.as<uint64_t>(), k1.as<uint64_t>());
+  cub::DoubleBuffer<uint32_t> dv(p0.as<uint32_t>(), p1.as<uint32_t>());
+  size_t temp = 0;
+  SF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, temp, dk, dv, (int64_t)n, 0, end_bit, t.stream));
+  DevBuf tmp(temp + 16);
+  SF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, temp, dk, dv, (int64_t)n, 0, end_bit, t.stream));
+  count_launch((uint64_t)((end_bit + 7) / 8) * 3);
+  if (dk.Current() == k0.as<uint64_t>()) keys_out = std::move(k0); else keys_out = std::move(k1);
+  if (dv.Current() == p0.as<uint32_t>()) pos_out = std::move(p0); else pos_out = std::move(p1);
+}
+
+static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_features_t* f) {
+  const uint64_t n = t.nnz;
+  int s = 0;
+  for (int m = 0; m < t.nmodes; ++m)
+    if (m != mode) s = m;
+  const uint64_t Is = t.dims[s];
+  memset(f, 0, sizeof(*f));
+  f->nnz = n;
+  f->dim = t.dims[mode];
+  f->nmodes = t.nmodes;
+  f->mode = mode;
+  f->secondary = s;
+  if (n > 0) {
+    DevBuf ss(n * 4 + 16), fs(n * 4 + 16), cnt(16), accb(sizeof(FeatAcc));
+    SF_CUDA(cudaMemsetAsync(cnt.p, 0, 16, t.stream));
+    SF_CUDA(cudaMemsetAsync(accb.p, 0, sizeof(FeatAcc), t.stream));
+    run_start_kernel<<<grid_for(n), 256, 0, t.stream>>>(keys, Is, n, ss.as<uint32_t>(), fs.as<uint32_t>(),
+                                                        cnt.as<unsigned long long>());
+    count_launch();
+    size_t temp = 0;
+    SF_CUDA(cub::DeviceScan::InclusiveScan(nullptr, temp, ss.as<uint32_t>(), ss.as<uint32_t>(), MaxOp(),
+                                           (int64_t)n, t.stream));
+    DevBuf tmp(temp + 16);
+    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, ss.as<uint32_t>(), ss.as<uint32_t>(), MaxOp(),
+                                           (int64_t)n, t.stream));
+    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, fs.as<uint32_t>(), fs.as<uint32_t>(), MaxOp(),
+                                           (int64_t)n, t.stream));
+    count_launch(4);
+    run_end_kernel<<<grid_for(n), 256, 0, t.stream>>>(keys, Is, n, ss.as<uint32_t>(), fs.as<uint32_t>(),
+                                                      accb.as<FeatAcc>());
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+    unsigned long long c[2];
+    FeatAcc a;
+    SF_CUDA(cudaMemcpyAsync(c, cnt.p, 16, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaMemcpyAsync(&a, accb.p, sizeof(FeatAcc), cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaStreamSynchronize(t.stream));
+    f->num_slices = c[0];
+    f->num_fibers = c[1];
+    f->max_nnz_per_slice = a.max_slice;
+    f->max_nnz_per_fiber = a.max_fiber;
+    f->sum_sq_nnz_per_slice = a.sum_sq;
+    for (int i = 0; i < SF_HIST_BINS; ++i) f->slice_hist[i] = a.hist[i];
+  }
+  f->slice_ratio = f->dim ? (double)f->num_slices / (double)f->dim : 0.0;
+  f->fiber_ratio = f->num_slices ? (double)f->num_fibers / (double)f->num_slices : 0.0;
+  f->avg_nnz_per_slice = f->num_slices ? (double)n / (double)f->num_slices : 0.0;
+  f->avg_nnz_per_fiber = f->num_fibers ? (double)n / (double)f->num_fibers : 0.0;
+  if (f->num_slices) {
+    double var = (double)f->sum_sq_nnz_per_slice / (double)f->num_slices -
+                 f->avg_nnz_per_slice * f->avg_nnz_per_slice;
+    f->std_nnz_per_slice = var > 0 ? sqrt(var) : 0.0;
+  }
+}
+
+void compute_features(Tensor& t, int mode, sf_features_t* out) {
+  if (!t.have_features[mode]) {
+    DevBuf keys, pos;
+    if (t.nnz) matricized_sort(t, mode, keys, pos);
+    features_from_sorted(t, mode, keys.as<uint64_t>(), &t.features[mode]);
+    t.have_features[mode] = true;
+  }
+  *out = t.features[mode];
+}
+
+// ---------------------------------------------------------------------------
+struct TileParams {
+  const uint32_t* ind[SF_MAX_MODES];
+  uint32_t block_rows[SF_MAX_MODES];
+  uint64_t ntiles[SF_MAX_MODES];
+  uint32_t staged_mask;
+  int nmodes;
+};
+
+__global__ void tile_key_kernel(TileParams tp, const uint32_t* __restrict__ pos, uint64_t n,
+                                uint64_t* __restrict__ tkey, uint32_t* __restrict__ tpos) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint32_t e = pos[k];
+    uint64_t t = 0;
+    for (int m = 0; m < tp.nmodes; ++m)
+      if (tp.staged_mask & (1u << m)) t = t * tp.ntiles[m] + tp.ind[m][e] / tp.block_rows[m];
+    tkey[k] = t;
+    tpos[k] = e;
+  }
+}
+
+struct GatherParams {
+  const uint32_t* src[SF_MAX_MODES];
+  uint32_t* dst[SF_MAX_MODES];
+  const float* vsrc;
+  float* vdst;
+  int nmodes;
+};
+
+__global__ void gather_kernel(GatherParams g, const uint32_t* __restrict__ perm, uint64_t n) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint32_t e = perm[k];
+    for (int m = 0; m < g.nmodes; ++m) g.dst[m][k] = g.src[m][e];
+    g.vdst[k] = g.vsrc[e];
+  }
+}
+
+// Chunk start flags: k starts a chunk iff (k - tile_start(k)) % C == 0.
+__global__ void tile_start_kernel(const uint64_t* __restrict__ tkey, uint64_t n, uint32_t* __restrict__ ts,
+                                  unsigned long long* __restrict__ ntiles) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long c = 0;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const bool st = (k == 0) || (tkey ? tkey[k] != tkey[k - 1] : false);
+    ts[k] = st ? (uint32_t)k : 0u;
+    c += st;
+  }
+  typedef cub::BlockReduce<unsigned long long, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  unsigned long long a = BR(tmp).Sum(c);
+  if (threadIdx.x == 0) atomicAdd(ntiles, a);
+}
+
+__global__ void chunk_flag_kernel(const uint32_t* __restrict__ ts, uint64_t n, uint32_t C,
+                                  uint32_t* __restrict__ flag) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride)
+    flag[k] = (((uint32_t)k - ts[k]) % C == 0u) ? 1u : 0u;
+}
+
+__global__ void chunk_scatter_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ excl,
+                                     const uint64_t* __restrict__ tkey, uint64_t n,
+                                     uint32_t* __restrict__ cbegin, uint64_t* __restrict__ ctile) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    if (flag[k]) {
+      const uint32_t j = excl[k];
+      cbegin[j] = (uint32_t)k;
+      ctile[j] = tkey ? tkey[k] : 0ull;
+    }
+  }
+}
+
+__global__ void set_u32_kernel(uint32_t* p, uint32_t v) { *p = v; }
+
+void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch) {
+  cudaEvent_t ev0, ev1;
+  SF_CUDA(cudaEventCreate(&ev0));
+  SF_CUDA(cudaEventCreate(&ev1));
+  SF_CUDA(cudaEventRecord(ev0, t.stream));
+  const int N = t.nmodes;
+  p.mode = mode;
+  p.rank = rank;
+  p.launch = launch;
+  const uint64_t n = t.nnz;
+  const uint64_t lo = (uint64_t)(((unsigned __int128)t.rank * n) / t.nranks);
+  const uint64_t hi = (uint64_t)(((unsigned __int128)(t.rank + 1) * n) / t.nranks);
+  const uint64_t nl = hi - lo;
+  p.nnz_local = nl;
+  if (nl >= (1ull << 32)) throw StatusError{SF_ERR_UNSUPPORTED, "shard nnz must be < 2^32"};
+
+  DevBuf keys, pos0;
+  if (n) matricized_sort(t, mode, keys, pos0);
+  if (!t.have_features[mode]) {
+    features_from_sorted(t, mode, keys.as<uint64_t>(), &t.features[mode]);
+    t.have_features[mode] = true;
+  }
+  p.feat = t.features[mode];
+
+  int s = 0;
+  for (int m = 0; m < N; ++m)
+    if (m != mode) s = m;
+  p.row_begin = p.row_end = 0;
+  if (nl) {
+    uint64_t kb, ke;
+    SF_CUDA(cudaMemcpyAsync(&kb, keys.as<uint64_t>() + lo, 8, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaMemcpyAsync(&ke, keys.as<uint64_t>() + hi - 1, 8, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaStreamSynchronize(t.stream));
+    p.row_begin = kb / t.dims[s];
+    p.row_end = ke / t.dims[s] + 1;
+  }
+  keys.release();
+
+  // Kernel order (positions into the raw COO).
+  const bool staged = (launch.kernel == SF_KERNEL_FRAG) && launch.staged_mask != 0;
+  DevBuf perm(nl * 4 + kPadBytes), tkeys;
+  if (nl) {
+    if (staged) {
+      TileParams tp{};
+      uint64_t total_tiles = 1;
+      for (int m = 0; m < N; ++m) {
+        tp.ind[m] = t.ind[m].as<uint32_t>();
+        if (launch.staged_mask & (1u << m)) {
+          tp.block_rows[m] = launch.block_rows[m];
+          tp.ntiles[m] = (t.dims[m] + launch.block_rows[m] - 1) / launch.block_rows[m];
+          total_tiles *= tp.ntiles[m];
+        }
+      }
+      tp.staged_mask = launch.staged_mask;
+      tp.nmodes = N;
+      DevBuf k0(nl * 8 + 16), k1(nl * 8 + 16), p1(nl * 4 + kPadBytes);
+      tile_key_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tp, pos0.as<uint32_t>() + lo, nl, k0.as<uint64_t>(),
+                                                         perm.as<uint32_t>());
+      count_launch();
+      SF_CUDA(cudaGetLastError());
+      pos0.release();
+      const int end_bit = std::max(1, bitlen(total_tiles - 1));
+      cub::DoubleBuffer<uint64_t> dk(k0.as<uint64_t>(), k1.as<uint64_t>());
+      cub::DoubleBuffer<uint32_t> dv(perm.as<uint32_t>(), p1.as<uint32_t>());
+      size_t temp = 0;
+      SF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, temp, dk, dv, (int64_t)nl, 0, end_bit, t.stream));
+      DevBuf tmp(temp + 16);
+      SF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, temp, dk, dv, (int64_t)nl, 0, end_bit, t.stream));
+      count_launch((uint64_t)((end_bit + 7) / 8) * 3);
+      if (dk.Current() == k0.as<uint64_t>()) tkeys = std::move(k0); else tkeys = std::move(k1);
+      if (dv.Current() != perm.as<uint32_t>()) perm = std::move(p1);
+    } else {
+      SF_CUDA(cudaMemcpyAsync(perm.p, pos0.as<uint32_t>() + lo, nl * 4, cudaMemcpyDeviceToDevice, t.stream));
+      pos0.release();
+    }
+  }
+
+  // Gather the kernel-order SoA arrays (padded for aligned bulk copies).
+  GatherParams g{};
+  for (int m = 0; m < N; ++m) {
+    p.ind[m].alloc(nl * 4 + kPadBytes);
+    SF_CUDA(cudaMemsetAsync(p.ind[m].p, 0, nl * 4 + kPadBytes, t.stream));
+    g.src[m] = t.ind[m].as<uint32_t>();
+    g.dst[m] = p.ind[m].as<uint32_t>();
+  }
+  p.val.alloc(nl * 4 + kPadBytes);
+  SF_CUDA(cudaMemsetAsync(p.val.p, 0, nl * 4 + kPadBytes, t.stream));
+  g.vsrc = t.val.as<float>();
+  g.vdst = p.val.as<float>();
+  g.nmodes = N;
+  if (nl) {
+    gather_kernel<<<grid_for(nl), 256, 0, t.stream>>>(g, perm.as<uint32_t>(), nl);
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+  }
+  p.perm = std::move(perm);
+
+  // Chunks.
+  p.num_chunks = 0;
+  p.num_tiles = 0;
+  if (nl) {
+    const uint32_t C = (uint32_t)std::max(1, launch.chunk_nnz);
+    DevBuf ts(nl * 4 + 16), flag(nl * 4 + 16), excl(nl * 4 + 16), cnt(16);
+    SF_CUDA(cudaMemsetAsync(cnt.p, 0, 16, t.stream));
+    const uint64_t* tk = staged ? tkeys.as<uint64_t>() : nullptr;
+    tile_start_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tk, nl, ts.as<uint32_t>(), cnt.as<unsigned long long>());
+    count_launch();
+    size_t temp = 0;
+    SF_CUDA(cub::DeviceScan::InclusiveScan(nullptr, temp, ts.as<uint32_t>(), ts.as<uint32_t>(), MaxOp(),
+                                           (int64_t)nl, t.stream));
+    size_t temp2 = 0;
+    SF_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, temp2, flag.as<uint32_t>(), excl.as<uint32_t>(),
+                                          (int64_t)nl, t.stream));
+    DevBuf tmp(std::max(temp, temp2) + 16);
+    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, ts.as<uint32_t>(), ts.as<uint32_t>(), MaxOp(),
+                                           (int64_t)nl, t.stream));
+    chunk_flag_kernel<<<grid_for(nl), 256, 0, t.stream>>>(ts.as<uint32_t>(), nl, C, flag.as<uint32_t>());
+    SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, temp2, flag.as<uint32_t>(), excl.as<uint32_t>(),
+                                          (int64_t)nl, t.stream));
+    count_launch(5);
+    uint32_t last_excl, last_flag;
+    unsigned long long ntiles;
+    SF_CUDA(cudaMemcpyAsync(&last_excl, excl.as<uint32_t>() + nl - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaMemcpyAsync(&last_flag, flag.as<uint32_t>() + nl - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaMemcpyAsync(&ntiles, cnt.p, 8, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaStreamSynchronize(t.stream));
+    p.num_chunks = (uint64_t)last_excl + last_flag;
+    p.num_tiles = ntiles;
+    p.chunk_begin.alloc((p.num_chunks + 1) * 4 + 16);
+    p.chunk_tile.alloc(p.num_chunks * 8 + 16);
+    chunk_scatter_kernel<<<grid_for(nl), 256, 0, t.stream>>>(flag.as<uint32_t>(), excl.as<uint32_t>(), tk, nl,
+                                                            p.chunk_begin.as<uint32_t>(),
+                                                            p.chunk_tile.as<uint64_t>());
+    set_u32_kernel<<<1, 1, 0, t.stream>>>(p.chunk_begin.as<uint32_t>() + p.num_chunks, (uint32_t)nl);
+    count_launch(2);
+    SF_CUDA(cudaGetLastError());
+  } else {
+    p.chunk_begin.alloc(16);
+    SF_CUDA(cudaMemsetAsync(p.chunk_begin.p, 0, 16, t.stream));
+  }
+  SF_CUDA(cudaEventRecord(ev1, t.stream));
+  SF_CUDA(cudaEventSynchronize(ev1));
+  float ms = 0;
+  SF_CUDA(cudaEventElapsedTime(&ms, ev0, ev1));
+  p.plan_ms = ms;
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+}
+
+}  // namespace sf

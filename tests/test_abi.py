@@ -1,0 +1,58 @@
+"""CPU-side checks of the C ABI boundary: the library loads without a GPU and
+exports every symbol include/scalfrag.h declares (no compute calls here)."""
+import ctypes
+import os
+import re
+import subprocess
+
+import paper_conf_cluster_linwds24_b200 as sf
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "scalfrag.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(sf_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_header_declares_the_north_star_calls():
+    d = _declared()
+    for name in ("sf_tensor_create", "sf_plan", "sf_mttkrp"):
+        assert name in d
+
+
+def test_library_exports_every_declared_symbol():
+    L = sf.lib()
+    out = subprocess.run(["nm", "-D", "--defined-only", sf._build.SO], capture_output=True, text=True).stdout
+    exported = {l.split()[-1] for l in out.splitlines() if " T " in l}
+    for name in _declared():
+        assert name in exported, name
+        assert hasattr(L, name)
+    assert set(sf.EXPORTED) == set(_declared())
+
+
+def test_status_strings_and_version():
+    L = sf.lib()
+    for code, name in sf.STATUS.items():
+        assert L.sf_status_string(code).decode() == name
+    assert "sm_100a" in sf.version()
+    assert sf.kernel_launches() == 0  # nothing launched on a CPU box
+
+
+def test_struct_layouts_match_header():
+    # sizes implied by include/scalfrag.h on LP64
+    assert ctypes.sizeof(sf.Launch) == 4 * 5 + 4 * 8
+    assert ctypes.sizeof(sf.Features) == 8 * 7 + 8 * 40 + 4 * 4 + 8 * 5
+    assert ctypes.sizeof(sf.PlanInfo) == ctypes.sizeof(sf.Features) + ctypes.sizeof(sf.Launch) + 4 + 8 * 7
+
+
+def test_no_oracle_in_product_path():
+    """The product package must not import or link anything under oracle/."""
+    pkg = os.path.join(ROOT, "paper_conf_cluster_linwds24_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
+                txt = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt, f
+                assert "oracle.c" not in txt and "liboracle" not in txt, f

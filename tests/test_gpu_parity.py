@@ -1,0 +1,215 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Floating point: max |Y_gpu - Y| / S <= 1e-4 per element (north_star), S the
+|.|-scale; rows without contributions must be exactly 0.  Exact-integer data
+(values {1..4}, factors {-2..2}, all partial sums < 2^24) must match bitwise.
+Integer preprocessing (perm, chunks, features) must match oracle/plan.py ==.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+import paper_conf_cluster_linwds24_b200 as sf
+from oracle import plan as oplan
+from tests import gpu_util as G
+
+pytestmark = pytest.mark.gpu
+
+FRAG, COO = sf.KERNEL_FRAG, sf.KERNEL_COO
+
+
+def _cfg_data(name, val_kind="unit", fac_kind="unit"):
+    cfg = synth.CONFIGS[name]
+    inds, vals = synth.config_tensor(cfg, val_kind=val_kind)
+    facs = synth.gen_factors(cfg.dims, cfg.rank, cfg.fseed, fac_kind)
+    return cfg, inds, vals, facs
+
+
+@pytest.mark.parametrize("name", ["tiny", "tiny_skew"])
+def test_configs0_all_modes_auto(cuda_device, name):
+    cfg, inds, vals, facs = _cfg_data(name)
+    Y, info = G.run(cfg.dims, inds, vals, facs, cfg.rank)
+    for n in range(cfg.nmodes):
+        G.assert_parity(Y[n], cfg.dims, inds, vals, facs, cfg.rank, n)
+
+
+def _launches(dims, n):
+    others = [m for m in range(len(dims)) if m != n]
+    yield sf.Launch.make(kernel=COO)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=1024, block_threads=256, staged={})
+    # stage every gathered mode in small blocks: many tiles, ragged last block
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=128, staged={m: max(1, dims[m] // 3 + 1) for m in others})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=256, block_threads=1024, staged={others[0]: 7})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=4096, ctas_per_sm=1, staged={others[-1]: dims[others[-1]]})
+
+
+@pytest.mark.parametrize("name", ["tiny", "tiny_skew"])
+def test_launch_variants(cuda_device, name):
+    cfg, inds, vals, facs = _cfg_data(name, "signed", "signed")
+    for n in range(cfg.nmodes):
+        for L in _launches(cfg.dims, n):
+            try:
+                Y, _ = G.run(cfg.dims, inds, vals, facs, cfg.rank, modes=[n], launch=L)
+            except sf.SfError as e:
+                raise AssertionError(f"mode {n} launch {L.as_dict()}: {e}")
+            G.assert_parity(Y[n], cfg.dims, inds, vals, facs, cfg.rank, n)
+
+
+@pytest.mark.parametrize("R", [16, 32, 64, 1, 7, 12])
+@pytest.mark.parametrize("dims", [(100, 80, 60), (300, 200), (10, 12, 14, 16), (5, 6, 4, 3, 7)])
+def test_ranks_and_orders(cuda_device, R, dims):
+    nnz = 3001  # ragged
+    inds, vals = synth.gen_coo(dims, nnz, 99, zipf=(0.8,) * len(dims), val_kind="signed")
+    facs = synth.gen_factors(dims, R, 77, "signed")
+    for staged in (False, True):
+        def L(n):
+            if not staged:
+                return sf.Launch.make(kernel=FRAG, chunk_nnz=100)
+            return sf.Launch.make(kernel=FRAG, chunk_nnz=100,
+                                  staged={m: max(1, dims[m] // 2) for m in range(len(dims)) if m != n})
+        Y, _ = G.run(dims, inds, vals, facs, R, launch=L)
+        for n in range(len(dims)):
+            G.assert_parity(Y[n], dims, inds, vals, facs, R, n)
+
+
+def test_exact_integers_bitwise(cuda_device):
+    dims, R = (200, 150, 170), 32
+    inds, vals = synth.gen_coo(dims, 20000, 5, zipf=(1.0, 1.0, 1.0), val_kind="int")
+    facs = synth.gen_factors(dims, R, 6, "int")
+    for n in range(3):
+        Y, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
+        assert np.max(S) < 2 ** 24
+        for L in _launches(dims, n):
+            Yg, _ = G.run(dims, inds, vals, facs, R, modes=[n], launch=L)
+            assert np.array_equal(Yg[n].astype(np.float64), Y), L.as_dict()
+
+
+def test_plan_bit_exact_vs_oracle(cuda_device):
+    dims = (300, 41, 530)
+    inds, vals = synth.gen_coo(dims, 25000, 8, zipf=(1.0, 0.5, 0.8))
+    facs = synth.gen_factors(dims, 16, 9)
+    ti, tv = G.dev_inds(inds), G.dev_f(vals)
+    with sf.Tensor(dims, ti, tv) as t:
+        for n in range(3):
+            f = t.features(n)
+            of = oplan.features(dims, inds, n)
+            for k in ("num_slices", "num_fibers", "max_nnz_per_slice", "max_nnz_per_fiber",
+                      "sum_sq_nnz_per_slice", "secondary"):
+                assert f[k] == of[k], k
+            assert f["slice_hist"] == list(of["slice_hist"])
+            others = [m for m in range(3) if m != n]
+            for staged in ({}, {others[0]: 13}, {others[0]: 40, others[1]: 7}):
+                L = sf.Launch.make(kernel=FRAG, chunk_nnz=100, staged=staged)
+                t.set_launch(n, 16, L)
+                perm, chunks = t.plan_export(n, 16)
+                ref = oplan.plan_order(dims, inds, n, tuple(sorted(staged)), staged)
+                assert np.array_equal(perm.astype(np.int64), ref)
+                tiles = oplan.tile_ids(dims, inds, tuple(sorted(staged)), staged, sel=ref)
+                ref_chunks = oplan.chunks(tiles, 100)
+                assert np.array_equal(chunks.astype(np.int64), ref_chunks)
+                info = t.plan_info(n, 16)
+                assert info["num_tiles"] == len(np.unique(tiles))
+
+
+def test_shards_emulated_on_one_gpu(cuda_device):
+    """§8(e): P shards of the matricized order; their outputs sum to the 1-GPU result
+    (exact on integer data); each shard touches only its row range."""
+    dims, R = (120, 90, 70), 16
+    inds, vals = synth.gen_coo(dims, 15000, 21, zipf=(1.2, 0.5, 0.5), val_kind="int")
+    facs = synth.gen_factors(dims, R, 22, "int")
+    for n in range(3):
+        Yfull, _ = oracle.mttkrp(dims, inds, vals, facs, R, n)
+        for P in (2, 3, 8):
+            acc = np.zeros_like(Yfull)
+            perm0 = oplan.matricized_order(dims, inds, n)
+            for p in range(P):
+                Y, info = G.run(dims, inds, vals, facs, R, modes=[n], shard=(P, p))
+                lo, hi = oplan.shard_range(len(vals), P, p)
+                rows = inds[n][perm0[lo:hi]]
+                assert info[n]["nnz_local"] == hi - lo
+                if hi > lo:
+                    assert info[n]["row_begin"] == rows.min() and info[n]["row_end"] == rows.max() + 1
+                outside = np.ones(dims[n], bool)
+                outside[info[n]["row_begin"]:info[n]["row_end"]] = False
+                assert not Y[n][outside].any()
+                acc += Y[n]
+            assert np.array_equal(acc, Yfull)
+
+
+def test_host_inputs_pageable_and_pinned(cuda_device):
+    cfg, inds, vals, facs = _cfg_data("tiny_skew")
+    Y, _ = G.run(cfg.dims, inds, vals, facs, cfg.rank, device_input=False)
+    for n in range(3):
+        G.assert_parity(Y[n], cfg.dims, inds, vals, facs, cfg.rank, n)
+    # pinned torch host tensors, many segments / streams
+    ti = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    tv = torch.from_numpy(vals).pin_memory()
+    tf = [G.dev_f(f) for f in facs]
+    with sf.Tensor(cfg.dims, ti, tv, segments=7, streams=3) as t:
+        for n in range(3):
+            t.plan(n, cfg.rank)
+            y = torch.empty((cfg.dims[n], cfg.rank), device="cuda:0")
+            t.mttkrp(n, tf, y)
+            torch.cuda.synchronize()
+            G.assert_parity(y.cpu().numpy(), cfg.dims, inds, vals, facs, cfg.rank, n)
+
+
+@pytest.mark.parametrize("segments,streams", [(1, 1), (4, 4), (13, 3)])
+def test_streamed_one_shot(cuda_device, segments, streams):
+    cfg, inds, vals, facs = _cfg_data("tiny_skew", "signed", "signed")
+    tf = [G.dev_f(f) for f in facs]
+    for n in range(3):
+        y = torch.full((cfg.dims[n], cfg.rank), float("nan"), device="cuda:0")
+        sf.mttkrp_streamed(cfg.dims, inds, vals, tf, n, y, segments, streams)
+        G.assert_parity(y.cpu().numpy(), cfg.dims, inds, vals, facs, cfg.rank, n)
+
+
+def test_edge_cases(cuda_device):
+    dims, R = (10, 9, 8), 16
+    facs = synth.gen_factors(dims, R, 1)
+    tf = [G.dev_f(f) for f in facs]
+    # empty tensor -> Y == 0
+    e = [np.zeros(0, np.uint32)] * 3
+    with sf.Tensor(dims, e, np.zeros(0, np.float32)) as t:
+        t.plan(0, R)
+        y = torch.full((10, R), 7.0, device="cuda:0")
+        t.mttkrp(0, tf, y)
+        torch.cuda.synchronize()
+        assert not y.any()
+    # one nonzero
+    one = [np.array([3], np.uint32), np.array([8], np.uint32), np.array([7], np.uint32)]
+    Y, _ = G.run(dims, one, np.array([0.5], np.float32), facs, R)
+    for n in range(3):
+        G.assert_parity(Y[n], dims, one, np.array([0.5], np.float32), facs, R, n)
+    # out-of-range index is rejected at create
+    bad = [np.array([3], np.uint32), np.array([9], np.uint32), np.array([0], np.uint32)]
+    with pytest.raises(sf.SfError) as ei:
+        sf.Tensor(dims, G.dev_inds(bad), G.dev_f(np.ones(1, np.float32)))
+    assert ei.value.status == 2
+    with pytest.raises(sf.SfError) as ei:
+        sf.Tensor(dims, bad, np.ones(1, np.float32))
+    assert ei.value.status == 2
+    # mttkrp before plan
+    with sf.Tensor(dims, one, np.ones(1, np.float32)) as t:
+        with pytest.raises(sf.SfError) as ei:
+            t.mttkrp(0, tf, torch.empty((10, R), device="cuda:0"))
+        assert ei.value.status == 4
+        with pytest.raises(sf.SfError):
+            t.plan(3, R)  # bad mode
+    # a single heavy row + a single heavy fiber (atomic chains across chunks)
+    n = 50000
+    heavy = [np.full(n, 2, np.uint32), np.full(n, 4, np.uint32), np.arange(n, dtype=np.uint32) % 8]
+    v = synth.gen_coo((8,), n, 3)[1]
+    Y, _ = G.run(dims, heavy, v, facs, R, launch=sf.Launch.make(kernel=FRAG, chunk_nnz=64))
+    for m in range(3):
+        G.assert_parity(Y[m], dims, heavy, v, facs, R, m)
+
+
+def test_kernel_launch_counter(cuda_device):
+    before = sf.kernel_launches()
+    cfg, inds, vals, facs = _cfg_data("tiny")
+    G.run(cfg.dims, inds, vals, facs, cfg.rank, modes=[0])
+    assert sf.kernel_launches() > before
