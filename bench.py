@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""ScalFrag-on-B200 benchmark: mode-n sparse MTTKRP (Eq. (4)).
+
+Contract (one JSON line on rank 0):
+  python bench.py [--gpus N --steps K --warmup W] [--config nell2] [--impl ours|reference]
+
+* workload: BASELINE.json configs[1] (nell-2-shaped 12092x9184x28818, nnz=76,879,419,
+  R=32), synthetic, seeded (synth/), the largest config whose metric is quoted at 1 GPU.
+* step: one sf_mttkrp per mode over all N modes (a CP-ALS sweep's MTTKRPs) on the
+  planned, HBM-resident tensor; for N>1 each rank owns a contiguous shard of every
+  mode's matricized order (§8(e)) and the step includes the boundary-row exchange
+  (NCCL all_gather + sf_rows_add).  Planning (sort/tile/features/select) is a
+  one-time cost per (mode, rank), reported as plan_ms, and is inside `e2e`.
+* value: GFLOP/s = sum_modes N*nnz*R / step time (flop convention N*nnz*R,
+  DESIGN.md reading R14), max over ranks, CUDA events on the launching stream.
+* e2e: the same metric through the public C ABI from PINNED HOST buffers:
+  sf_tensor_create (segmented H2D + validate) + factor H2D + sf_plan (all modes)
+  + sf_mttkrp (all modes) + D2H of every Y, every step.
+* roofline: dominant kernel = frag_kernel; algorithmic bytes per launch =
+  4(N+1)*nnz + 4R*sum_m I_m, over its event-timed duration.
+* cpu_baseline: the oracle (oracle/oracle.c, fp64, 1 thread) on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "src": "fallback (B200_PROFILING.md)"}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json)"}
+    return PEAKS_FALLBACK
+
+
+# ---------------------------------------------------------------------------
+# clocks sampler (nvidia-smi during the timed region)
+# ---------------------------------------------------------------------------
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", str(self.index)],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx.append(float(parts[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+def bytes_model(cfg):
+    N = cfg.nmodes
+    return 4 * (N + 1) * cfg.nnz + 4 * cfg.rank * sum(cfg.dims)
+
+
+def flops_per_mode(cfg, nnz=None):
+    return cfg.nmodes * (cfg.nnz if nnz is None else nnz) * cfg.rank
+
+
+def cpu_oracle_sample(cfg, inds, vals, facs, sample_nnz):
+    """Time the oracle (as it stands, 1 thread) on the first `sample_nnz` nonzeros, all modes."""
+    import oracle
+    n = min(sample_nnz, len(vals))
+    si = [a[:n] for a in inds]
+    sv = vals[:n]
+    oracle.lib()
+    t0 = time.perf_counter()
+    for m in range(cfg.nmodes):
+        oracle.mttkrp(cfg.dims, si, sv, facs, cfg.rank, m, with_scale=False)
+    dt = time.perf_counter() - t0
+    return n, dt
+
+
+def run_reference(args, cfg, rank, world):
+    """--impl reference: the oracle (the tier's reference arm) on host cores."""
+    if rank != 0:
+        return
+    per_step = args.ref_sample
+    inds, vals = synth.config_tensor(cfg, 0, per_step)
+    facs = synth.config_factors(cfg)
+    import oracle
+    oracle.lib()
+    for _ in range(args.warmup):
+        for m in range(cfg.nmodes):
+            oracle.mttkrp(cfg.dims, inds, vals, facs, cfg.rank, m, with_scale=False)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for m in range(cfg.nmodes):
+            oracle.mttkrp(cfg.dims, inds, vals, facs, cfg.rank, m, with_scale=False)
+    dt = time.perf_counter() - t0
+    flops = flops_per_mode(cfg, per_step) * cfg.nmodes * args.steps
+    v = flops / dt / 1e9
+    line = {"metric": "MTTKRP GFLOP/s (all modes, N*nnz*R convention)", "value": v, "unit": "GFLOP/s",
+            "impl": "reference", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": workload_config(cfg, world),
+            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+                             "sample": f"first {per_step} nonzeros of the workload per step, all {cfg.nmodes} modes"},
+            "e2e": {"value": v, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(cfg, world):
+    return {"workload": f"{cfg.name}: {cfg.note}", "dims": list(cfg.dims), "nnz": cfg.nnz,
+            "rank": cfg.rank, "zipf": list(cfg.zipf), "modes": cfg.nmodes,
+            "parallelism": f"nnz-shard{world}" if world > 1 else "single",
+            "l2": "inputs larger than L2: each mode streams its own 4(N+1)*nnz-byte sorted copy "
+                  "(>1 GB) per launch; factors are gathered through L2 as the method intends",
+            "step": "one sf_mttkrp per mode over all modes (+ boundary exchange at N>1)"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="nell2")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-sample", type=int, default=8_000_000)
+    ap.add_argument("--ref-sample", type=int, default=1_000_000)
+    ap.add_argument("--launch-json", default=None, help="override launches: {mode: launch dict}")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    cfg = synth.CONFIGS[args.config]
+
+    if args.impl == "reference":
+        run_reference(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_linwds24_b200 as sf
+    from paper_conf_cluster_linwds24_b200 import dist as sfdist
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    N, R = cfg.nmodes, cfg.rank
+
+    # ---- synthetic input (every rank holds the full raw COO, §8(e) v1) ----
+    t_gen = time.perf_counter()
+    inds, vals = synth.config_tensor(cfg)
+    facs = synth.config_factors(cfg)
+    t_gen = time.perf_counter() - t_gen
+    h_inds = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    h_vals = torch.from_numpy(vals).pin_memory()
+    h_facs = [torch.from_numpy(f).pin_memory() for f in facs]
+    d_facs = [f.to(dev) for f in h_facs]
+    stream = torch.cuda.Stream(device=dev)
+
+    # ---- resident tensor + plans ----
+    T = sf.Tensor(cfg.dims, h_inds, h_vals)
+    if world > 1:
+        T.set_shard(world, rank)
+    overrides = json.loads(args.launch_json) if args.launch_json else {}
+    plan_ms = {}
+    for n in range(N):
+        if str(n) in overrides:
+            T.set_launch(n, R, sf.Launch.make(**overrides[str(n)]))
+        else:
+            T.plan(n, R)
+        plan_ms[n] = T.plan_info(n, R)["plan_ms"]
+    infos = {n: T.plan_info(n, R) for n in range(N)}
+    outs = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
+    exch = sfdist.BoundaryExchange(world, rank, R, dev) if world > 1 else None
+
+    def step(ev=None):
+        for n in range(N):
+            if ev is not None:
+                ev[n][0].record(stream)
+            T.mttkrp(n, d_facs, outs[n], stream=stream)
+            if ev is not None:
+                ev[n][1].record(stream)
+            if exch is not None:
+                exch.combine(outs[n], infos[n]["row_begin"], infos[n]["row_end"], stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+
+    evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in range(N)]
+           for _ in range(args.steps)]
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    clk = ClockSampler(local_rank)
+    clk.start()
+    time.sleep(0.3)
+    launches0 = sf.kernel_launches()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    t0.record(stream)
+    for k in range(args.steps):
+        step(evs[k])
+    t1.record(stream)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    launches = sf.kernel_launches() - launches0
+    clocks = clk.stop()
+    ms_total = t0.elapsed_time(t1)
+    if world > 1:
+        tt = torch.tensor([ms_total], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms_total = float(tt.item())
+    ms_step = ms_total / args.steps
+    flops_step = flops_per_mode(cfg) * N
+    value = flops_step / (ms_step * 1e-3) / 1e9
+    per_mode_ms = {n: statistics.mean(evs[k][n][0].elapsed_time(evs[k][n][1]) for k in range(args.steps))
+                   for n in range(N)}
+    bm = bytes_model(cfg)
+    peaks = load_peaks()
+    mean_launch_ms = statistics.mean(per_mode_ms.values())
+    # at N>1 each launch processes this rank's shard: bytes of its nonzeros + all factors
+    nnz_local = statistics.mean(infos[n]["nnz_local"] for n in range(N))
+    bytes_launch = 4 * (N + 1) * nnz_local + 4 * R * sum(cfg.dims)
+    achieved = bytes_launch / (mean_launch_ms * 1e-3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            d = json.load(open(prof))
+            if d.get("config") == cfg.name and world == 1:
+                traffic = d.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    # ---- e2e through the public API from pinned host buffers ----
+    e2e = None
+    if not args.no_e2e:
+        h_out = [torch.empty((cfg.dims[n], R), dtype=torch.float32).pin_memory() for n in range(N)]
+        h2d = sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4 + sum(f.numel() * 4 for f in h_facs)
+        d2h = sum(o.numel() * 4 for o in h_out)
+
+        def e2e_step():
+            with sf.Tensor(cfg.dims, h_inds, h_vals) as T2:
+                if world > 1:
+                    T2.set_shard(world, rank)
+                df = [f.to(dev, non_blocking=True) for f in h_facs]
+                for n in range(N):
+                    if str(n) in overrides:
+                        T2.set_launch(n, R, sf.Launch.make(**overrides[str(n)]))
+                    else:
+                        T2.plan(n, R)
+                inf = {n: T2.plan_info(n, R) for n in range(N)}
+                for n in range(N):
+                    o = torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev)
+                    T2.mttkrp(n, df, o, stream=stream)
+                    if exch is not None:
+                        exch.combine(o, inf[n]["row_begin"], inf[n]["row_end"], stream)
+                    with torch.cuda.stream(stream):
+                        h_out[n].copy_(o, non_blocking=True)
+                torch.cuda.synchronize(dev)
+
+        e2e_step()  # warm-up
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        s0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        torch.cuda.synchronize(dev)
+        e2e_ms = (time.perf_counter() - s0) / args.e2e_steps * 1e3
+        if world > 1:
+            tt = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            e2e_ms = float(tt.item())
+        e2e = {"value": flops_step / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms,
+               "steps": args.e2e_steps,
+               "includes": "sf_tensor_create(pinned host COO, segmented H2D+validate) + factor H2D + "
+                           "sf_plan x N + sf_mttkrp x N + D2H of every Y (host wall clock)"}
+
+    # ---- CPU oracle baseline (rank 0, N=1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        n_s, dt = cpu_oracle_sample(cfg, inds, vals, facs, args.cpu_sample)
+        cpu = {"value": flops_per_mode(cfg, n_s) * N / dt / 1e9, "unit": "GFLOP/s", "cores": 1,
+               "kind": "oracle", "sample": f"first {n_s} of {cfg.nnz} nonzeros, all {N} modes, "
+                                            f"fp64 single thread, {dt:.1f} s"}
+
+    if rank == 0:
+        line = {
+            "metric": "MTTKRP GFLOP/s (all modes, N*nnz*R convention)",
+            "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": workload_config(cfg, world),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                         "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                         "kernel": "frag_kernel", "peak_src": peaks["src"],
+                         "bytes_per_launch": bytes_launch, "launch_ms": mean_launch_ms},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches),
+            "clocks": clocks,
+            "per_mode": {str(n): {"ms": per_mode_ms[n], "gflops": flops_per_mode(cfg) / per_mode_ms[n] / 1e6,
+                                  "eff_gbs": bm / (per_mode_ms[n] * 1e-3) / 1e9, "plan_ms": plan_ms[n],
+                                  "launch": infos[n]["launch"], "num_tiles": infos[n]["num_tiles"],
+                                  "num_chunks": infos[n]["num_chunks"]}
+                         for n in range(N)},
+            "gen_s": t_gen,
+        }
+        print(json.dumps(line), flush=True)
+    T.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -155,6 +155,15 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
                              const float* const* factors, int rank, int mode, float* out,
                              int segments, int streams);
 
+/* Boundary-row exchange helper for multi-GPU row shards (§8(e)): for k < count with
+ * rows[k] >= 0 (device int64 array):
+ *   op 0 (PACK): buf[k, :] = Y[rows[k], :]      op 1 (ADD): Y[rows[k], :] += buf[k, :]
+ *   op 2 (ZERO): Y[rows[k], :] = 0
+ * Y, rows, buf are device pointers; Y is I x rank row-major.  Stream-ordered. */
+typedef enum { SF_ROWS_PACK = 0, SF_ROWS_ADD = 1, SF_ROWS_ZERO = 2 } sf_rows_op_t;
+sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int count, int op,
+                     void* stream);
+
 /* ---- diagnostics -------------------------------------------------------- */
 const char* sf_status_string(sf_status s);
 const char* sf_last_error(void);

@@ -93,7 +93,7 @@ class PlanInfo(ctypes.Structure):
 EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
             "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
             "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
-            "sf_kernel_launches", "sf_version"]
+            "sf_kernel_launches", "sf_version", "sf_rows_op"]
 
 
 def lib(build_if_missing: bool = True):
@@ -119,9 +119,10 @@ def lib(build_if_missing: bool = True):
             L.sf_plan_export.argtypes = [P, I, I, P, P]
             L.sf_mttkrp.argtypes = [P, I, P, I, P, P]
             L.sf_mttkrp_streamed.argtypes = [I, P, U64, P, P, P, I, I, P, I, I]
+            L.sf_rows_op.argtypes = [P, I, P, P, I, I, P]
             for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
                        "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
-                       "sf_mttkrp", "sf_mttkrp_streamed"]:
+                       "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op"]:
                 getattr(L, fn).restype = ctypes.c_int
             L.sf_status_string.argtypes = [I]
             L.sf_status_string.restype = ctypes.c_char_p
@@ -252,3 +253,12 @@ def mttkrp_streamed(dims, inds, vals, factors, mode, out, segments=8, streams=4)
     _check(lib().sf_mttkrp_streamed(N, d, int(len(vals)), ip, _ptr(vals), fp, int(out.shape[1]), int(mode),
                                     _ptr(out), int(segments), int(streams)))
     return out
+
+
+ROWS_PACK, ROWS_ADD, ROWS_ZERO = 0, 1, 2
+
+
+def rows_op(Y, rows, buf, op, stream=None):
+    """Boundary-row pack / add / zero on device tensors (sf_rows_op)."""
+    _check(lib().sf_rows_op(_ptr(Y), int(Y.shape[1]), _ptr(rows), _ptr(buf), int(rows.numel()), int(op),
+                            _stream_handle(stream)))

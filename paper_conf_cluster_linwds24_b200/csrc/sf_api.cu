@@ -446,6 +446,17 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
   });
 }
 
+sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int count, int op,
+                     void* stream) {
+  return guard([&]() -> sf_status {
+    if (count < 0 || rank < 1 || op < 0 || op > 2) throw StatusError{SF_ERR_INVALID_ARG, "bad rows_op args"};
+    if (count == 0) return SF_OK;
+    if (!Y || !rows || (op != 2 && !buf)) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    launch_rows_op(Y, rank, rows, buf, count, op, static_cast<cudaStream_t>(stream));
+    return SF_OK;
+  });
+}
+
 const char* sf_status_string(sf_status s) {
   switch (s) {
     case SF_OK: return "SF_OK";

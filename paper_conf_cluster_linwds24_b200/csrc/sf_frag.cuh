@@ -1,0 +1,345 @@
+// sf_frag.cuh - the fragment MTTKRP kernel template (§8(a) A6/A7).
+//
+// Y(i_n(e), :) += v_e * prod_{m != n} A_m(i_m(e), :)   (Eq. (4))
+//
+// Persistent CTAs walk the chunks ("segments") of the planned order
+// (tile, i_n, i_s, pos).  Per chunk:
+//   * one elected thread issues N+1 one-dimensional TMA bulk copies
+//     (cp.async.bulk.shared::cluster.global.mbarrier) of the chunk's SoA fields into a
+//     double-buffered shared-memory stage; the next chunk streams in while this one is
+//     computed;
+//   * when the tile changes, the factor blocks of the S "staged" modes are bulk-copied
+//     into shared memory (the paper's "times_mat in shared memory");
+//   * lane groups of LPN = R/4 lanes (one float4 rank slice per lane) walk contiguous
+//     stretches of the chunk; a group accumulates in registers while i_n is unchanged
+//     and flushes one red.global.add.v4.f32 per run edge.
+// Template parameters: N modes, rank R, S staged gathered modes.  Gathered "slots"
+// 0..S-1 are the staged modes (ascending mode id; gathered from shared memory),
+// slots S..N-2 the others (gathered from global memory through L1/L2).  Slot order
+// only changes the order of the fp32 products, not which terms are summed.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "sf_internal.h"
+
+namespace sf {
+
+struct FragParams {
+  const uint32_t* ind[SF_MAX_MODES];  // kernel-order indices of every mode
+  const float* val;
+  const float* fac[SF_MAX_MODES];     // by mode
+  float* out;
+  const uint32_t* chunk_begin;        // num_chunks + 1
+  const uint64_t* chunk_tile;         // num_chunks
+  uint32_t num_chunks;
+  uint32_t nnz;
+  int mode;
+  int slot_mode[SF_MAX_MODES];        // gathered slot -> mode (staged slots first)
+  uint32_t block_rows[SF_MAX_MODES];  // per staged slot
+  uint32_t ntiles[SF_MAX_MODES];      // per staged slot
+  uint32_t dims[SF_MAX_MODES];        // per mode
+  uint32_t fac_off[SF_MAX_MODES];     // per staged slot: float offset of its block in smem
+  uint32_t stage_words;               // words per field per pipeline stage
+};
+
+constexpr int kFragStages = 2;
+constexpr int kFragUnroll = 4;
+
+namespace detail {
+
+__device__ __forceinline__ void red_add_v4_nomem(float* addr, const float4& v) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(addr), "f"(v.x), "f"(v.y), "f"(v.z),
+               "f"(v.w));
+}
+
+__device__ __forceinline__ uint32_t su32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ float4 lds128(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(addr));
+  return v;
+}
+
+__device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count));
+}
+__device__ __forceinline__ void fence_barrier_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(dst)),
+      "l"(src), "r"(bytes), "r"(su32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  const uint32_t a = su32(bar);
+  do {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0,1,0,p; }"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+
+}  // namespace detail
+
+template <int N, int R, int S>
+__global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
+  using namespace detail;
+  constexpr int LPN = R / 4;  // lanes per nonzero
+  constexpr int G = N - 1;    // gathered slots
+  constexpr int RB = R * 4;   // bytes per factor row
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);  // [kFragStages] stream + [1] factors
+  float* stage_base = reinterpret_cast<float*>(smem_raw + 128);
+  float* fac_smem = stage_base + (size_t)kFragStages * (N + 1) * p.stage_words;
+
+  const int tid = threadIdx.x;
+  const int sub = tid % LPN;
+  const int group = tid / LPN;
+  const int ngroups = blockDim.x / LPN;
+
+  // This CTA's chunks: those whose begin lies in [c*nnz/G, (c+1)*nnz/G).
+  const uint64_t grid = gridDim.x;
+  auto lower = [&](uint64_t target) {
+    uint32_t lo = 0, hi = p.num_chunks;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if ((uint64_t)__ldg(p.chunk_begin + mid) < target) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+  };
+  const uint32_t j0 = lower(((uint64_t)blockIdx.x * p.nnz) / grid);
+  const uint32_t j1 = lower(((uint64_t)(blockIdx.x + 1) * p.nnz) / grid);
+  if (j0 >= j1) return;
+
+  if (tid == 0) {
+    for (int s = 0; s <= kFragStages; ++s) mbar_init(&bars[s], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+
+  auto issue = [&](uint32_t j, int s) {
+    const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
+    const uint32_t start = b & ~3u;
+    const uint32_t bytes = (((e - start) + 3u) & ~3u) * 4u;
+    float* dst = stage_base + (size_t)s * (N + 1) * p.stage_words;
+    mbar_expect_tx(&bars[s], bytes * (N + 1));
+#pragma unroll
+    for (int m = 0; m < N; ++m) bulk_g2s(dst + (size_t)m * p.stage_words, p.ind[m] + start, bytes, &bars[s]);
+    bulk_g2s(dst + (size_t)N * p.stage_words, p.val + start, bytes, &bars[s]);
+  };
+  if (tid == 0)
+    for (int s = 0; s < kFragStages && j0 + s < j1; ++s) issue(j0 + s, s);
+
+  // Per-slot gather bases.  Staged slots: shared address of row 0 of the *virtual*
+  // full factor (block base minus tile_row0 * RB), so addr = base + idx * RB.
+  const float4* sbase[S > 0 ? S : 1];
+  const float4* gbase[G - S > 0 ? G - S : 1];
+#pragma unroll
+  for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]) + sub;
+  uint64_t cur_tile = ~0ull;
+  uint32_t fac_phase = 0;
+
+  for (uint32_t j = j0; j < j1; ++j) {
+    const int s = (int)((j - j0) % kFragStages);
+    const uint32_t parity = ((j - j0) / kFragStages) & 1u;
+
+    if constexpr (S > 0) {
+      const uint64_t tile = __ldg(p.chunk_tile + j);
+      if (tile != cur_tile) {
+        cur_tile = tile;
+        uint64_t t = tile;
+        uint32_t row0[S];
+#pragma unroll
+        for (int q = S - 1; q >= 0; --q) {
+          const uint32_t qq = (uint32_t)(t % p.ntiles[q]);
+          t /= p.ntiles[q];
+          row0[q] = qq * p.block_rows[q];
+        }
+        __syncthreads();  // everyone is done with the previous blocks
+        if (tid == 0) {
+          uint32_t total = 0;
+#pragma unroll
+          for (int q = 0; q < S; ++q) total += min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]) * RB;
+          mbar_expect_tx(&bars[kFragStages], total);
+#pragma unroll
+          for (int q = 0; q < S; ++q) {
+            const uint32_t rows = min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]);
+            bulk_g2s(fac_smem + p.fac_off[q], p.fac[p.slot_mode[q]] + (size_t)row0[q] * R, rows * RB,
+                     &bars[kFragStages]);
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < S; ++q)
+          sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) + sub -
+                     (ptrdiff_t)row0[q] * LPN;
+        mbar_wait(&bars[kFragStages], fac_phase);
+        fac_phase ^= 1u;
+      }
+    }
+
+    mbar_wait(&bars[s], parity);
+
+    const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
+    const uint32_t n = e - b;
+    const float* sb = stage_base + (size_t)s * (N + 1) * p.stage_words + (b - (b & ~3u));
+    uint32_t L = (n + ngroups - 1) / ngroups;
+    // the 32/LPN groups of a warp read word g*L + k: distinct banks iff gcd(L,32) <= LPN
+    if (LPN < 32)
+      while (L % (2u * LPN) == 0u) ++L;
+    const uint32_t k0 = group * L;
+    const uint32_t k1 = min(n, k0 + L);
+    if (k0 < k1) {
+      const uint32_t* sOut = reinterpret_cast<const uint32_t*>(sb + (size_t)p.mode * p.stage_words);
+      const float* sVal = sb + (size_t)N * p.stage_words;
+      const uint32_t* sIdx[G];
+#pragma unroll
+      for (int q = 0; q < G; ++q)
+        sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * p.stage_words);
+      float* outp = p.out + 4 * sub;
+      uint32_t cur = sOut[k0];
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      uint32_t k = k0;
+      // batches of kFragUnroll: all loads first, then the sequential segmented reduction
+      // gather slot q of nonzero k (staged: shared memory, else global via L1/L2)
+      auto gather = [&](int q, uint32_t kk) -> float4 {
+        if (q < S) return sbase[q < S ? q : 0][sIdx[q][kk] * LPN];
+        return ldg128(gbase[q >= S ? q - S : 0] + (size_t)sIdx[q][kk] * LPN);
+      };
+      for (; k + kFragUnroll <= k1; k += kFragUnroll) {
+        uint32_t ii[kFragUnroll];
+        float4 pr[kFragUnroll], la[kFragUnroll];
+#pragma unroll
+        for (int u = 0; u < kFragUnroll; ++u) {
+          ii[u] = sOut[k + u];
+          const float v = sVal[k + u];
+          pr[u] = make_float4(v, v, v, v);
+        }
+#pragma unroll
+        for (int q = 0; q < G; ++q) {
+#pragma unroll
+          for (int u = 0; u < kFragUnroll; ++u) {
+            const float4 a = gather(q, k + u);
+            if (q + 1 < G) {
+              pr[u].x *= a.x; pr[u].y *= a.y; pr[u].z *= a.z; pr[u].w *= a.w;
+            } else {
+              la[u] = a;
+            }
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < kFragUnroll; ++u) {
+          if (ii[u] != cur) {
+            red_add_v4_nomem(outp + (size_t)cur * R, acc);
+            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            cur = ii[u];
+          }
+          acc.x = fmaf(pr[u].x, la[u].x, acc.x);
+          acc.y = fmaf(pr[u].y, la[u].y, acc.y);
+          acc.z = fmaf(pr[u].z, la[u].z, acc.z);
+          acc.w = fmaf(pr[u].w, la[u].w, acc.w);
+        }
+      }
+      for (; k < k1; ++k) {
+        const uint32_t i = sOut[k];
+        const float v = sVal[k];
+        float4 pr = make_float4(v, v, v, v), la = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+        for (int q = 0; q < G; ++q) {
+          const float4 a = gather(q, k);
+          if (q + 1 < G) {
+            pr.x *= a.x; pr.y *= a.y; pr.z *= a.z; pr.w *= a.w;
+          } else {
+            la = a;
+          }
+        }
+        if (i != cur) {
+          red_add_v4_nomem(outp + (size_t)cur * R, acc);
+          acc = make_float4(0.f, 0.f, 0.f, 0.f);
+          cur = i;
+        }
+        acc.x = fmaf(pr.x, la.x, acc.x);
+        acc.y = fmaf(pr.y, la.y, acc.y);
+        acc.z = fmaf(pr.z, la.z, acc.z);
+        acc.w = fmaf(pr.w, la.w, acc.w);
+      }
+      red_add_v4_nomem(outp + (size_t)cur * R, acc);
+    }
+    __syncthreads();  // stage s fully consumed
+    if (tid == 0 && j + kFragStages < j1) issue(j + kFragStages, s);
+  }
+}
+
+// Per-R dispatch (defined in sf_frag_r{16,32,64}.cu).
+void frag_launch_r16(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
+void frag_launch_r32(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
+void frag_launch_r64(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
+int frag_occ_r16(int N, int S, int threads, size_t smem);
+int frag_occ_r32(int N, int S, int threads, size_t smem);
+int frag_occ_r64(int N, int S, int threads, size_t smem);
+
+template <int N, int R, int S>
+void frag_launch_one(const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s) {
+  auto k = frag_kernel<N, R, S>;
+  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  k<<<grid, threads, smem, s>>>(fp);
+}
+
+template <int N, int R, int S>
+int frag_occ_one(int threads, size_t smem) {
+  auto k = frag_kernel<N, R, S>;
+  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int nb = 0;
+  SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));
+  return nb;
+}
+
+// (N, S) -> instantiation, for one R.
+#define SF_FRAG_NS_SWITCH(R, FN, ...)                  \
+  switch (N * 10 + S) {                                \
+    case 20: return FN<2, R, 0>(__VA_ARGS__);          \
+    case 21: return FN<2, R, 1>(__VA_ARGS__);          \
+    case 30: return FN<3, R, 0>(__VA_ARGS__);          \
+    case 31: return FN<3, R, 1>(__VA_ARGS__);          \
+    case 32: return FN<3, R, 2>(__VA_ARGS__);          \
+    case 40: return FN<4, R, 0>(__VA_ARGS__);          \
+    case 41: return FN<4, R, 1>(__VA_ARGS__);          \
+    case 42: return FN<4, R, 2>(__VA_ARGS__);          \
+    case 43: return FN<4, R, 3>(__VA_ARGS__);          \
+    case 50: return FN<5, R, 0>(__VA_ARGS__);          \
+    case 51: return FN<5, R, 1>(__VA_ARGS__);          \
+    case 52: return FN<5, R, 2>(__VA_ARGS__);          \
+    case 53: return FN<5, R, 3>(__VA_ARGS__);          \
+    case 54: return FN<5, R, 4>(__VA_ARGS__);          \
+    default: break;                                    \
+  }
+
+#define SF_DEFINE_FRAG_R(R)                                                                              \
+  void frag_launch_r##R(int N, int S, const FragParams& fp, int grid, int threads, size_t smem,          \
+                        cudaStream_t s) {                                                                \
+    SF_FRAG_NS_SWITCH(R, frag_launch_one, fp, grid, threads, smem, s);                                   \
+    throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: unsupported (N, S)"};                           \
+  }                                                                                                      \
+  int frag_occ_r##R(int N, int S, int threads, size_t smem) {                                            \
+    SF_FRAG_NS_SWITCH(R, frag_occ_one, threads, smem);                                                   \
+    return 0;                                                                                            \
+  }
+
+}  // namespace sf

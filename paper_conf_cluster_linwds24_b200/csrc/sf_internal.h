@@ -108,6 +108,7 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
                 cudaStream_t s);
 int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem);
 bool frag_supported(int nmodes, int rank);
+void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s);
 void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
                       uint32_t* const* inds, int* d_flag, cudaStream_t s);
 

@@ -27,6 +27,7 @@
 #include <algorithm>
 #include <cstdio>
 
+#include "sf_frag.cuh"
 #include "sf_internal.h"
 
 namespace sf {
@@ -200,220 +201,54 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
 }
 
 // ---------------------------------------------------------------------------
-// Fragment kernel
+// Boundary-row helper (multi-GPU exchange, §8(e))
 // ---------------------------------------------------------------------------
-struct FragParams {
-  const uint32_t* ind[SF_MAX_MODES];  // kernel-order indices, every mode
-  const float* val;
-  const float* fac[SF_MAX_MODES];
-  float* out;
-  const uint32_t* chunk_begin;  // num_chunks + 1
-  const uint64_t* chunk_tile;   // num_chunks
-  uint32_t num_chunks;
-  uint32_t nnz;
-  int mode;
-  uint32_t staged_mask;
-  uint32_t block_rows[SF_MAX_MODES];
-  uint32_t ntiles[SF_MAX_MODES];   // ceil(I_m / block_rows[m]) for staged modes
-  uint32_t dims[SF_MAX_MODES];
-  uint32_t fac_off[SF_MAX_MODES];  // float offset of the staged block of mode m in smem
-  uint32_t stage_words;            // words per field per pipeline stage
-};
-
-constexpr int kStages = 2;
-
-template <int N, int R>
-__global__ void __launch_bounds__(1024) frag_kernel(FragParams p) {
-  constexpr int LPN = R / 4;  // lanes per nonzero
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);  // [kStages] stream + [1] factors
-  float* stage_base = reinterpret_cast<float*>(smem_raw + 128);
-  float* fac_smem = stage_base + (size_t)kStages * (N + 1) * p.stage_words;
-
-  const int tid = threadIdx.x;
-  const int sub = tid % LPN;
-  const int group = tid / LPN;
-  const int ngroups = blockDim.x / LPN;
-
-  // This CTA's chunk range: chunks whose begin lies in [c*nnz/G, (c+1)*nnz/G).
-  const uint64_t G = gridDim.x;
-  auto lower = [&](uint64_t target) {
-    uint32_t lo = 0, hi = p.num_chunks;
-    while (lo < hi) {
-      uint32_t mid = (lo + hi) >> 1;
-      if ((uint64_t)p.chunk_begin[mid] < target) lo = mid + 1; else hi = mid;
-    }
-    return lo;
-  };
-  const uint32_t j0 = lower(((uint64_t)blockIdx.x * p.nnz) / G);
-  const uint32_t j1 = lower(((uint64_t)(blockIdx.x + 1) * p.nnz) / G);
-  if (j0 >= j1) return;
-
-  if (tid == 0) {
-    for (int s = 0; s <= kStages; ++s) mbar_init(&bars[s], 1);
-    fence_barrier_init();
-  }
-  __syncthreads();
-
-  // Producer: issue the N+1 bulk copies of chunk j into stage s (aligned superset).
-  auto issue = [&](uint32_t j, int s) {
-    const uint32_t b = p.chunk_begin[j], e = p.chunk_begin[j + 1];
-    const uint32_t start = b & ~3u;
-    const uint32_t bytes = (((e - start) + 3u) & ~3u) * 4u;
-    float* dst = stage_base + (size_t)s * (N + 1) * p.stage_words;
-    mbar_expect_tx(&bars[s], bytes * (N + 1));
-#pragma unroll
-    for (int m = 0; m < N; ++m) bulk_g2s(dst + (size_t)m * p.stage_words, p.ind[m] + start, bytes, &bars[s]);
-    bulk_g2s(dst + (size_t)N * p.stage_words, p.val + start, bytes, &bars[s]);
-  };
-
-  if (tid == 0) {
-    for (int s = 0; s < kStages && j0 + s < j1; ++s) issue(j0 + s, s);
-  }
-
-  uint64_t cur_tile = ~0ull;
-  uint32_t base[N];
-#pragma unroll
-  for (int m = 0; m < N; ++m) base[m] = 0;
-  uint32_t fac_phase = 0;
-
-  for (uint32_t j = j0; j < j1; ++j) {
-    const int s = (int)((j - j0) % kStages);
-    const uint32_t parity = ((j - j0) / kStages) & 1u;
-
-    // (Re)stage factor blocks when the tile changes.
-    if (p.staged_mask) {
-      const uint64_t tile = p.chunk_tile[j];
-      if (tile != cur_tile) {
-        cur_tile = tile;
-        uint64_t t = tile;
-#pragma unroll
-        for (int m = N - 1; m >= 0; --m) {
-          if (p.staged_mask & (1u << m)) {
-            const uint32_t q = (uint32_t)(t % p.ntiles[m]);
-            t /= p.ntiles[m];
-            base[m] = q * p.block_rows[m];
-          }
-        }
-        __syncthreads();  // everyone is done with the previous block
-        if (tid == 0) {
-          uint32_t total = 0;
-#pragma unroll
-          for (int m = 0; m < N; ++m)
-            if (p.staged_mask & (1u << m)) {
-              const uint32_t rows = min(p.block_rows[m], p.dims[m] - base[m]);
-              total += rows * R * 4u;
-            }
-          mbar_expect_tx(&bars[kStages], total);
-#pragma unroll
-          for (int m = 0; m < N; ++m)
-            if (p.staged_mask & (1u << m)) {
-              const uint32_t rows = min(p.block_rows[m], p.dims[m] - base[m]);
-              bulk_g2s(fac_smem + p.fac_off[m], p.fac[m] + (size_t)base[m] * R, rows * R * 4u,
-                       &bars[kStages]);
-            }
-        }
-        mbar_wait(&bars[kStages], fac_phase);
-        fac_phase ^= 1u;
-      }
-    }
-
-    mbar_wait(&bars[s], parity);
-
-    const uint32_t b = p.chunk_begin[j], e = p.chunk_begin[j + 1];
-    const uint32_t off = b - (b & ~3u);
-    const uint32_t n = e - b;
-    const float* sb = stage_base + (size_t)s * (N + 1) * p.stage_words + off;
-    // stretch length per group, bumped so the groups of one warp hit distinct banks
-    uint32_t L = (n + ngroups - 1) / ngroups;
-    // (the 32/LPN groups of a warp read word g*L + k: distinct banks iff gcd(L,32) <= LPN)
-    if (LPN < 32)
-      while (L % (2u * LPN) == 0u) ++L;
-    const uint32_t k0 = group * L;
-    const uint32_t k1 = min(n, k0 + L);
-    if (k0 < k1) {
-      const uint32_t* sI = reinterpret_cast<const uint32_t*>(sb);
-      const float* sV = sb + (size_t)N * p.stage_words;
-      uint32_t cur = sI[(size_t)p.mode * p.stage_words + k0];
-      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-      for (uint32_t k = k0; k < k1; ++k) {
-        const float v = sV[k];
-        float4 prod = make_float4(v, v, v, v);
-#pragma unroll
-        for (int m = 0; m < N; ++m) {
-          if (m == p.mode) continue;
-          const uint32_t im = sI[(size_t)m * p.stage_words + k];
-          float4 a;
-          if (p.staged_mask & (1u << m))
-            a = lds_f4(fac_smem + p.fac_off[m] + (im - base[m]) * R + 4 * sub);
-          else
-            a = ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub);
-          prod = f4mul(prod, a);
-        }
-        const uint32_t i = sI[(size_t)p.mode * p.stage_words + k];
-        if (i != cur) {
-          red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
-          acc = make_float4(0.f, 0.f, 0.f, 0.f);
-          cur = i;
-        }
-        acc.x += prod.x;
-        acc.y += prod.y;
-        acc.z += prod.z;
-        acc.w += prod.w;
-      }
-      red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
-    }
-    __syncthreads();  // stage s fully consumed
-    if (tid == 0 && j + kStages < j1) issue(j + kStages, s);
+__global__ void rows_op_kernel(float* __restrict__ Y, int R, const int64_t* __restrict__ rows,
+                               float* __restrict__ buf, int count, int op) {
+  const int k = blockIdx.x;
+  if (k >= count) return;
+  const int64_t r = rows[k];
+  if (r < 0) return;
+  for (int c = threadIdx.x; c < R; c += blockDim.x) {
+    float* y = Y + (size_t)r * R + c;
+    if (op == 0) buf[(size_t)k * R + c] = *y;
+    else if (op == 1) *y += buf[(size_t)k * R + c];
+    else *y = 0.f;
   }
 }
 
-template <int N, int R>
-static void frag_launch_t(const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s) {
-  auto k = frag_kernel<N, R>;
-  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  k<<<grid, threads, smem, s>>>(fp);
+void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s) {
+  if (count <= 0) return;
+  rows_op_kernel<<<count, 128, 0, s>>>(Y, R, rows, buf, count, op);
+  count_launch();
+  SF_CUDA(cudaGetLastError());
 }
-
-template <int N, int R>
-static int frag_occ_t(int threads, size_t smem) {
-  auto k = frag_kernel<N, R>;
-  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int nb = 0;
-  SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));
-  return nb;
-}
-
-#define SF_FRAG_DISPATCH(FN, ...)                                        \
-  switch (nmodes * 1000 + rank) {                                        \
-    case 2016: return FN<2, 16>(__VA_ARGS__);                            \
-    case 2032: return FN<2, 32>(__VA_ARGS__);                            \
-    case 2064: return FN<2, 64>(__VA_ARGS__);                            \
-    case 3016: return FN<3, 16>(__VA_ARGS__);                            \
-    case 3032: return FN<3, 32>(__VA_ARGS__);                            \
-    case 3064: return FN<3, 64>(__VA_ARGS__);                            \
-    case 4016: return FN<4, 16>(__VA_ARGS__);                            \
-    case 4032: return FN<4, 32>(__VA_ARGS__);                            \
-    case 4064: return FN<4, 64>(__VA_ARGS__);                            \
-    case 5016: return FN<5, 16>(__VA_ARGS__);                            \
-    case 5032: return FN<5, 32>(__VA_ARGS__);                            \
-    case 5064: return FN<5, 64>(__VA_ARGS__);                            \
-    default: break;                                                      \
-  }
 
 bool frag_supported(int nmodes, int rank) {
   return nmodes >= 2 && nmodes <= 5 && (rank == 16 || rank == 32 || rank == 64);
 }
 
-int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem) {
-  SF_FRAG_DISPATCH(frag_occ_t, threads, smem);
-  return 0;
+static int frag_occ(int N, int R, int S, int threads, size_t smem) {
+  switch (R) {
+    case 16: return frag_occ_r16(N, S, threads, smem);
+    case 32: return frag_occ_r32(N, S, threads, smem);
+    case 64: return frag_occ_r64(N, S, threads, smem);
+    default: return 0;
+  }
 }
 
-static void frag_launch(int nmodes, int rank, const FragParams& fp, int grid, int threads,
-                        size_t smem, cudaStream_t s) {
-  SF_FRAG_DISPATCH(frag_launch_t, fp, grid, threads, smem, s);
-  throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: unsupported (nmodes, rank)"};
+int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem) {
+  return frag_occ(nmodes, rank, 0, threads, smem);
+}
+
+static void frag_launch(int N, int R, int S, const FragParams& fp, int grid, int threads, size_t smem,
+                        cudaStream_t s) {
+  switch (R) {
+    case 16: return frag_launch_r16(N, S, fp, grid, threads, smem, s);
+    case 32: return frag_launch_r32(N, S, fp, grid, threads, smem, s);
+    case 64: return frag_launch_r64(N, S, fp, grid, threads, smem, s);
+    default: throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: unsupported rank"};
+  }
 }
 
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
@@ -441,29 +276,31 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   fp.num_chunks = (uint32_t)p.num_chunks;
   fp.nnz = (uint32_t)p.nnz_local;
   fp.mode = n;
-  fp.staged_mask = p.launch.staged_mask;
   fp.stage_words = (uint32_t)p.launch.chunk_nnz + 8;
+  // slots: staged modes first (ascending mode id = tile-id fold order), then the rest
+  int S = 0, q = 0;
   uint32_t off = 0;
-  for (int m = 0; m < N; ++m) {
-    if (p.launch.staged_mask & (1u << m)) {
-      fp.block_rows[m] = p.launch.block_rows[m];
-      fp.ntiles[m] = (uint32_t)((t.dims[m] + fp.block_rows[m] - 1) / fp.block_rows[m]);
-      fp.fac_off[m] = off;
-      off += fp.block_rows[m] * (uint32_t)R;
-    } else {
-      fp.block_rows[m] = 1;
-      fp.ntiles[m] = 1;
+  for (int m = 0; m < N; ++m)
+    if (m != n && (p.launch.staged_mask & (1u << m))) {
+      fp.slot_mode[q] = m;
+      fp.block_rows[q] = p.launch.block_rows[m];
+      fp.ntiles[q] = (uint32_t)((t.dims[m] + fp.block_rows[q] - 1) / fp.block_rows[q]);
+      fp.fac_off[q] = off;
+      off += fp.block_rows[q] * (uint32_t)R;
+      ++q;
+      ++S;
     }
-  }
+  for (int m = 0; m < N; ++m)
+    if (m != n && !(p.launch.staged_mask & (1u << m))) fp.slot_mode[q++] = m;
   const size_t smem = frag_smem_bytes(t, n, R, p.launch);
   const int threads = p.launch.block_threads;
   int per_sm = p.launch.ctas_per_sm;
-  const int occ = frag_max_ctas_per_sm(N, R, threads, smem);
+  const int occ = frag_occ(N, R, S, threads, smem);
   if (occ <= 0) throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: launch does not fit an SM"};
   if (per_sm <= 0 || per_sm > occ) per_sm = occ;
   int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
   grid = std::max(grid, 1);
-  frag_launch(N, R, fp, grid, threads, smem, s);
+  frag_launch(N, R, S, fp, grid, threads, smem, s);
   count_launch();
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {

@@ -1,0 +1,113 @@
+#!/usr/bin/env python
+"""Exhaustive launch sweep (validates the adaptive selector, §8(a) A4; PAPER.md
+§III-A Fig. 4 L157-167 and §IV-B).
+
+For each mode of a config: time sf_mttkrp under every launch in a grid
+(kernel x staged-mode subset x block rows x chunk length x threads), then report the
+selector's pick, its rank and its throughput relative to the sweep best.
+Writes one JSON object per line to stdout (and --out).
+"""
+from __future__ import annotations
+
+import argparse
+import itertools
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+
+def time_launch(T, n, R, facs, out, L, sf, torch, reps=5):
+    try:
+        T.set_launch(n, R, L)
+    except sf.SfError as e:
+        return None, str(e)
+    s = torch.cuda.current_stream()
+    for _ in range(2):
+        T.mttkrp(n, facs, out)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(reps):
+        T.mttkrp(n, facs, out)
+    e1.record(s)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps, None
+
+
+def grid(dims, n, R, quick):
+    others = [m for m in range(len(dims)) if m != n]
+    row_opts = [256, 512, 775, 1024, 1536] if not quick else [512, 775]
+    chunks = [512, 1024, 2048] if not quick else [1024]
+    threads = [256, 512, 1024] if not quick else [512]
+    staged_sets = [()]
+    for k in range(1, len(others) + 1):
+        staged_sets += list(itertools.combinations(others, k))
+    for st in staged_sets:
+        rows_choices = [()] if not st else itertools.product(row_opts, repeat=len(st))
+        for rows in rows_choices:
+            for C, th in itertools.product(chunks, threads):
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C,
+                       "staged": {m: min(r, dims[m]) for m, r in zip(st, rows)}}
+    yield {"kernel": 1}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="nell2")
+    ap.add_argument("--modes", default=None)
+    ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    import torch
+
+    import paper_conf_cluster_linwds24_b200 as sf
+    cfg = synth.CONFIGS[args.config]
+    inds, vals = synth.config_tensor(cfg)
+    facs = [torch.from_numpy(f).cuda() for f in synth.config_factors(cfg)]
+    R = cfg.rank
+    T = sf.Tensor(cfg.dims, [torch.from_numpy(a.view(np.int32)) for a in inds], torch.from_numpy(vals))
+    modes = [int(x) for x in args.modes.split(",")] if args.modes else range(cfg.nmodes)
+    outf = open(args.out, "w") if args.out else None
+    flops = cfg.nmodes * cfg.nnz * R
+    for n in modes:
+        out = torch.empty((cfg.dims[n], R), device="cuda")
+        T.plan(n, R)
+        pick = T.plan_info(n, R)["launch"]
+        t_pick, _ = time_launch(T, n, R, facs, out, sf.Launch.make(
+            kernel=2 if pick["kernel"] == "frag" else 1, block_threads=pick["block_threads"],
+            ctas_per_sm=pick["ctas_per_sm"], chunk_nnz=pick["chunk_nnz"],
+            staged={m: r for m, r in enumerate(pick["block_rows"]) if pick["staged_mask"] >> m & 1}),
+            sf, torch)
+        results = []
+        t0 = time.time()
+        for g in grid(cfg.dims, n, R, args.quick):
+            L = sf.Launch.make(**g)
+            ms, err = time_launch(T, n, R, facs, out, L, sf, torch)
+            rec = {"mode": n, "launch": g, "ms": ms, "err": err,
+                   "gflops": flops / cfg.nmodes / ms / 1e6 if ms else None}
+            results.append(rec)
+            line = json.dumps(rec)
+            print(line, flush=True)
+            if outf:
+                outf.write(line + "\n")
+        ok = sorted([r for r in results if r["ms"]], key=lambda r: r["ms"])
+        best = ok[0]
+        rank_of_pick = sum(1 for r in ok if r["ms"] < t_pick) + 1
+        summ = {"summary": True, "config": cfg.name, "mode": n, "pick": pick, "pick_ms": t_pick,
+                "best": best["launch"], "best_ms": best["ms"], "pick_over_best": best["ms"] / t_pick,
+                "pick_rank": rank_of_pick, "n_launches": len(ok), "sweep_s": time.time() - t0}
+        print(json.dumps(summ), flush=True)
+        if outf:
+            outf.write(json.dumps(summ) + "\n")
+    T.close()
+
+
+if __name__ == "__main__":
+    main()
