@@ -157,6 +157,13 @@ def run_reference(args, cfg, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def launch_from_json(sf, d):
+    d = dict(d)
+    if "staged" in d:
+        d["staged"] = {int(k): int(v) for k, v in d["staged"].items()}
+    return sf.Launch.make(**d)
+
+
 def workload_config(cfg, world):
     return {"workload": f"{cfg.name}: {cfg.note}", "dims": list(cfg.dims), "nnz": cfg.nnz,
             "rank": cfg.rank, "zipf": list(cfg.zipf), "modes": cfg.nmodes,
@@ -217,11 +224,14 @@ def main():
     T = sf.Tensor(cfg.dims, h_inds, h_vals)
     if world > 1:
         T.set_shard(world, rank)
-    overrides = json.loads(args.launch_json) if args.launch_json else {}
+    overrides = {}
+    if args.launch_json:
+        src = args.launch_json
+        overrides = json.load(open(src[1:])) if src.startswith("@") else json.loads(src)
     plan_ms = {}
     for n in range(N):
         if str(n) in overrides:
-            T.set_launch(n, R, sf.Launch.make(**overrides[str(n)]))
+            T.set_launch(n, R, launch_from_json(sf, overrides[str(n)]))
         else:
             T.plan(n, R)
         plan_ms[n] = T.plan_info(n, R)["plan_ms"]
@@ -304,7 +314,7 @@ def main():
                 df = [f.to(dev, non_blocking=True) for f in h_facs]
                 for n in range(N):
                     if str(n) in overrides:
-                        T2.set_launch(n, R, sf.Launch.make(**overrides[str(n)]))
+                        T2.set_launch(n, R, launch_from_json(sf, overrides[str(n)]))
                     else:
                         T2.plan(n, R)
                 inf = {n: T2.plan_info(n, R) for n in range(N)}

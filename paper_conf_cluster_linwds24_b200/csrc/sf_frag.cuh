@@ -99,21 +99,65 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 
 }  // namespace detail
 
+// Lane mapping.  VEC = floats per lane (4 for R <= 16, else 8), LPN = R / VEC lanes per
+// nonzero.  A lane owns the two (VEC = 8) or one (VEC = 4) 16-byte chunks c0, c1 of a
+// factor row.  R = 32: the two groups of a quarter-warp read complementary chunk sets
+// (group parity p: c0 = 2t+p, c1 = 2t+1-p), so every 128-bit shared load of a
+// quarter-warp touches all 32 banks once; R >= 64: c0 = t, c1 = t + LPN.
+template <int R>
+struct LaneMap {
+  static constexpr int VEC = (R >= 32) ? 8 : 4;
+  static constexpr int LPN = R / VEC;
+  __device__ __forceinline__ static void chunks(int t, int group, int& c0, int& c1) {
+    if constexpr (VEC == 4) {
+      c0 = t;
+      c1 = t;
+    } else if constexpr (R == 32) {
+      const int par = group & 1;
+      c0 = 2 * t + par;
+      c1 = 2 * t + 1 - par;
+    } else {
+      c0 = t;
+      c1 = t + LPN;
+    }
+  }
+};
+
+struct F8 {
+  float4 a, b;
+};
+
+__device__ __forceinline__ void f4mul_(float4& x, const float4& y) {
+  x.x *= y.x; x.y *= y.y; x.z *= y.z; x.w *= y.w;
+}
+__device__ __forceinline__ void f4fma_(float4& acc, const float4& x, const float4& y) {
+  acc.x = fmaf(x.x, y.x, acc.x);
+  acc.y = fmaf(x.y, y.y, acc.y);
+  acc.z = fmaf(x.z, y.z, acc.z);
+  acc.w = fmaf(x.w, y.w, acc.w);
+}
+
 template <int N, int R, int S>
 __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   using namespace detail;
-  constexpr int LPN = R / 4;  // lanes per nonzero
-  constexpr int G = N - 1;    // gathered slots
-  constexpr int RB = R * 4;   // bytes per factor row
+  using LM = LaneMap<R>;
+  constexpr int VEC = LM::VEC;
+  constexpr int LPN = LM::LPN;  // lanes per nonzero
+  constexpr int G = N - 1;      // gathered slots
+  constexpr int RB = R * 4;     // bytes per factor row
+  constexpr int R4 = R / 4;     // float4 per factor row
+  constexpr int U = (VEC == 8) ? 2 : kFragUnroll;  // batch (register budget: 64 at 1024 thr)
   extern __shared__ __align__(128) unsigned char smem_raw[];
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);  // [kFragStages] stream + [1] factors
   float* stage_base = reinterpret_cast<float*>(smem_raw + 128);
   float* fac_smem = stage_base + (size_t)kFragStages * (N + 1) * p.stage_words;
 
   const int tid = threadIdx.x;
-  const int sub = tid % LPN;
+  const int lane_in_group = tid % LPN;
   const int group = tid / LPN;
   const int ngroups = blockDim.x / LPN;
+  int c0, c1;
+  LM::chunks(lane_in_group, group, c0, c1);
 
   // This CTA's chunks: those whose begin lies in [c*nnz/G, (c+1)*nnz/G).
   const uint64_t grid = gridDim.x;
@@ -148,12 +192,13 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   if (tid == 0)
     for (int s = 0; s < kFragStages && j0 + s < j1; ++s) issue(j0 + s, s);
 
-  // Per-slot gather bases.  Staged slots: shared address of row 0 of the *virtual*
-  // full factor (block base minus tile_row0 * RB), so addr = base + idx * RB.
+  // Per-slot gather bases (float4 pointers to row 0).  Staged slots point at row 0 of
+  // the *virtual* full factor (block base minus the tile's first row), so one formula
+  // row * R4 + chunk serves both.
   const float4* sbase[S > 0 ? S : 1];
   const float4* gbase[G - S > 0 ? G - S : 1];
 #pragma unroll
-  for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]) + sub;
+  for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]);
   uint64_t cur_tile = ~0ull;
   uint32_t fac_phase = 0;
 
@@ -188,8 +233,7 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
         }
 #pragma unroll
         for (int q = 0; q < S; ++q)
-          sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) + sub -
-                     (ptrdiff_t)row0[q] * LPN;
+          sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (ptrdiff_t)row0[q] * R4;
         mbar_wait(&bars[kFragStages], fac_phase);
         fac_phase ^= 1u;
       }
@@ -213,74 +257,85 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
 #pragma unroll
       for (int q = 0; q < G; ++q)
         sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * p.stage_words);
-      float* outp = p.out + 4 * sub;
-      uint32_t cur = sOut[k0];
-      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-      uint32_t k = k0;
-      // batches of kFragUnroll: all loads first, then the sequential segmented reduction
-      // gather slot q of nonzero k (staged: shared memory, else global via L1/L2)
-      auto gather = [&](int q, uint32_t kk) -> float4 {
-        if (q < S) return sbase[q < S ? q : 0][sIdx[q][kk] * LPN];
-        return ldg128(gbase[q >= S ? q - S : 0] + (size_t)sIdx[q][kk] * LPN);
+      float* out0 = p.out + 4 * c0;
+      float* out1 = p.out + 4 * c1;
+      // gather slot q of nonzero kk (staged: shared memory, else global via L1/L2)
+      auto gather = [&](int q, uint32_t kk) -> F8 {
+        const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
+        const size_t row = (size_t)sIdx[q][kk] * R4;
+        F8 r;
+        if (q < S) {
+          r.a = base[row + c0];
+          if constexpr (VEC == 8) r.b = base[row + c1];
+        } else {
+          r.a = ldg128(base + row + c0);
+          if constexpr (VEC == 8) r.b = ldg128(base + row + c1);
+        }
+        return r;
       };
-      for (; k + kFragUnroll <= k1; k += kFragUnroll) {
-        uint32_t ii[kFragUnroll];
-        float4 pr[kFragUnroll], la[kFragUnroll];
+      uint32_t cur = sOut[k0];
+      float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
+      auto flush = [&]() {
+        red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
+        if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
+        acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
+        acc1 = acc0;
+      };
+      uint32_t k = k0;
+      // batches of U: all loads first, then the sequential segmented reduction
+      // y += v * (a_0 * ... * a_{G-1}): G-1 FMUL + 1 FFMA per float, VEC+1 live regs per nnz
+      for (; k + U <= k1; k += U) {
+        uint32_t ii[U];
+        float vv[U];
+        F8 pr[U];
 #pragma unroll
-        for (int u = 0; u < kFragUnroll; ++u) {
+        for (int u = 0; u < U; ++u) {
           ii[u] = sOut[k + u];
-          const float v = sVal[k + u];
-          pr[u] = make_float4(v, v, v, v);
+          vv[u] = sVal[k + u];
         }
 #pragma unroll
         for (int q = 0; q < G; ++q) {
 #pragma unroll
-          for (int u = 0; u < kFragUnroll; ++u) {
-            const float4 a = gather(q, k + u);
-            if (q + 1 < G) {
-              pr[u].x *= a.x; pr[u].y *= a.y; pr[u].z *= a.z; pr[u].w *= a.w;
+          for (int u = 0; u < U; ++u) {
+            const F8 a = gather(q, k + u);
+            if (q == 0) {
+              pr[u] = a;
             } else {
-              la[u] = a;
+              f4mul_(pr[u].a, a.a);
+              if constexpr (VEC == 8) f4mul_(pr[u].b, a.b);
             }
           }
         }
 #pragma unroll
-        for (int u = 0; u < kFragUnroll; ++u) {
+        for (int u = 0; u < U; ++u) {
           if (ii[u] != cur) {
-            red_add_v4_nomem(outp + (size_t)cur * R, acc);
-            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            flush();
             cur = ii[u];
           }
-          acc.x = fmaf(pr[u].x, la[u].x, acc.x);
-          acc.y = fmaf(pr[u].y, la[u].y, acc.y);
-          acc.z = fmaf(pr[u].z, la[u].z, acc.z);
-          acc.w = fmaf(pr[u].w, la[u].w, acc.w);
+          const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
+          f4fma_(acc0, vb, pr[u].a);
+          if constexpr (VEC == 8) f4fma_(acc1, vb, pr[u].b);
         }
       }
       for (; k < k1; ++k) {
         const uint32_t i = sOut[k];
         const float v = sVal[k];
-        float4 pr = make_float4(v, v, v, v), la = make_float4(0.f, 0.f, 0.f, 0.f);
+        F8 pr = gather(0, k);
 #pragma unroll
-        for (int q = 0; q < G; ++q) {
-          const float4 a = gather(q, k);
-          if (q + 1 < G) {
-            pr.x *= a.x; pr.y *= a.y; pr.z *= a.z; pr.w *= a.w;
-          } else {
-            la = a;
-          }
+        for (int q = 1; q < G; ++q) {
+          const F8 a = gather(q, k);
+          f4mul_(pr.a, a.a);
+          if constexpr (VEC == 8) f4mul_(pr.b, a.b);
         }
         if (i != cur) {
-          red_add_v4_nomem(outp + (size_t)cur * R, acc);
-          acc = make_float4(0.f, 0.f, 0.f, 0.f);
+          flush();
           cur = i;
         }
-        acc.x = fmaf(pr.x, la.x, acc.x);
-        acc.y = fmaf(pr.y, la.y, acc.y);
-        acc.z = fmaf(pr.z, la.z, acc.z);
-        acc.w = fmaf(pr.w, la.w, acc.w);
+        const float4 vb = make_float4(v, v, v, v);
+        f4fma_(acc0, vb, pr.a);
+        if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
       }
-      red_add_v4_nomem(outp + (size_t)cur * R, acc);
+      flush();
     }
     __syncthreads();  // stage s fully consumed
     if (tid == 0 && j + kFragStages < j1) issue(j + kFragStages, s);
