@@ -70,7 +70,11 @@ typedef struct {
   uint32_t staged_mask;  /* FRAG: bit m set => factor m is staged in shared memory by
                             blocks of block_rows[m] rows (a "tensor block") */
   uint32_t block_rows[SF_MAX_MODES];
+  uint32_t flags;        /* FRAG: SF_LAUNCH_PREFETCH_L2 = prefetch each stretch's global
+                            factor rows into L2 before gathering (memory-level parallelism
+                            without registers) */
 } sf_launch_t;
+#define SF_LAUNCH_PREFETCH_L2 1u
 
 /* Tensor feature vector (reading R4). Integers are exact. */
 typedef struct {

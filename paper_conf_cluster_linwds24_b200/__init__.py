@@ -23,6 +23,7 @@ _lib = None
 SF_MAX_MODES = 8
 SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
+LAUNCH_PREFETCH_L2 = 1
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",
@@ -38,19 +39,21 @@ class SfError(RuntimeError):
 class Launch(ctypes.Structure):
     _fields_ = [("kernel", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("chunk_nnz", ctypes.c_int32),
-                ("staged_mask", ctypes.c_uint32), ("block_rows", ctypes.c_uint32 * SF_MAX_MODES)]
+                ("staged_mask", ctypes.c_uint32), ("block_rows", ctypes.c_uint32 * SF_MAX_MODES),
+                ("flags", ctypes.c_uint32)]
 
     def as_dict(self):
         return {"kernel": {0: "auto", 1: "coo", 2: "frag"}.get(self.kernel, self.kernel),
                 "block_threads": self.block_threads, "ctas_per_sm": self.ctas_per_sm,
                 "chunk_nnz": self.chunk_nnz, "staged_mask": self.staged_mask,
-                "block_rows": list(self.block_rows)}
+                "block_rows": list(self.block_rows), "flags": self.flags}
 
     @classmethod
-    def make(cls, kernel=KERNEL_FRAG, block_threads=512, ctas_per_sm=0, chunk_nnz=1024,
-             staged=None):
-        """staged: {mode: block_rows}"""
+    def make(cls, kernel=KERNEL_FRAG, block_threads=512, ctas_per_sm=0, chunk_nnz=128,
+             staged=None, flags=0):
+        """staged: {mode: block_rows}; flags: LAUNCH_PREFETCH_L2"""
         l = cls()
+        l.flags = flags
         l.kernel, l.block_threads, l.ctas_per_sm, l.chunk_nnz = kernel, block_threads, ctas_per_sm, chunk_nnz
         mask = 0
         for m, r in (staged or {}).items():

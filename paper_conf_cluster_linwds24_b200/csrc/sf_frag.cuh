@@ -42,6 +42,7 @@ struct FragParams {
   uint32_t dims[SF_MAX_MODES];        // per mode
   uint32_t fac_off[SF_MAX_MODES];     // per staged slot: float offset of its block in smem
   uint32_t stage_words;               // words per field per pipeline stage
+  uint32_t prefetch;                  // 1: prefetch a stretch's global rows into L2 first
 };
 
 constexpr int kFragStages = 2;
@@ -67,6 +68,10 @@ __device__ __forceinline__ float4 lds128(uint32_t addr) {
 }
 
 __device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
+
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count));
@@ -143,21 +148,30 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   using LM = LaneMap<R>;
   constexpr int VEC = LM::VEC;
   constexpr int LPN = LM::LPN;  // lanes per nonzero
+  constexpr int GPW = 32 / LPN; // lane groups per warp
   constexpr int G = N - 1;      // gathered slots
   constexpr int RB = R * 4;     // bytes per factor row
   constexpr int R4 = R / 4;     // float4 per factor row
   constexpr int U = (VEC == 8) ? 2 : kFragUnroll;  // batch (register budget: 64 at 1024 thr)
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);  // [kFragStages] stream + [1] factors
-  float* stage_base = reinterpret_cast<float*>(smem_raw + 128);
-  float* fac_smem = stage_base + (size_t)kFragStages * (N + 1) * p.stage_words;
 
   const int tid = threadIdx.x;
-  const int lane_in_group = tid % LPN;
-  const int group = tid / LPN;
-  const int ngroups = blockDim.x / LPN;
+  const int warp = tid >> 5;
+  const int lane = tid & 31;
+  const int nwarps = blockDim.x >> 5;
+  const int lane_in_group = lane % LPN;
+  const int group = lane / LPN;  // group within the warp
   int c0, c1;
   LM::chunks(lane_in_group, group, c0, c1);
+
+  // smem: [bars: 2 per warp + 1 factor barrier, 128-B aligned] [per-warp stage rings] [factor blocks]
+  const uint32_t SW = p.stage_words;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);
+  const uint32_t bar_bytes = ((2u * nwarps + 1u) * 8u + 127u) & ~127u;
+  float* ring = reinterpret_cast<float*>(smem_raw + bar_bytes) + (size_t)warp * kFragStages * (N + 1) * SW;
+  float* fac_smem = reinterpret_cast<float*>(smem_raw + bar_bytes) + (size_t)nwarps * kFragStages * (N + 1) * SW;
+  uint64_t* wbar = bars + 2 * warp;
+  uint64_t* fbar = bars + 2 * nwarps;
 
   // This CTA's chunks: those whose begin lies in [c*nnz/G, (c+1)*nnz/G).
   const uint64_t grid = gridDim.x;
@@ -173,172 +187,193 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   const uint32_t j1 = lower(((uint64_t)(blockIdx.x + 1) * p.nnz) / grid);
   if (j0 >= j1) return;
 
-  if (tid == 0) {
-    for (int s = 0; s <= kFragStages; ++s) mbar_init(&bars[s], 1);
+  if (lane == 0) {
+    mbar_init(&wbar[0], 1);
+    mbar_init(&wbar[1], 1);
+    if (warp == 0) mbar_init(fbar, 1);
     fence_barrier_init();
   }
   __syncthreads();
 
-  auto issue = [&](uint32_t j, int s) {
+  // lane 0 of this warp: bulk-copy chunk j's N+1 fields into stage st (aligned superset)
+  auto issue = [&](uint32_t j, int st) {
     const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
     const uint32_t start = b & ~3u;
     const uint32_t bytes = (((e - start) + 3u) & ~3u) * 4u;
-    float* dst = stage_base + (size_t)s * (N + 1) * p.stage_words;
-    mbar_expect_tx(&bars[s], bytes * (N + 1));
+    float* dst = ring + (size_t)st * (N + 1) * SW;
+    mbar_expect_tx(&wbar[st], bytes * (N + 1));
 #pragma unroll
-    for (int m = 0; m < N; ++m) bulk_g2s(dst + (size_t)m * p.stage_words, p.ind[m] + start, bytes, &bars[s]);
-    bulk_g2s(dst + (size_t)N * p.stage_words, p.val + start, bytes, &bars[s]);
+    for (int m = 0; m < N; ++m) bulk_g2s(dst + (size_t)m * SW, p.ind[m] + start, bytes, &wbar[st]);
+    bulk_g2s(dst + (size_t)N * SW, p.val + start, bytes, &wbar[st]);
   };
-  if (tid == 0)
-    for (int s = 0; s < kFragStages && j0 + s < j1; ++s) issue(j0 + s, s);
 
-  // Per-slot gather bases (float4 pointers to row 0).  Staged slots point at row 0 of
-  // the *virtual* full factor (block base minus the tile's first row), so one formula
-  // row * R4 + chunk serves both.
+  // Gather bases (float4 pointers to row 0).  Staged slots point at row 0 of the
+  // *virtual* full factor (block base minus the tile's first row).
   const float4* sbase[S > 0 ? S : 1];
   const float4* gbase[G - S > 0 ? G - S : 1];
 #pragma unroll
   for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]);
-  uint64_t cur_tile = ~0ull;
   uint32_t fac_phase = 0;
+  uint32_t it = 0;  // chunks this warp has consumed (stage = it % 2, parity = (it / 2) & 1)
 
-  for (uint32_t j = j0; j < j1; ++j) {
-    const int s = (int)((j - j0) % kFragStages);
-    const uint32_t parity = ((j - j0) / kFragStages) & 1u;
-
+  uint32_t seg = j0;
+  while (seg < j1) {
+    // tile segment [seg, seg_end): chunks of one tile (the whole range when S == 0)
+    uint32_t seg_end = j1;
     if constexpr (S > 0) {
-      const uint64_t tile = __ldg(p.chunk_tile + j);
-      if (tile != cur_tile) {
-        cur_tile = tile;
-        uint64_t t = tile;
-        uint32_t row0[S];
-#pragma unroll
-        for (int q = S - 1; q >= 0; --q) {
-          const uint32_t qq = (uint32_t)(t % p.ntiles[q]);
-          t /= p.ntiles[q];
-          row0[q] = qq * p.block_rows[q];
-        }
-        __syncthreads();  // everyone is done with the previous blocks
-        if (tid == 0) {
-          uint32_t total = 0;
-#pragma unroll
-          for (int q = 0; q < S; ++q) total += min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]) * RB;
-          mbar_expect_tx(&bars[kFragStages], total);
-#pragma unroll
-          for (int q = 0; q < S; ++q) {
-            const uint32_t rows = min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]);
-            bulk_g2s(fac_smem + p.fac_off[q], p.fac[p.slot_mode[q]] + (size_t)row0[q] * R, rows * RB,
-                     &bars[kFragStages]);
-          }
-        }
-#pragma unroll
-        for (int q = 0; q < S; ++q)
-          sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (ptrdiff_t)row0[q] * R4;
-        mbar_wait(&bars[kFragStages], fac_phase);
-        fac_phase ^= 1u;
+      const uint64_t tile = __ldg(p.chunk_tile + seg);
+      uint32_t lo = seg + 1, hi = j1;  // first chunk with a different (larger) tile
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (__ldg(p.chunk_tile + mid) == tile) lo = mid + 1; else hi = mid;
       }
+      seg_end = lo;
+      uint64_t t = tile;
+      uint32_t row0[S];
+#pragma unroll
+      for (int q = S - 1; q >= 0; --q) {
+        const uint32_t qq = (uint32_t)(t % p.ntiles[q]);
+        t /= p.ntiles[q];
+        row0[q] = qq * p.block_rows[q];
+      }
+      __syncthreads();  // every warp is done with the previous blocks
+      if (tid == 0) {
+        uint32_t total = 0;
+#pragma unroll
+        for (int q = 0; q < S; ++q) total += min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]) * RB;
+        mbar_expect_tx(fbar, total);
+#pragma unroll
+        for (int q = 0; q < S; ++q) {
+          const uint32_t rows = min(p.block_rows[q], p.dims[p.slot_mode[q]] - row0[q]);
+          bulk_g2s(fac_smem + p.fac_off[q], p.fac[p.slot_mode[q]] + (size_t)row0[q] * R, rows * RB, fbar);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < S; ++q)
+        sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (ptrdiff_t)row0[q] * R4;
     }
-
-    mbar_wait(&bars[s], parity);
-
-    const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
-    const uint32_t n = e - b;
-    const float* sb = stage_base + (size_t)s * (N + 1) * p.stage_words + (b - (b & ~3u));
-    uint32_t L = (n + ngroups - 1) / ngroups;
-    // the 32/LPN groups of a warp read word g*L + k: distinct banks iff gcd(L,32) <= LPN
-    if (LPN < 32)
-      while (L % (2u * LPN) == 0u) ++L;
-    const uint32_t k0 = group * L;
-    const uint32_t k1 = min(n, k0 + L);
-    if (k0 < k1) {
-      const uint32_t* sOut = reinterpret_cast<const uint32_t*>(sb + (size_t)p.mode * p.stage_words);
-      const float* sVal = sb + (size_t)N * p.stage_words;
-      const uint32_t* sIdx[G];
+    // this warp's chunks of the segment: seg + warp, seg + warp + nwarps, ...
+    uint32_t jn = seg + warp;
+    if (lane == 0) {
+      if (jn < seg_end) issue(jn, it % kFragStages);
+      if (jn + nwarps < seg_end) issue(jn + nwarps, (it + 1) % kFragStages);
+    }
+    if constexpr (S > 0) {
+      mbar_wait(fbar, fac_phase);
+      fac_phase ^= 1u;
+    }
+    for (uint32_t j = jn; j < seg_end; j += nwarps, ++it) {
+      const int st = (int)(it % kFragStages);
+      mbar_wait(&wbar[st], (it / kFragStages) & 1u);
+      const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
+      const uint32_t n = e - b;
+      const float* sb = ring + (size_t)st * (N + 1) * SW + (b - (b & ~3u));
+      uint32_t L = (n + GPW - 1) / GPW;
+      // the GPW groups of a warp read word g*L + k: distinct banks iff gcd(L,32) <= LPN
+      if (LPN < 32)
+        while (L % (2u * LPN) == 0u) ++L;
+      const uint32_t k0 = group * L;
+      const uint32_t k1 = min(n, k0 + L);
+      if (k0 < k1) {
+        const uint32_t* sOut = reinterpret_cast<const uint32_t*>(sb + (size_t)p.mode * SW);
+        const float* sVal = sb + (size_t)N * SW;
+        const uint32_t* sIdx[G];
 #pragma unroll
-      for (int q = 0; q < G; ++q)
-        sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * p.stage_words);
-      float* out0 = p.out + 4 * c0;
-      float* out1 = p.out + 4 * c1;
-      // gather slot q of nonzero kk (staged: shared memory, else global via L1/L2)
-      auto gather = [&](int q, uint32_t kk) -> F8 {
-        const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
-        const size_t row = (size_t)sIdx[q][kk] * R4;
-        F8 r;
-        if (q < S) {
-          r.a = base[row + c0];
-          if constexpr (VEC == 8) r.b = base[row + c1];
-        } else {
-          r.a = ldg128(base + row + c0);
-          if constexpr (VEC == 8) r.b = ldg128(base + row + c1);
-        }
-        return r;
-      };
-      uint32_t cur = sOut[k0];
-      float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
-      auto flush = [&]() {
-        red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
-        if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
-        acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
-        acc1 = acc0;
-      };
-      uint32_t k = k0;
-      // batches of U: all loads first, then the sequential segmented reduction
-      // y += v * (a_0 * ... * a_{G-1}): G-1 FMUL + 1 FFMA per float, VEC+1 live regs per nnz
-      for (; k + U <= k1; k += U) {
-        uint32_t ii[U];
-        float vv[U];
-        F8 pr[U];
+        for (int q = 0; q < G; ++q) sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * SW);
+        float* out0 = p.out + 4 * c0;
+        float* out1 = p.out + 4 * c1;
+        // gather slot q of nonzero kk (staged: shared memory, else global via L1/L2)
+        auto gather = [&](int q, uint32_t kk) -> F8 {
+          const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
+          const size_t row = (size_t)sIdx[q][kk] * R4;
+          F8 r;
+          if (q < S) {
+            r.a = base[row + c0];
+            if constexpr (VEC == 8) r.b = base[row + c1];
+          } else {
+            r.a = ldg128(base + row + c0);
+            if constexpr (VEC == 8) r.b = ldg128(base + row + c1);
+          }
+          return r;
+        };
+        // Memory-level parallelism without registers: request every global row of this
+        // stretch into L2 up front (one 32-byte sector per lane), then gather.
+        if constexpr (G - S > 0) {
+          if (p.prefetch && (VEC == 8 || (lane_in_group & 1) == 0)) {
+            for (uint32_t kk = k0; kk < k1; ++kk) {
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          ii[u] = sOut[k + u];
-          vv[u] = sVal[k + u];
-        }
-#pragma unroll
-        for (int q = 0; q < G; ++q) {
-#pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const F8 a = gather(q, k + u);
-            if (q == 0) {
-              pr[u] = a;
-            } else {
-              f4mul_(pr[u].a, a.a);
-              if constexpr (VEC == 8) f4mul_(pr[u].b, a.b);
+              for (int q = S; q < G; ++q)
+                prefetch_l2(gbase[q - S] + (size_t)sIdx[q][kk] * R4 + c0);
             }
           }
         }
+        uint32_t cur = sOut[k0];
+        float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
+        auto flush = [&]() {
+          red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
+          if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
+          acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
+          acc1 = acc0;
+        };
+        uint32_t k = k0;
+        // y += v * (a_0 * ... * a_{G-1}): G-1 FMUL + 1 FFMA per float
+        for (; k + U <= k1; k += U) {
+          uint32_t ii[U];
+          float vv[U];
+          F8 pr[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          if (ii[u] != cur) {
-            flush();
-            cur = ii[u];
+          for (int u = 0; u < U; ++u) {
+            ii[u] = sOut[k + u];
+            vv[u] = sVal[k + u];
           }
-          const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
-          f4fma_(acc0, vb, pr[u].a);
-          if constexpr (VEC == 8) f4fma_(acc1, vb, pr[u].b);
-        }
-      }
-      for (; k < k1; ++k) {
-        const uint32_t i = sOut[k];
-        const float v = sVal[k];
-        F8 pr = gather(0, k);
 #pragma unroll
-        for (int q = 1; q < G; ++q) {
-          const F8 a = gather(q, k);
-          f4mul_(pr.a, a.a);
-          if constexpr (VEC == 8) f4mul_(pr.b, a.b);
+          for (int q = 0; q < G; ++q) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+              const F8 a = gather(q, k + u);
+              if (q == 0) {
+                pr[u] = a;
+              } else {
+                f4mul_(pr[u].a, a.a);
+                if constexpr (VEC == 8) f4mul_(pr[u].b, a.b);
+              }
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            if (ii[u] != cur) {
+              flush();
+              cur = ii[u];
+            }
+            const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
+            f4fma_(acc0, vb, pr[u].a);
+            if constexpr (VEC == 8) f4fma_(acc1, vb, pr[u].b);
+          }
         }
-        if (i != cur) {
-          flush();
-          cur = i;
+        for (; k < k1; ++k) {
+          const uint32_t i = sOut[k];
+          const float v = sVal[k];
+          F8 pr = gather(0, k);
+#pragma unroll
+          for (int q = 1; q < G; ++q) {
+            const F8 a = gather(q, k);
+            f4mul_(pr.a, a.a);
+            if constexpr (VEC == 8) f4mul_(pr.b, a.b);
+          }
+          if (i != cur) {
+            flush();
+            cur = i;
+          }
+          const float4 vb = make_float4(v, v, v, v);
+          f4fma_(acc0, vb, pr.a);
+          if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
         }
-        const float4 vb = make_float4(v, v, v, v);
-        f4fma_(acc0, vb, pr.a);
-        if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
+        flush();
       }
-      flush();
+      __syncwarp();  // every lane is done reading stage st
+      if (lane == 0 && j + 2u * nwarps < seg_end) issue(j + 2u * nwarps, st);
     }
-    __syncthreads();  // stage s fully consumed
-    if (tid == 0 && j + kFragStages < j1) issue(j + kFragStages, s);
+    seg = seg_end;
   }
 }
 

@@ -21,9 +21,13 @@ namespace sf {
 
 static constexpr int kStagesHost = 2;  // must match frag_kernel's kStages
 
+// Shared memory of frag_kernel: mbarriers (2 per warp + 1), one double-buffered stage
+// ring of (N+1) x (C+8) words per warp (C = chunk_nnz, a per-warp chunk), factor blocks.
 size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l) {
   (void)mode;
-  size_t b = 128 + (size_t)kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
+  const size_t nwarps = (size_t)std::max(1, l.block_threads / 32);
+  size_t b = ((2 * nwarps + 1) * 8 + 127) & ~(size_t)127;
+  b += nwarps * kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
   for (int m = 0; m < t.nmodes; ++m)
     if (l.staged_mask & (1u << m)) b += (size_t)l.block_rows[m] * rank * 4;
   return b;
@@ -35,7 +39,7 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   if (l.kernel == SF_KERNEL_FRAG && !frag_supported(N, rank)) l.kernel = SF_KERNEL_COO;
   l.block_threads = std::min(1024, std::max(64, (l.block_threads / 32) * 32));
   if (l.ctas_per_sm < 0) l.ctas_per_sm = 0;
-  if (l.chunk_nnz <= 0) l.chunk_nnz = 1024;
+  if (l.chunk_nnz <= 0) l.chunk_nnz = 128;
   l.chunk_nnz = std::min(16384, std::max(16, (l.chunk_nnz + 3) / 4 * 4));
   uint32_t mask = 0;
   for (int m = 0; m < N; ++m) {
@@ -50,21 +54,29 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   l.staged_mask = (l.kernel == SF_KERNEL_FRAG) ? mask : 0u;
 }
 
-// Rough per-nonzero cost model in "on-chip bytes".
-struct Cand {
-  uint32_t mask;
-  uint32_t rows[SF_MAX_MODES];
-  double cost;
-};
+// Selector rules, calibrated on the sweeps in profiles/:
+//  * a gathered mode is staged WHOLE (one tile, loaded once per CTA) when its factor
+//    fits the shared-memory budget next to the stream stages;
+//  * otherwise a mode is staged in BLOCKS only if the factors are L2-resident (the
+//    tensor is "dense enough") and every staged row is reused often inside its tile:
+//    nnz * block_rows / I_m >= kMinReuse * block_rows  <=>  nnz / I_m >= kMinReuse
+//    (hyper-sparse tensors lose to block staging by up to 1000x: each tile would be
+//    staged for a handful of nonzeros);
+//  * at most one block-staged mode (two block-staged modes multiply the tile count and
+//    split output-row runs into short (tile,row) pieces whose flushes dominate);
+//  * per-warp chunks of C = 128 nonzeros, 512 threads (sweep optima, profiles/).
+static constexpr double kMinReuse = 256.0;
+static constexpr uint32_t kBlockRows = 256;
 
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank,
                           uint64_t nnz_local) {
+  (void)f;
   sf_launch_t l{};
   const int N = t.nmodes;
   l.kernel = frag_supported(N, rank) ? SF_KERNEL_FRAG : SF_KERNEL_COO;
   l.block_threads = 512;
   l.ctas_per_sm = 0;
-  l.chunk_nnz = 1024;
+  l.chunk_nnz = 128;
   l.staged_mask = 0;
   if (l.kernel != SF_KERNEL_FRAG || nnz_local == 0) {
     normalize_launch(t, mode, rank, l);
@@ -72,68 +84,42 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
   }
   const double R4 = 4.0 * rank;
   const double L2 = 96.0 * 1024 * 1024;  // usable L2 for factors (of ~126 MB)
-  const size_t base_smem = frag_smem_bytes(t, mode, rank, l);
-  const double budget_rows =
-      std::floor(((double)t.smem_optin - (double)base_smem - 1024.0) / R4);
-  double total_fac = 0;
+  double fac_bytes = 0;
   for (int m = 0; m < N; ++m)
-    if (m != mode) total_fac += (double)t.dims[m] * R4;
-  const double nnz = (double)nnz_local;
-  const double slices = std::max<double>(1.0, (double)f.num_slices);
-  Cand best{0, {}, 1e300};
-  const int G = N - 1;
-  int gm[SF_MAX_MODES], k = 0;
+    if (m != mode) fac_bytes += (double)t.dims[m] * R4;
+  // 1) whole-mode staging of small modes (largest first that fits)
+  // keep two CTAs per SM: half the shared memory per CTA
+  double budget = (double)t.smem_optin / 2 - (double)frag_smem_bytes(t, mode, rank, l) - 1024.0;
+  int order[SF_MAX_MODES], k = 0;
   for (int m = 0; m < N; ++m)
-    if (m != mode) gm[k++] = m;
-  for (uint32_t sub = 0; sub < (1u << G); ++sub) {
-    Cand c{0, {}, 0};
-    int ns = 0;
-    for (int q = 0; q < G; ++q)
-      if (sub & (1u << q)) { c.mask |= 1u << gm[q]; ++ns; }
-    // block rows: small modes whole, the rest share the remaining budget equally
-    double rows_left = budget_rows;
-    int left = ns;
-    bool ok = true;
-    std::vector<int> order;
-    for (int q = 0; q < G; ++q)
-      if (sub & (1u << q)) order.push_back(gm[q]);
-    std::sort(order.begin(), order.end(), [&](int a, int b) { return t.dims[a] < t.dims[b]; });
-    for (int m : order) {
-      const double share = std::floor(rows_left / left);
-      if (share < 64) { ok = false; break; }
-      const double r = std::min<double>((double)t.dims[m], share);
-      c.rows[m] = (uint32_t)r;
-      rows_left -= r;
-      --left;
+    if (m != mode) order[k++] = m;
+  std::sort(order, order + k, [&](int a, int b) { return t.dims[a] < t.dims[b]; });
+  for (int q = 0; q < k; ++q) {
+    const int m = order[q];
+    const double bytes = (double)t.dims[m] * R4;
+    if (bytes <= budget) {
+      l.staged_mask |= 1u << m;
+      l.block_rows[m] = (uint32_t)t.dims[m];
+      budget -= bytes;
     }
-    if (!ok) continue;
-    double T = 1;
-    double staged_rows = 0;
-    for (int m : order) {
-      T *= std::ceil((double)t.dims[m] / c.rows[m]);
-      staged_rows += c.rows[m];
-    }
-    double cost = 4.0 * (N + 1);  // stream bytes (HBM)
-    // gathers of non-staged modes: L2 hits ~1.0 per byte; misses to HBM much worse
-    double unstaged_fac = 0;
-    for (int q = 0; q < G; ++q)
-      if (!(sub & (1u << q))) unstaged_fac += (double)t.dims[gm[q]] * R4;
-    const double l2_w = unstaged_fac <= L2 ? 1.0 : 1.0 + 2.0 * (1.0 - L2 / unstaged_fac);
-    for (int q = 0; q < G; ++q)
-      if (!(sub & (1u << q))) cost += R4 * l2_w;
-    cost += ns * R4 * 0.35;                                   // shared-memory gathers
-    const double tiles_touched = std::min(T, nnz);
-    const double ctas = (double)t.num_sms;
-    cost += (staged_rows * R4) * (tiles_touched + ctas) / nnz;  // block staging traffic
-    const double pairs = std::min(nnz, tiles_touched * slices);  // (tile,row) runs
-    cost += R4 * 1.5 * (pairs / nnz + 0.05);                     // flush atomics
-    c.cost = cost;
-    if (c.cost < best.cost) best = c;
   }
-  l.staged_mask = best.mask;
-  for (int m = 0; m < N; ++m) l.block_rows[m] = (best.mask & (1u << m)) ? best.rows[m] : 0;
-  (void)total_fac;
+  // 2) one block-staged mode when factors are L2-resident and rows are reused enough
+  if (l.staged_mask == 0 && fac_bytes <= L2) {
+    int best = -1;
+    for (int q = 0; q < k; ++q) {
+      const int m = order[q];
+      if ((double)nnz_local / (double)t.dims[m] >= kMinReuse) { best = m; break; }
+    }
+    if (best >= 0) {
+      l.staged_mask = 1u << best;
+      l.block_rows[best] = kBlockRows;
+    }
+  }
   normalize_launch(t, mode, rank, l);
+  if (frag_smem_bytes(t, mode, rank, l) > t.smem_optin) {  // safety: drop staging
+    l.staged_mask = 0;
+    normalize_launch(t, mode, rank, l);
+  }
   return l;
 }
 

@@ -43,17 +43,18 @@ def time_launch(T, n, R, facs, out, L, sf, torch, reps=5):
 
 def grid(dims, n, R, quick):
     others = [m for m in range(len(dims)) if m != n]
-    row_opts = [256, 512, 775, 1024, 1536] if not quick else [512, 775]
-    chunks = [512, 1024, 2048] if not quick else [1024]
+    row_opts = [128, 256, 384, 512, 775] if not quick else [256, 512]
+    chunks = [64, 128, 256] if not quick else [128]
     threads = [256, 512, 1024] if not quick else [512]
     staged_sets = [()]
     for k in range(1, len(others) + 1):
         staged_sets += list(itertools.combinations(others, k))
     for st in staged_sets:
-        rows_choices = [()] if not st else itertools.product(row_opts, repeat=len(st))
+        opts = {m: sorted(set(row_opts + ([dims[m]] if dims[m] <= 2048 else []))) for m in st}
+        rows_choices = [()] if not st else itertools.product(*[opts[m] for m in st])
         for rows in rows_choices:
-            for C, th in itertools.product(chunks, threads):
-                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C,
+            for C, th, fl in itertools.product(chunks, threads, (0, 1)):
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl,
                        "staged": {m: min(r, dims[m]) for m, r in zip(st, rows)}}
     yield {"kernel": 1}
 
@@ -83,7 +84,8 @@ def main():
         t_pick, _ = time_launch(T, n, R, facs, out, sf.Launch.make(
             kernel=2 if pick["kernel"] == "frag" else 1, block_threads=pick["block_threads"],
             ctas_per_sm=pick["ctas_per_sm"], chunk_nnz=pick["chunk_nnz"],
-            staged={m: r for m, r in enumerate(pick["block_rows"]) if pick["staged_mask"] >> m & 1}),
+            staged={m: r for m, r in enumerate(pick["block_rows"]) if pick["staged_mask"] >> m & 1},
+            flags=pick.get("flags", 0)),
             sf, torch)
         results = []
         t0 = time.time()

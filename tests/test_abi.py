@@ -42,9 +42,10 @@ def test_status_strings_and_version():
 
 def test_struct_layouts_match_header():
     # sizes implied by include/scalfrag.h on LP64
-    assert ctypes.sizeof(sf.Launch) == 4 * 5 + 4 * 8
+    assert ctypes.sizeof(sf.Launch) == 4 * 5 + 4 * 8 + 4
     assert ctypes.sizeof(sf.Features) == 8 * 7 + 8 * 40 + 4 * 4 + 8 * 5
-    assert ctypes.sizeof(sf.PlanInfo) == ctypes.sizeof(sf.Features) + ctypes.sizeof(sf.Launch) + 4 + 8 * 7
+    head = ctypes.sizeof(sf.Features) + ctypes.sizeof(sf.Launch)
+    assert ctypes.sizeof(sf.PlanInfo) == head + (-head % 8) + 8 * 7
 
 
 def test_no_oracle_in_product_path():

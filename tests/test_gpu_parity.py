@@ -36,14 +36,16 @@ def test_configs0_all_modes_auto(cuda_device, name):
 
 
 def _launches(dims, n):
+    """Launch variants; chunk_nnz is a per-warp chunk."""
     others = [m for m in range(len(dims)) if m != n]
     yield sf.Launch.make(kernel=COO)
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={})
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=1024, block_threads=256, staged={})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=16, staged={})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=128, block_threads=256, staged={})
     # stage every gathered mode in small blocks: many tiles, ragged last block
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=128, staged={m: max(1, dims[m] // 3 + 1) for m in others})
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=256, block_threads=1024, staged={others[0]: 7})
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=4096, ctas_per_sm=1, staged={others[-1]: dims[others[-1]]})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=32, staged={m: max(1, dims[m] // 3 + 1) for m in others})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, block_threads=1024, staged={others[0]: 7})
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=256, block_threads=128, ctas_per_sm=1,
+                         staged={others[-1]: dims[others[-1]]})
 
 
 @pytest.mark.parametrize("name", ["tiny", "tiny_skew"])
