@@ -42,10 +42,13 @@ struct FragParams {
   uint32_t dims[SF_MAX_MODES];        // per mode
   uint32_t fac_off[SF_MAX_MODES];     // per staged slot: float offset of its block in smem
   uint32_t stage_words;               // words per field per pipeline stage
-  uint32_t prefetch;                  // 1: prefetch a stretch's global rows into L2 first
+  uint32_t prefetch;                  // launch flags: 1 L2 prefetch, 2 L1::no_allocate gathers
 };
 
 constexpr int kFragStages = 2;
+#ifndef SF_LDG256_OP
+#define SF_LDG256_OP "ld.global.nc.v8.f32"
+#endif
 constexpr int kFragUnroll = 4;
 
 namespace detail {
@@ -68,6 +71,17 @@ __device__ __forceinline__ float4 lds128(uint32_t addr) {
 }
 
 __device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
+
+__device__ __forceinline__ void ldg256(const float4* p, float4& a, float4& b) {
+  asm(SF_LDG256_OP " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+      : "l"(p));
+}
+__device__ __forceinline__ void ldg256_na(const float4* p, float4& a, float4& b) {
+  asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+      : "l"(p));
+}
 
 __device__ __forceinline__ void prefetch_l2(const void* p) {
   asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
@@ -105,27 +119,16 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 }  // namespace detail
 
 // Lane mapping.  VEC = floats per lane (4 for R <= 16, else 8), LPN = R / VEC lanes per
-// nonzero.  A lane owns the two (VEC = 8) or one (VEC = 4) 16-byte chunks c0, c1 of a
-// factor row.  R = 32: the two groups of a quarter-warp read complementary chunk sets
-// (group parity p: c0 = 2t+p, c1 = 2t+1-p), so every 128-bit shared load of a
-// quarter-warp touches all 32 banks once; R >= 64: c0 = t, c1 = t + LPN.
+// nonzero.  VEC = 8: lane t owns the 32 contiguous bytes of 16-byte chunks 2t, 2t+1 of a
+// factor row: a global gather is ONE 256-bit load (ld.global.nc.v8.f32, sm_100), and a
+// shared-memory gather is two 128-bit loads issued in parity order (quarter-warp
+// half p = (lane>>2)&1 reads chunk 2t+p first), so the 8 lanes of a quarter-warp touch
+// all 32 banks exactly once per load; the pair is swapped back into (2t, 2t+1).
+// VEC = 4: lane t owns chunk t.
 template <int R>
 struct LaneMap {
   static constexpr int VEC = (R >= 32) ? 8 : 4;
   static constexpr int LPN = R / VEC;
-  __device__ __forceinline__ static void chunks(int t, int group, int& c0, int& c1) {
-    if constexpr (VEC == 4) {
-      c0 = t;
-      c1 = t;
-    } else if constexpr (R == 32) {
-      const int par = group & 1;
-      c0 = 2 * t + par;
-      c1 = 2 * t + 1 - par;
-    } else {
-      c0 = t;
-      c1 = t + LPN;
-    }
-  }
 };
 
 struct F8 {
@@ -161,8 +164,9 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   const int nwarps = blockDim.x >> 5;
   const int lane_in_group = lane % LPN;
   const int group = lane / LPN;  // group within the warp
-  int c0, c1;
-  LM::chunks(lane_in_group, group, c0, c1);
+  const int c0 = (VEC == 8) ? 2 * lane_in_group : lane_in_group;  // first owned 16-B chunk
+  const int par = (lane >> 2) & 1;                                 // smem issue order (VEC 8)
+  const bool l1na = (p.prefetch & 2u) != 0;                        // gathers skip L1 allocation
 
   // smem: [bars: 2 per warp + 1 factor barrier, 128-B aligned] [per-warp stage rings] [factor blocks]
   const uint32_t SW = p.stage_words;
@@ -281,25 +285,32 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
 #pragma unroll
         for (int q = 0; q < G; ++q) sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * SW);
         float* out0 = p.out + 4 * c0;
-        float* out1 = p.out + 4 * c1;
+        float* out1 = out0 + 4;
         // gather slot q of nonzero kk (staged: shared memory, else global via L1/L2)
         auto gather = [&](int q, uint32_t kk) -> F8 {
           const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
           const size_t row = (size_t)sIdx[q][kk] * R4;
           F8 r;
-          if (q < S) {
-            r.a = base[row + c0];
-            if constexpr (VEC == 8) r.b = base[row + c1];
+          if constexpr (VEC == 8) {
+            if (q < S) {
+              const float4 x = base[row + c0 + par];
+              const float4 y = base[row + c0 + 1 - par];
+              r.a = par ? y : x;
+              r.b = par ? x : y;
+            } else if (l1na) {
+              ldg256_na(base + row + c0, r.a, r.b);
+            } else {
+              ldg256(base + row + c0, r.a, r.b);
+            }
           } else {
-            r.a = ldg128(base + row + c0);
-            if constexpr (VEC == 8) r.b = ldg128(base + row + c1);
+            r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
           }
           return r;
         };
         // Memory-level parallelism without registers: request every global row of this
         // stretch into L2 up front (one 32-byte sector per lane), then gather.
         if constexpr (G - S > 0) {
-          if (p.prefetch && (VEC == 8 || (lane_in_group & 1) == 0)) {
+          if ((p.prefetch & 1u) && (VEC == 8 || (lane_in_group & 1) == 0)) {
             for (uint32_t kk = k0; kk < k1; ++kk) {
 #pragma unroll
               for (int q = S; q < G; ++q)

@@ -5,9 +5,9 @@
 // model.  The model will output an optimal launch parameter combination".  The paper's
 // model is a DecisionTree regressor trained on sweeps of its RTX 3090 kernel (L197);
 // that model and its training data are prior art for another GPU and another kernel.
-// Here the selector is an analytic cost model over the features of PAPER.md L195 plus
-// dims / nnz / R / shared-memory capacity, and it is validated against an exhaustive
-// launch sweep (tests/test_gpu_select.py, bench.py --sweep).
+// Here the selector is a set of rules over the features of PAPER.md L195 plus dims /
+// nnz / R / shared-memory capacity, calibrated on and validated against an exhaustive
+// launch sweep (sweep.py; DESIGN.md §5 Selector).
 //
 // Decision: which gathered factors to stage in shared memory as blocks ("tensor
 // blocks ... based on the resource constraints of hardware") and the
@@ -78,6 +78,7 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
   l.ctas_per_sm = 0;
   l.chunk_nnz = 128;
   l.staged_mask = 0;
+  l.flags = SF_LAUNCH_L1_NO_ALLOCATE;  // measured: -1..-8% time on every config swept
   if (l.kernel != SF_KERNEL_FRAG || nnz_local == 0) {
     normalize_launch(t, mode, rank, l);
     return l;
