@@ -9,9 +9,9 @@ Definitions (readings R9-R12):
 
 * Matricized order ("ScalFrag first matricizes the input tensor
   and then chunks the matricized tensor"): nonzeros sorted stably by the key
-  (i_n, i_s), where i_s is the highest-numbered mode != n -- the most
-  significant part of the X_(n) column index in Kolda-Bader order (reading
-  R3/R10).  Ties keep input order.
+  (i_n, i_s), where s is the gathered mode with the smallest dimension (ties:
+  the higher mode index) -- the fiber key with the most reuse of A_s rows
+  (reading R10).  Ties keep input order.
 * Shards (multi-GPU): rank p of P owns matricized positions
   [floor(p*nnz/P), floor((p+1)*nnz/P)).
 * Tiles ("tensor blocks ... based on the resource constraints of hardware",
@@ -30,13 +30,18 @@ from __future__ import annotations
 import numpy as np
 
 
-def secondary_mode(nmodes: int, mode: int) -> int:
-    return max(m for m in range(nmodes) if m != mode)
+def secondary_mode(nmodes: int, mode: int, dims=None) -> int:
+    """DESIGN.md reading R10: the gathered mode with the smallest dimension (ties: the
+    higher mode index); without dims, the highest-numbered mode != n."""
+    others = [m for m in range(nmodes) if m != mode]
+    if dims is None:
+        return max(others)
+    return min(others, key=lambda m: (int(dims[m]), -m))
 
 
 def matricized_order(dims, inds, mode):
     """Stable argsort by (i_n, i_s)  (uint64 key i_n * I_s + i_s)."""
-    s = secondary_mode(len(dims), mode)
+    s = secondary_mode(len(dims), mode, dims)
     key = inds[mode].astype(np.uint64) * np.uint64(dims[s]) + inds[s].astype(np.uint64)
     return np.argsort(key, kind="stable").astype(np.int64)
 
@@ -89,7 +94,7 @@ def features(dims, inds, mode):
     N = len(dims)
     In = int(dims[mode])
     nnz = len(inds[0])
-    s = secondary_mode(N, mode)
+    s = secondary_mode(N, mode, dims)
     cnt = np.bincount(inds[mode].astype(np.int64), minlength=In) if nnz else np.zeros(In, np.int64)
     nz = cnt[cnt > 0]
     key = inds[mode].astype(np.uint64) * np.uint64(dims[s]) + inds[s].astype(np.uint64)

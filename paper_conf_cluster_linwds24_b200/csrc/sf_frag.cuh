@@ -166,7 +166,6 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   const int group = lane / LPN;  // group within the warp
   const int c0 = (VEC == 8) ? 2 * lane_in_group : lane_in_group;  // first owned 16-B chunk
   const int par = (lane >> 2) & 1;                                 // smem issue order (VEC 8)
-  const bool l1na = (p.prefetch & 2u) != 0;                        // gathers skip L1 allocation
 
   // smem: [bars: 2 per warp + 1 factor barrier, 128-B aligned] [per-warp stage rings] [factor blocks]
   const uint32_t SW = p.stage_words;
@@ -297,10 +296,8 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
               const float4 y = base[row + c0 + 1 - par];
               r.a = par ? y : x;
               r.b = par ? x : y;
-            } else if (l1na) {
-              ldg256_na(base + row + c0, r.a, r.b);
             } else {
-              ldg256(base + row + c0, r.a, r.b);
+              ldg256_na(base + row + c0, r.a, r.b);  // L1::no_allocate (measured faster)
             }
           } else {
             r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);

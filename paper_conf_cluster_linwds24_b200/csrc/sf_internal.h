@@ -92,6 +92,18 @@ struct Tensor {
   ~Tensor();
 };
 
+// Secondary sort key of mode n (reading R10): the gathered mode with the
+// smallest dimension (ties: the higher mode index) -- the (i_n, i_s) fibers with the most
+// reuse of A_s rows.
+inline int secondary_mode(const Tensor& t, int mode) {
+  int s = -1;
+  for (int m = 0; m < t.nmodes; ++m) {
+    if (m == mode) continue;
+    if (s < 0 || t.dims[m] <= t.dims[s]) s = m;
+  }
+  return s;
+}
+
 // ---- planning (sf_plan.cu) ----
 void compute_features(Tensor& t, int mode, sf_features_t* out);
 void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch);

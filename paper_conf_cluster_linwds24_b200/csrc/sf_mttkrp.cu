@@ -277,7 +277,7 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   fp.nnz = (uint32_t)p.nnz_local;
   fp.mode = n;
   fp.stage_words = (uint32_t)p.launch.chunk_nnz + 8;
-  fp.prefetch = p.launch.flags & (SF_LAUNCH_PREFETCH_L2 | SF_LAUNCH_L1_NO_ALLOCATE);
+  fp.prefetch = p.launch.flags & SF_LAUNCH_PREFETCH_L2;
   // slots: staged modes first (ascending mode id = tile-id fold order), then the rest
   int S = 0, q = 0;
   uint32_t off = 0;
@@ -293,6 +293,7 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
     }
   for (int m = 0; m < N; ++m)
     if (m != n && !(p.launch.staged_mask & (1u << m))) fp.slot_mode[q++] = m;
+
   const size_t smem = frag_smem_bytes(t, n, R, p.launch);
   const int threads = p.launch.block_threads;
   int per_sm = p.launch.ctas_per_sm;

@@ -5,7 +5,7 @@
 // launch parameters based on the sparsity features of the matrixed tensor after
 // chunking."  Here, per (mode n, rank):
 //   1. matricized order: stable LSD radix sort of the key i_n * I_s + i_s with the
-//      input position as payload (s = highest mode != n; reading R10);
+//      input position as payload (s = smallest gathered mode; reading R10);
 //   2. features from run lengths of that order;
 //   3. shard cut [floor(p*nnz/P), floor((p+1)*nnz/P)) of that order (§8(e));
 //   4. tiles ("tensor blocks ... based on the resource constraints of hardware",
@@ -131,9 +131,7 @@ struct MaxOp {
 // Matricized sort of the whole tensor for `mode`. Returns sorted keys + positions.
 static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_out) {
   const uint64_t n = t.nnz;
-  int s = 0;
-  for (int m = 0; m < t.nmodes; ++m)
-    if (m != mode) s = m;
+  const int s = secondary_mode(t, mode);
   const uint64_t Is = t.dims[s];
   DevBuf k0(n * 8 + 16), k1(n * 8 + 16), p0(n * 4 + 16), p1(n * 4 + 16);
   key_matricized_kernel<<<grid_for(n), 256, 0, t.stream>>>(t.ind[mode].as<uint32_t>(),
@@ -155,9 +153,7 @@ static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_o
 
 static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_features_t* f) {
   const uint64_t n = t.nnz;
-  int s = 0;
-  for (int m = 0; m < t.nmodes; ++m)
-    if (m != mode) s = m;
+  const int s = secondary_mode(t, mode);
   const uint64_t Is = t.dims[s];
   memset(f, 0, sizeof(*f));
   f->nnz = n;
@@ -319,9 +315,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   }
   p.feat = t.features[mode];
 
-  int s = 0;
-  for (int m = 0; m < N; ++m)
-    if (m != mode) s = m;
+  const int s = secondary_mode(t, mode);
   p.row_begin = p.row_end = 0;
   if (nl) {
     uint64_t kb, ke;

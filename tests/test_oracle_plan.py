@@ -19,7 +19,9 @@ def test_matricized_order_brute(dims):
     inds = _coo(1, dims, 700)
     N = len(dims)
     for n in range(N):
-        s = max(m for m in range(N) if m != n)
+        # reading R10: secondary = smallest gathered dim, ties -> higher mode index
+        cand = [m for m in range(N) if m != n]
+        s = sorted(cand, key=lambda m: (dims[m], -m))[0]
         ref = sorted(range(700), key=lambda e: (int(inds[n][e]), int(inds[s][e]), e))
         assert list(plan.matricized_order(dims, inds, n)) == ref
 
@@ -31,7 +33,7 @@ def test_plan_order_tiles_and_shards_brute(nranks):
     staged = (1, 2)
     br = {1: 8, 2: 10}
     for n in (0,):
-        s = 2
+        s = 1  # smallest gathered dim (33 < 57)
         base = sorted(range(900), key=lambda e: (int(inds[n][e]), int(inds[s][e]), e))
         allpos = []
         for p in range(nranks):
@@ -78,7 +80,7 @@ def test_features_brute():
     inds = _coo(4, dims, 3000)
     for n in range(3):
         f = plan.features(dims, inds, n)
-        s = max(m for m in range(3) if m != n)
+        s = sorted([m for m in range(3) if m != n], key=lambda m: (dims[m], -m))[0]
         sl, fb = {}, {}
         for e in range(3000):
             i = int(inds[n][e])
