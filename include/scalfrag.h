@@ -75,6 +75,7 @@ typedef struct {
                             without registers) */
 } sf_launch_t;
 #define SF_LAUNCH_PREFETCH_L2 1u
+#define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation
                                        (ld.global.nc.L1::no_allocate.v8.f32; measured faster) */
 

@@ -22,6 +22,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 #include "sf_internal.h"
 
 namespace sf {
@@ -42,7 +44,9 @@ struct FragParams {
   uint32_t dims[SF_MAX_MODES];        // per mode
   uint32_t fac_off[SF_MAX_MODES];     // per staged slot: float offset of its block in smem
   uint32_t stage_words;               // words per field per pipeline stage
-  uint32_t prefetch;                  // launch flags: 1 L2 prefetch, 2 L1::no_allocate gathers
+  uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
+  uint32_t row_end;                   // this shard's rows end (exclusive)
+  uint32_t prefetch;                  // launch flags: 1 L2 prefetch
 };
 
 constexpr int kFragStages = 2;
@@ -51,7 +55,25 @@ constexpr int kFragStages = 2;
 #endif
 constexpr int kFragUnroll = 4;
 
+// Lane-group stretch of a chunk of n nonzeros (shared with the A5 boundary pre-pass):
+// ceil(n / GPW) bumped so the GPW groups of a warp, reading word g*L + k, hit distinct
+// banks (gcd(L, 32) <= LPN).
+__host__ __device__ __forceinline__ uint32_t stretch_len(uint32_t n, uint32_t GPW, uint32_t LPN) {
+  uint32_t L = (n + GPW - 1) / GPW;
+  if (LPN < 32)
+    while (L % (2u * LPN) == 0u) ++L;
+  return L;
+}
+
 namespace detail {
+
+__device__ __forceinline__ void st256(float* p, const float4& a, const float4& b) {
+  asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(a.x), "f"(a.y), "f"(a.z),
+               "f"(a.w), "f"(b.x), "f"(b.y), "f"(b.z), "f"(b.w));
+}
+__device__ __forceinline__ void st128(float* p, const float4& a) {
+  asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(a.x), "f"(a.y), "f"(a.z), "f"(a.w));
+}
 
 __device__ __forceinline__ void red_add_v4_nomem(float* addr, const float4& v) {
   asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(addr), "f"(v.x), "f"(v.y), "f"(v.z),
@@ -271,10 +293,7 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
       const uint32_t b = __ldg(p.chunk_begin + j), e = __ldg(p.chunk_begin + j + 1);
       const uint32_t n = e - b;
       const float* sb = ring + (size_t)st * (N + 1) * SW + (b - (b & ~3u));
-      uint32_t L = (n + GPW - 1) / GPW;
-      // the GPW groups of a warp read word g*L + k: distinct banks iff gcd(L,32) <= LPN
-      if (LPN < 32)
-        while (L % (2u * LPN) == 0u) ++L;
+      const uint32_t L = stretch_len(n, GPW, LPN);
       const uint32_t k0 = group * L;
       const uint32_t k1 = min(n, k0 + L);
       if (k0 < k1) {
@@ -317,11 +336,55 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
         }
         uint32_t cur = sOut[k0];
         float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
-        auto flush = [&]() {
-          red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
-          if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
+        // A5 (owner mode, unstaged plans only): runs wholly inside this stretch are
+        // STORED (this group owns the row); the stretch's first/last run is atomically
+        // added when it continues into the neighbouring stretch (those rows were zeroed by
+        // the boundary pre-pass); empty rows between runs are zeroed by the group that
+        // owns the run after the gap.  Otherwise (staged tiles) Y was memset and every
+        // flush is an atomic.
+        bool shared = true;       // current run may be shared with another stretch/tile
+        bool last_shared = true;  // the stretch's last run continues past k1
+        if constexpr (S == 0) {
+          if (p.owner) {
+            const uint32_t P0 = b + k0, P1 = b + k1;
+            const uint32_t* gOut = p.ind[p.mode];
+            const uint32_t first = sOut[k0];
+            const uint32_t before = (P0 > 0) ? __ldg(gOut + P0 - 1) : 0xFFFFFFFFu;
+            shared = (P0 > 0) && before == first;
+            last_shared = (P1 < p.nnz) && __ldg(gOut + P1) == sOut[k1 - 1];
+            if (!shared && P0 > 0)  // gap rows (before, first) belong to this group
+              for (uint32_t r = before + 1; r < first; ++r) {
+                if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
+                                              make_float4(0.f, 0.f, 0.f, 0.f));
+                else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
+              }
+          }
+        }
+        auto flush_run = [&](bool atomic) {
+          if (atomic) {
+            red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
+            if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
+          } else {
+            if constexpr (VEC == 8) st256(out0 + (size_t)cur * R, acc0, acc1);
+            else st128(out0 + (size_t)cur * R, acc0);
+          }
           acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
           acc1 = acc0;
+        };
+        // run edge inside the stretch: close `cur`, zero the gap up to the next row i
+        auto flush = [&]() { flush_run(shared); };
+        auto advance = [&](uint32_t i) {
+          if constexpr (S == 0) {
+            if (p.owner) {
+              for (uint32_t r = cur + 1; r < i; ++r) {
+                if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
+                                              make_float4(0.f, 0.f, 0.f, 0.f));
+                else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
+              }
+              shared = false;
+            }
+          }
+          cur = i;
         };
         uint32_t k = k0;
         // y += v * (a_0 * ... * a_{G-1}): G-1 FMUL + 1 FFMA per float
@@ -351,7 +414,7 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
           for (int u = 0; u < U; ++u) {
             if (ii[u] != cur) {
               flush();
-              cur = ii[u];
+              advance(ii[u]);
             }
             const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
             f4fma_(acc0, vb, pr[u].a);
@@ -370,13 +433,13 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
           }
           if (i != cur) {
             flush();
-            cur = i;
+            advance(i);
           }
           const float4 vb = make_float4(v, v, v, v);
           f4fma_(acc0, vb, pr.a);
           if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
         }
-        flush();
+        flush_run(shared || last_shared);
       }
       __syncwarp();  // every lane is done reading stage st
       if (lane == 0 && j + 2u * nwarps < seg_end) issue(j + 2u * nwarps, st);
@@ -385,11 +448,37 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   }
 }
 
+// A5 pre-pass for owner mode: zero the rows whose run crosses a stretch boundary (they
+// receive atomic partial sums), i.e. rows(pos) with row(pos) == row(pos-1) at every
+// stretch start pos.  One thread per (chunk, group).
+template <int R>
+__global__ void boundary_zero_kernel(const uint32_t* __restrict__ chunk_begin, uint32_t num_chunks,
+                                     const uint32_t* __restrict__ rows, float* __restrict__ out) {
+  using LM = LaneMap<R>;
+  constexpr uint32_t GPW = 32 / LM::LPN;
+  const uint64_t total = (uint64_t)num_chunks * GPW;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
+    const uint32_t j = (uint32_t)(t / GPW), g = (uint32_t)(t % GPW);
+    const uint32_t b = chunk_begin[j], e = chunk_begin[j + 1];
+    const uint32_t pos = b + g * stretch_len(e - b, GPW, LM::LPN);
+    if (pos >= e || pos == 0) continue;
+    const uint32_t r = rows[pos];
+    if (rows[pos - 1] != r) continue;
+    float4* y = reinterpret_cast<float4*>(out + (size_t)r * R);
+#pragma unroll
+    for (int c = 0; c < R / 4; ++c) y[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
 // Per-R dispatch (defined in sf_frag_r{16,32,64}.cu).
 void frag_launch_r16(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
 void frag_launch_r32(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
 void frag_launch_r64(int N, int S, const FragParams& fp, int grid, int threads, size_t smem, cudaStream_t s);
 int frag_occ_r16(int N, int S, int threads, size_t smem);
+void boundary_zero_r16(const uint32_t* cb, uint32_t nc, const uint32_t* rows, float* out, cudaStream_t s);
+void boundary_zero_r32(const uint32_t* cb, uint32_t nc, const uint32_t* rows, float* out, cudaStream_t s);
+void boundary_zero_r64(const uint32_t* cb, uint32_t nc, const uint32_t* rows, float* out, cudaStream_t s);
 int frag_occ_r32(int N, int S, int threads, size_t smem);
 int frag_occ_r64(int N, int S, int threads, size_t smem);
 
@@ -438,6 +527,12 @@ int frag_occ_one(int threads, size_t smem) {
   int frag_occ_r##R(int N, int S, int threads, size_t smem) {                                            \
     SF_FRAG_NS_SWITCH(R, frag_occ_one, threads, smem);                                                   \
     return 0;                                                                                            \
+  }                                                                                                      \
+  void boundary_zero_r##R(const uint32_t* cb, uint32_t nc, const uint32_t* rows, float* out,            \
+                          cudaStream_t s) {                                                              \
+    const uint64_t total = (uint64_t)nc * (32 / LaneMap<R>::LPN);                                        \
+    const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((total + 255) / 256, 148 * 16));     \
+    boundary_zero_kernel<R><<<grid, 256, 0, s>>>(cb, nc, rows, out);                                    \
   }
 
 }  // namespace sf

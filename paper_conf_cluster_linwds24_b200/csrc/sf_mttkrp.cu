@@ -254,10 +254,30 @@ static void frag_launch(int N, int R, int S, const FragParams& fp, int grid, int
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
                    cudaStream_t s) {
   const int N = t.nmodes, R = p.rank, n = p.mode;
-  // A5 (v1): zero the output, then every flush is an atomic add.
-  SF_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * t.dims[n] * (size_t)R, s));
+  const bool frag = p.launch.kernel == SF_KERNEL_FRAG && frag_supported(N, R);
+  // A5: unstaged fragment plans run in owner mode (whole runs stored, gaps zeroed by
+  // their owner, only run-crossing rows pre-zeroed); everything else zeroes Y and adds.
+  const bool owner = frag && p.launch.staged_mask == 0 && p.nnz_local > 0 &&
+                     !(p.launch.flags & SF_LAUNCH_NO_OWNER_STORES);
+  const size_t row_bytes = sizeof(float) * (size_t)R;
+  if (!owner) {
+    SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * t.dims[n], s));
+  } else {
+    if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
+    if (p.row_end < t.dims[n])
+      SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (t.dims[n] - p.row_end), s));
+    const uint32_t* cb = p.chunk_begin.as<uint32_t>();
+    const uint32_t* rows = p.ind[n].as<uint32_t>();
+    switch (R) {
+      case 16: boundary_zero_r16(cb, (uint32_t)p.num_chunks, rows, out, s); break;
+      case 32: boundary_zero_r32(cb, (uint32_t)p.num_chunks, rows, out, s); break;
+      default: boundary_zero_r64(cb, (uint32_t)p.num_chunks, rows, out, s); break;
+    }
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+  }
   if (p.nnz_local == 0) return;
-  if (p.launch.kernel == SF_KERNEL_COO || !frag_supported(N, R)) {
+  if (!frag) {
     uint32_t* ind[SF_MAX_MODES];
     for (int m = 0; m < N; ++m) ind[m] = p.ind[m].as<uint32_t>();
     launch_coo(N, t.dims, p.nnz_local, ind, p.val.as<float>(), factors, R, n, out, s);
@@ -278,6 +298,8 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   fp.mode = n;
   fp.stage_words = (uint32_t)p.launch.chunk_nnz + 8;
   fp.prefetch = p.launch.flags & SF_LAUNCH_PREFETCH_L2;
+  fp.owner = owner ? 1u : 0u;
+  fp.row_end = (uint32_t)p.row_end;
   // slots: staged modes first (ascending mode id = tile-id fold order), then the rest
   int S = 0, q = 0;
   uint32_t off = 0;

@@ -57,9 +57,8 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
 // Selector rules, calibrated on the sweeps in profiles/:
 //  * a gathered mode is staged WHOLE (one tile, loaded once per CTA) when its factor
 //    fits the shared-memory budget next to the stream stages;
-//  * otherwise a mode is staged in BLOCKS only if the factors are L2-resident (the
-//    tensor is "dense enough") and every staged row is reused often inside its tile:
-//    nnz * block_rows / I_m >= kMinReuse * block_rows  <=>  nnz / I_m >= kMinReuse
+//  * otherwise the gathered mode with the most reuse is staged in BLOCKS if every staged
+//    row is reused often inside its tile: nnz / I_m >= kMinReuse
 //    (hyper-sparse tensors lose to block staging by up to 1000x: each tile would be
 //    staged for a handful of nonzeros);
 //  * at most one block-staged mode (two block-staged modes multiply the tile count and
@@ -84,10 +83,6 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
     return l;
   }
   const double R4 = 4.0 * rank;
-  const double L2 = 96.0 * 1024 * 1024;  // usable L2 for factors (of ~126 MB)
-  double fac_bytes = 0;
-  for (int m = 0; m < N; ++m)
-    if (m != mode) fac_bytes += (double)t.dims[m] * R4;
   // 1) whole-mode staging of small modes (largest first that fits)
   // keep two CTAs per SM: half the shared memory per CTA
   double budget = (double)t.smem_optin / 2 - (double)frag_smem_bytes(t, mode, rank, l) - 1024.0;
@@ -104,12 +99,17 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
       budget -= bytes;
     }
   }
-  // 2) one block-staged mode when factors are L2-resident and rows are reused enough
-  if (l.staged_mask == 0 && fac_bytes <= L2) {
+  // 2) otherwise block-stage the gathered mode whose rows are reused most, if every staged
+  //    row is reused >= kMinReuse times on average (nnz / I_m)
+  if (l.staged_mask == 0) {
     int best = -1;
+    double reuse = 0;
     for (int q = 0; q < k; ++q) {
       const int m = order[q];
-      if ((double)nnz_local / (double)t.dims[m] >= kMinReuse) { best = m; break; }
+      const double r = (double)nnz_local / (double)t.dims[m];
+      // tiny factors (< 512 KB) stay hot in L1/L2 anyway: staging them only costs smem
+      if ((double)t.dims[m] * R4 < 512.0 * 1024) continue;
+      if (r >= kMinReuse && r > reuse) { best = m; reuse = r; }
     }
     if (best >= 0) {
       l.staged_mask = 1u << best;
