@@ -144,6 +144,21 @@ sf_status sf_plan_info(sf_tensor_t t, int mode, int rank, sf_plan_info_t* out);
 sf_status sf_plan_export(sf_tensor_t t, int mode, int rank, uint64_t* perm_host,
                          uint64_t* chunks_host);
 
+/* ---- learned launch selector (§IV-B) ---- */
+
+#define SF_SELECTOR_MAX_FEATURES 32
+#define SF_SELECTOR_MAX_CANDIDATES 16
+/* The selector's feature vector for (mode, rank) of this handle/shard (log2-scaled sizes,
+ * PAPER.md L195 features); returns the count in *n (<= SF_SELECTOR_MAX_FEATURES). */
+sf_status sf_selector_features(sf_tensor_t t, int mode, int rank, double* x, int* n);
+/* The discrete launch classes the learned model chooses among (class id = index). */
+sf_status sf_selector_candidates(sf_tensor_t t, int mode, int rank, sf_launch_t* out, int* n);
+/* Install a decision tree (sklearn tree_ layout: node arrays; leaf iff left < 0; value =
+ * class id).  n_nodes = 0 removes it (rule-based selection).  Process-global; later
+ * sf_plan calls use it.  Copies the arrays. */
+sf_status sf_set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
+                                const int32_t* right, const int32_t* value, int n_nodes, int n_features);
+
 /* ---- the hot path (§8(a) A5-A7) ---------------------------------------- */
 
 /* Y = mode-`mode` MTTKRP.  factors: host array of nmodes DEVICE pointers (factors[mode]

@@ -96,7 +96,8 @@ class PlanInfo(ctypes.Structure):
 EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
             "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
             "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
-            "sf_kernel_launches", "sf_version", "sf_rows_op"]
+            "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
+            "sf_selector_candidates", "sf_set_selector_model"]
 
 
 def lib(build_if_missing: bool = True):
@@ -123,9 +124,13 @@ def lib(build_if_missing: bool = True):
             L.sf_mttkrp.argtypes = [P, I, P, I, P, P]
             L.sf_mttkrp_streamed.argtypes = [I, P, U64, P, P, P, I, I, P, I, I]
             L.sf_rows_op.argtypes = [P, I, P, P, I, I, P]
+            L.sf_selector_features.argtypes = [P, I, I, P, ctypes.POINTER(I)]
+            L.sf_selector_candidates.argtypes = [P, I, I, P, ctypes.POINTER(I)]
+            L.sf_set_selector_model.argtypes = [P, P, P, P, P, I, I]
             for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
                        "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
-                       "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op"]:
+                       "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op", "sf_selector_features",
+                       "sf_selector_candidates", "sf_set_selector_model"]:
                 getattr(L, fn).restype = ctypes.c_int
             L.sf_status_string.argtypes = [I]
             L.sf_status_string.restype = ctypes.c_char_p
@@ -136,7 +141,46 @@ def lib(build_if_missing: bool = True):
             L.sf_version.argtypes = []
             L.sf_version.restype = ctypes.c_char_p
             _lib = L
+        if _lib is not None and not getattr(lib, "_model_loaded", False):
+            lib._model_loaded = True
+            if os.environ.get("SF_SELECTOR", DEFAULT_SELECTOR) == "model" and os.path.exists(MODEL_PATH):
+                _install_model(_lib, MODEL_PATH)
     return _lib
+
+
+MODEL_PATH = os.path.join(_HERE, "selector_model.json")
+# "rules" (sf_select.cpp, calibrated on sweeps) or "model" (the learned DecisionTree,
+# tools/train_selector.py).  See DESIGN.md §5 for the held-out comparison that sets this.
+DEFAULT_SELECTOR = "rules"
+
+
+def _install_model(L, path):
+    """Install the learned launch selector (tools/train_selector.py) into the library."""
+    import json
+    import numpy as np
+    m = json.load(open(path))
+    t = m["tree"]
+    arrs = [np.ascontiguousarray(t[k], dtype=dt) for k, dt in
+            (("feature", np.int32), ("threshold", np.float64), ("left", np.int32), ("right", np.int32),
+             ("value", np.int32))]
+    rc = L.sf_set_selector_model(*[a.ctypes.data for a in arrs], len(arrs[0]), int(m["n_features"]))
+    if rc != 0:
+        raise SfError(rc, L.sf_last_error().decode())
+
+
+def set_selector_model(model):
+    """model: dict with 'tree' (feature/threshold/left/right/value lists) and 'n_features',
+    or None to fall back to the rule-based selector."""
+    L = lib()
+    if model is None:
+        _check(L.sf_set_selector_model(None, None, None, None, None, 0, 0))
+        return
+    import json
+    import tempfile
+    with tempfile.NamedTemporaryFile("w", suffix=".json", delete=False) as f:
+        json.dump(model, f)
+    _install_model(L, f.name)
+    os.unlink(f.name)
 
 
 def _check(rc):
@@ -236,6 +280,23 @@ class Tensor:
         _check(lib().sf_plan_export(self._h, int(mode), int(rank), perm.ctypes.data if perm.size else None,
                                     chunks.ctypes.data if chunks.size else None))
         return perm, chunks
+
+    def selector_features(self, mode, rank):
+        x = (ctypes.c_double * 32)()
+        n = ctypes.c_int(0)
+        _check(lib().sf_selector_features(self._h, int(mode), int(rank), x, ctypes.byref(n)))
+        return [x[i] for i in range(n.value)]
+
+    def selector_candidates(self, mode, rank):
+        arr = (Launch * 16)()
+        n = ctypes.c_int(0)
+        _check(lib().sf_selector_candidates(self._h, int(mode), int(rank), arr, ctypes.byref(n)))
+        out = []
+        for i in range(n.value):
+            l = Launch()
+            ctypes.memmove(ctypes.byref(l), ctypes.byref(arr[i]), ctypes.sizeof(Launch))
+            out.append(l)
+        return out
 
     def mttkrp(self, mode, factors, out, rank=None, stream=None):
         """out <- mode-`mode` MTTKRP (device tensors; stream-ordered)."""

@@ -457,6 +457,43 @@ sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int co
   });
 }
 
+sf_status sf_selector_features(sf_tensor_t h, int mode, int rank, double* x, int* n) {
+  return guard([&]() -> sf_status {
+    if (!h || !x || !n) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    SF_CUDA(cudaSetDevice(t->device));
+    sf_features_t f;
+    compute_features(*t, mode, &f);
+    const uint64_t lo = (uint64_t)(((unsigned __int128)t->rank * t->nnz) / t->nranks);
+    const uint64_t hi = (uint64_t)(((unsigned __int128)(t->rank + 1) * t->nnz) / t->nranks);
+    *n = selector_features(*t, f, mode, rank, hi - lo, x);
+    return SF_OK;
+  });
+}
+
+sf_status sf_selector_candidates(sf_tensor_t h, int mode, int rank, sf_launch_t* out, int* n) {
+  return guard([&]() -> sf_status {
+    if (!h || !out || !n) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    *n = selector_candidates(*t, mode, rank, out);
+    return SF_OK;
+  });
+}
+
+sf_status sf_set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
+                                const int32_t* right, const int32_t* value, int n_nodes, int n_features) {
+  return guard([&]() -> sf_status {
+    if (n_nodes < 0 || (n_nodes > 0 && (!feature || !threshold || !left || !right || !value)))
+      throw StatusError{SF_ERR_INVALID_ARG, "bad model arrays"};
+    for (int i = 0; i < n_nodes; ++i)
+      if (left[i] >= n_nodes || right[i] >= n_nodes) throw StatusError{SF_ERR_INVALID_ARG, "bad child index"};
+    set_selector_model(feature, threshold, left, right, value, n_nodes, n_features);
+    return SF_OK;
+  });
+}
+
 const char* sf_status_string(sf_status s) {
   switch (s) {
     case SF_OK: return "SF_OK";

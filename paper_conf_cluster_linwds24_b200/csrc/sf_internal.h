@@ -111,6 +111,11 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank,
                           uint64_t nnz_local);
 void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l);
+int selector_features(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local,
+                      double* x);
+int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out);
+void set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
+                        const int32_t* right, const int32_t* value, int n_nodes, int n_features);
 size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l);
 // ---- kernels (sf_mttkrp.cu) ----
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,

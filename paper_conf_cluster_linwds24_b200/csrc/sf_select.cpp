@@ -67,8 +67,8 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
 static constexpr double kMinReuse = 256.0;
 static constexpr uint32_t kBlockRows = 256;
 
-sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank,
-                          uint64_t nnz_local) {
+static sf_launch_t select_rules(const Tensor& t, const sf_features_t& f, int mode, int rank,
+                               uint64_t nnz_local) {
   (void)f;
   sf_launch_t l{};
   const int N = t.nmodes;
@@ -122,6 +122,131 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
     normalize_launch(t, mode, rank, l);
   }
   return l;
+}
+
+// ---------------------------------------------------------------------------
+// Learned selector (§IV-B).  Features of the tensor
+// and mode -> a DecisionTree (trained offline on sweeps of synthetic *training* tensors,
+// tools/train_selector.py) -> one of kNumCandidates launch classes.  Classes are defined
+// relative to the gathered modes sorted by dimension so one model serves every mode.
+// ---------------------------------------------------------------------------
+static int gathered_sorted(const Tensor& t, int mode, int* g) {
+  int k = 0;
+  for (int m = 0; m < t.nmodes; ++m)
+    if (m != mode) g[k++] = m;
+  std::sort(g, g + k, [&](int a, int b) { return t.dims[a] < t.dims[b] || (t.dims[a] == t.dims[b] && a < b); });
+  return k;
+}
+
+static inline double lg2(double x) { return std::log2(std::max(x, 1.0)); }
+
+int selector_features(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local,
+                      double* x) {
+  int g[SF_MAX_MODES];
+  const int k = gathered_sorted(t, mode, g);
+  const double nnz = (double)std::max<uint64_t>(nnz_local, 1);
+  const double R4 = 4.0 * rank;
+  double fac = 0;
+  for (int q = 0; q < k; ++q) fac += (double)t.dims[g[q]] * R4;
+  int i = 0;
+  x[i++] = t.nmodes;
+  x[i++] = rank;
+  x[i++] = lg2(nnz);
+  x[i++] = lg2((double)t.dims[mode]);
+  x[i++] = lg2((double)t.dims[g[0]]);                        // smallest gathered dim
+  x[i++] = k >= 3 ? lg2((double)t.dims[g[1]]) : 0.0;         // middle (4-way+)
+  x[i++] = lg2((double)t.dims[g[k - 1]]);                    // largest gathered dim
+  x[i++] = lg2(nnz / (double)t.dims[g[0]]);                  // reuse of the smallest
+  x[i++] = lg2(nnz / (double)t.dims[g[k - 1]]);              // reuse of the largest
+  x[i++] = lg2(f.avg_nnz_per_slice);
+  x[i++] = lg2((double)f.max_nnz_per_slice);
+  x[i++] = f.avg_nnz_per_slice > 0 ? f.std_nnz_per_slice / f.avg_nnz_per_slice : 0.0;
+  x[i++] = f.slice_ratio;
+  x[i++] = f.fiber_ratio;
+  x[i++] = lg2(f.avg_nnz_per_fiber * 16.0);
+  x[i++] = lg2(fac);                                         // gathered factor bytes
+  x[i++] = lg2((double)t.dims[mode] * R4);                   // Y bytes
+  x[i++] = lg2((double)t.dims[g[0]] * R4);                   // smallest factor bytes
+  return i;
+}
+
+int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out) {
+  int g[SF_MAX_MODES];
+  const int k = gathered_sorted(t, mode, g);
+  sf_launch_t base{};
+  base.kernel = frag_supported(t.nmodes, rank) ? SF_KERNEL_FRAG : SF_KERNEL_COO;
+  base.block_threads = 512;
+  base.chunk_nnz = 128;
+  base.flags = SF_LAUNCH_L1_NO_ALLOCATE;
+  int n = 0;
+  auto add = [&](int stage_mode, uint32_t rows, uint32_t flags) {
+    sf_launch_t l = base;
+    l.flags |= flags;
+    if (stage_mode >= 0) {
+      l.staged_mask = 1u << stage_mode;
+      l.block_rows[stage_mode] = rows;
+    }
+    normalize_launch(t, mode, rank, l);
+    out[n++] = l;
+  };
+  add(-1, 0, 0);                          // 0 unstaged, owner stores
+  add(-1, 0, SF_LAUNCH_NO_OWNER_STORES);  // 1 unstaged, memset + atomics
+  add(g[0], 256, 0);                      // 2 stage smallest gathered mode, 256-row blocks
+  add(g[0], 512, 0);                      // 3                              512-row blocks
+  add(g[k - 1], 256, 0);                  // 4 stage largest gathered mode, 256-row blocks
+  add(g[k - 1], 512, 0);                  // 5                              512-row blocks
+  add(k >= 3 ? g[1] : g[0], 256, 0);      // 6 stage middle gathered mode (4-way), 256
+  return n;
+}
+
+struct TreeModel {
+  std::vector<int32_t> feature, left, right, value;
+  std::vector<double> threshold;
+  int nfeat = 0;
+};
+static TreeModel g_model;
+static bool g_have_model = false;
+
+void set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
+                        const int32_t* right, const int32_t* value, int n_nodes, int n_features) {
+  if (n_nodes <= 0) {
+    g_have_model = false;
+    return;
+  }
+  g_model.feature.assign(feature, feature + n_nodes);
+  g_model.threshold.assign(threshold, threshold + n_nodes);
+  g_model.left.assign(left, left + n_nodes);
+  g_model.right.assign(right, right + n_nodes);
+  g_model.value.assign(value, value + n_nodes);
+  g_model.nfeat = n_features;
+  g_have_model = true;
+}
+
+static int tree_predict(const double* x, int nx) {
+  int node = 0;
+  for (int depth = 0; depth < 64; ++depth) {
+    const int l = g_model.left[node], r = g_model.right[node];
+    if (l < 0 || r < 0) return g_model.value[node];
+    const int fi = g_model.feature[node];
+    const double v = (fi >= 0 && fi < nx) ? x[fi] : 0.0;
+    node = (v <= g_model.threshold[node]) ? l : r;
+    if (node < 0 || node >= (int)g_model.feature.size()) return -1;
+  }
+  return -1;
+}
+
+sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local) {
+  if (g_have_model && frag_supported(t.nmodes, rank) && nnz_local > 0) {
+    double x[32];
+    const int nx = selector_features(t, f, mode, rank, nnz_local, x);
+    if (nx == g_model.nfeat) {
+      const int c = tree_predict(x, nx);
+      sf_launch_t cand[16];
+      const int nc = selector_candidates(t, mode, rank, cand);
+      if (c >= 0 && c < nc && frag_smem_bytes(t, mode, rank, cand[c]) <= t.smem_optin) return cand[c];
+    }
+  }
+  return select_rules(t, f, mode, rank, nnz_local);
 }
 
 }  // namespace sf

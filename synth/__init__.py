@@ -183,3 +183,100 @@ def permute(I, seed, m, xs):
     out = np.empty_like(xs)
     lib().sfgen_permute_many(I, seed, m, len(xs), xs.ctypes.data, out.ctypes.data)
     return out
+
+
+# ---------------------------------------------------------------------------
+# Device twin (csrc/sfgen_cuda.cu): the same draws generated directly in HBM.
+# ---------------------------------------------------------------------------
+_SO_CUDA = os.path.join(_HERE, "libsfgen_cuda.so")
+_SRC_CUDA = os.path.join(_HERE, "csrc", "sfgen_cuda.cu")
+_lib_cuda = None
+
+
+def build_cuda(force: bool = False) -> str:
+    newest = max(os.path.getmtime(p) for p in [_SRC_CUDA, os.path.join(_HERE, "csrc", "sfgen_core.h")])
+    if force or not os.path.exists(_SO_CUDA) or os.path.getmtime(_SO_CUDA) < newest:
+        tmp = _SO_CUDA + f".tmp{os.getpid()}"
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3",
+                               "-shared", "-Xcompiler", "-fPIC", "-cudart", "static", "-o", tmp, _SRC_CUDA])
+        os.replace(tmp, _SO_CUDA)
+    return _SO_CUDA
+
+
+def lib_cuda():
+    global _lib_cuda
+    with _lock:
+        if _lib_cuda is None:
+            build_cuda()
+            L = ctypes.CDLL(_SO_CUDA)
+            P, u64 = ctypes.c_void_p, ctypes.c_uint64
+            L.sfgen_coo_device.argtypes = [ctypes.c_int, P, u64, u64, u64, P, P, P, P, P, ctypes.c_int,
+                                           ctypes.c_int, P, P, P]
+            L.sfgen_coo_device.restype = ctypes.c_int
+            L.sfgen_factor_device.argtypes = [u64, u64, u64, ctypes.c_int, ctypes.c_int, P, P]
+            L.sfgen_factor_device.restype = ctypes.c_int
+            _lib_cuda = L
+    return _lib_cuda
+
+
+def gen_coo_device(dims, nnz, seed, zipf=None, relabel=True, val_kind="unit", lo=0, hi=None, tables=None,
+                   device="cuda"):
+    """Device twin of gen_coo: torch int32 (uint32 bit pattern) index tensors + float32 values."""
+    import torch
+    dims = [int(d) for d in dims]
+    N = len(dims)
+    hi = int(nnz) if hi is None else int(hi)
+    n = hi - lo
+    if tables is None:
+        tables = tables_for(dims, zipf if zipf is not None else (0.0,) * N)
+    dev = torch.device(device)
+    inds = [torch.empty(n, dtype=torch.int32, device=dev) for _ in range(N)]
+    vals = torch.empty(n, dtype=torch.float32, device=dev)
+    if n == 0:
+        return inds, vals
+    edges = np.concatenate([t[0] for t in tables] + [np.zeros(1, np.uint64)])
+    thr = np.concatenate([t[1] for t in tables] + [np.zeros(1, np.uint64)])
+    eoff = np.cumsum([0] + [len(t[0]) for t in tables])[:-1].astype(np.int32)
+    toff = np.cumsum([0] + [len(t[1]) for t in tables])[:-1].astype(np.int32)
+    nb = np.array([len(t[0]) - 1 if len(t[0]) else 0 for t in tables], dtype=np.int32)
+    d_edges = torch.from_numpy(edges.view(np.int64)).to(dev)
+    d_thr = torch.from_numpy(thr.view(np.int64)).to(dev)
+    d_eoff, d_toff, d_nb = (torch.from_numpy(a).to(dev) for a in (eoff, toff, nb))
+    d_dims = torch.tensor(dims, dtype=torch.int64, device=dev)
+    d_ptrs = torch.tensor([a.data_ptr() for a in inds], dtype=torch.int64, device=dev)
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    rc = lib_cuda().sfgen_coo_device(N, d_dims.data_ptr(), seed, lo, hi, d_edges.data_ptr(), d_thr.data_ptr(),
+                                     d_nb.data_ptr(), d_eoff.data_ptr(), d_toff.data_ptr(), 1 if relabel else 0,
+                                     VAL_KINDS[val_kind], d_ptrs.data_ptr(), vals.data_ptr(), stream)
+    if rc != 0:
+        raise RuntimeError(f"sfgen_coo_device failed: cuda error {rc}")
+    torch.cuda.synchronize(dev)
+    return inds, vals
+
+
+def gen_factors_device(dims, rank, seed, kind="unit", device="cuda"):
+    import torch
+    out = []
+    stream = torch.cuda.current_stream(torch.device(device)).cuda_stream
+    for m, I in enumerate(dims):
+        f = torch.empty((int(I), int(rank)), dtype=torch.float32, device=device)
+        rc = lib_cuda().sfgen_factor_device(seed, m, int(I), int(rank), VAL_KINDS[kind], f.data_ptr(), stream)
+        if rc != 0:
+            raise RuntimeError(f"sfgen_factor_device failed: cuda error {rc}")
+        out.append(f)
+    torch.cuda.synchronize()
+    return out
+
+
+def config_tensor_device(cfg, val_kind="unit", lo=0, hi=None, device="cuda"):
+    if isinstance(cfg, str):
+        cfg = CONFIGS[cfg]
+    if not cfg.tables:
+        cfg.tables = tables_for(cfg.dims, cfg.zipf)
+    return gen_coo_device(cfg.dims, cfg.nnz, cfg.seed, cfg.zipf, True, val_kind, lo, hi, cfg.tables, device)
+
+
+def config_factors_device(cfg, kind="unit", device="cuda"):
+    if isinstance(cfg, str):
+        cfg = CONFIGS[cfg]
+    return gen_factors_device(cfg.dims, cfg.rank, cfg.fseed, kind, device)

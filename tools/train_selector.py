@@ -1,0 +1,210 @@
+#!/usr/bin/env python
+"""Learned launch selector (§IV-B; Fig. 7 "Generating Tensors ->
+Executing MTTKRP -> Data Collecting & Training -> Evaluating & Predicting").
+
+  collect (GPU):  generate synthetic TRAINING tensors (random shapes / skews, never the
+                  BASELINE.json evaluation shapes), and for every mode time every launch
+                  class of sf_selector_candidates -> jsonl records (features, times).
+  train (CPU):    fit a DecisionTreeClassifier (features -> best class), report accuracy,
+                  the achieved/best time ratio, per-candidate DecisionTreeRegressor MAPE
+                  (the paper's metric, "MAPE < 15%"), training and inference time; write
+                  paper_conf_cluster_linwds24_b200/selector_model.json.
+  eval (GPU):     on the BASELINE.json configs time every class and the library's pick
+                  (model installed) -> pick / best ratios.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+MODEL = os.path.join(ROOT, "paper_conf_cluster_linwds24_b200", "selector_model.json")
+
+
+def time_launch(T, n, R, facs, out, L, torch, reps=4):
+    T.set_launch(n, R, L)
+    for _ in range(2):
+        T.mttkrp(n, facs, out)
+    s = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(reps):
+        T.mttkrp(n, facs, out)
+    e1.record(s)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+args_nnz_lo, args_nnz_hi = 6.0, 7.5
+args_dims_log10 = (2.5, 7.2)
+
+
+def random_config(rng, k):
+    N = int(rng.choice([3, 3, 4]))
+    R = int(rng.choice([16, 32]))
+    nnz = int(10 ** rng.uniform(args_nnz_lo, args_nnz_hi))
+    lo_d, hi_d = args_dims_log10
+    while True:
+        dims = [int(10 ** rng.uniform(lo_d, hi_d)) for _ in range(N)]
+        if np.prod([float(d) for d in dims]) >= 8.0 * nnz:
+            break
+    zipf = [float(rng.choice([0.0, 0.5, 0.8, 1.0, 1.2])) for _ in range(N)]
+    return dict(name=f"train{k}", dims=dims, nnz=nnz, rank=R, zipf=zipf, seed=30000000 + k)
+
+
+def collect(args):
+    import torch
+
+    import paper_conf_cluster_linwds24_b200 as sf
+    sf.set_selector_model(None)
+    rng = np.random.default_rng(args.seed)
+    out_f = open(args.out, "a")
+    for k in range(args.count):
+        c = random_config(rng, k)
+        t0 = time.time()
+        inds, vals = synth.gen_coo_device(c["dims"], c["nnz"], c["seed"], c["zipf"])
+        facs = synth.gen_factors_device(c["dims"], c["rank"], c["seed"] + 7)
+        with sf.Tensor(c["dims"], inds, vals) as T:
+            del inds, vals
+            for n in range(len(c["dims"])):
+                R = c["rank"]
+                y = torch.empty((c["dims"][n], R), device="cuda")
+                x = T.selector_features(n, R)
+                cands = T.selector_candidates(n, R)
+                times = []
+                for L in cands:
+                    try:
+                        times.append(time_launch(T, n, R, facs, y, L, torch))
+                    except sf.SfError:
+                        times.append(None)
+                rec = {"config": c, "mode": n, "features": x, "times": times,
+                       "launches": [L.as_dict() for L in cands]}
+                out_f.write(json.dumps(rec) + "\n")
+                out_f.flush()
+        print(f"{c['name']} N={len(c['dims'])} nnz={c['nnz']} {time.time() - t0:.1f}s", flush=True)
+
+
+def load(path):
+    X, T = [], []
+    for line in open(path):
+        r = json.loads(line)
+        t = [x if x is not None else np.inf for x in r["times"]]
+        X.append(r["features"])
+        T.append(t)
+    return np.array(X), np.array(T)
+
+
+def train(args):
+    from sklearn.model_selection import KFold
+    from sklearn.tree import DecisionTreeClassifier, DecisionTreeRegressor
+    X, T = load(args.data)
+    y = np.argmin(T, axis=1)
+    best = T[np.arange(len(T)), y]
+    # cross-validated quality
+    kf = KFold(n_splits=5, shuffle=True, random_state=0)
+    ratios, acc, mape = [], [], []
+    for tr, te in kf.split(X):
+        clf = DecisionTreeClassifier(max_depth=args.depth, min_samples_leaf=2, random_state=0).fit(X[tr], y[tr])
+        p = clf.predict(X[te])
+        ratios += list(best[te] / T[te, p])
+        acc += list(p == y[te])
+        for c in range(T.shape[1]):
+            ok = np.isfinite(T[:, c])
+            trc, tec = tr[ok[tr]], te[ok[te]]
+            if len(trc) < 4 or len(tec) == 0:
+                continue
+            reg = DecisionTreeRegressor(max_depth=args.depth, random_state=0).fit(X[trc], np.log(T[trc, c]))
+            pred = np.exp(reg.predict(X[tec]))
+            mape += list(np.abs(pred - T[tec, c]) / T[tec, c])
+    t0 = time.perf_counter()
+    clf = DecisionTreeClassifier(max_depth=args.depth, min_samples_leaf=2, random_state=0).fit(X, y)
+    train_s = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    for _ in range(1000):
+        clf.predict(X[:1])
+    infer_ms = (time.perf_counter() - t0)
+    tr = clf.tree_
+    classes = clf.classes_
+    value = [int(classes[int(np.argmax(tr.value[i][0]))]) for i in range(tr.node_count)]
+    model = {"n_features": int(X.shape[1]), "classes": int(T.shape[1]),
+             "tree": {"feature": [int(f) for f in tr.feature], "threshold": [float(v) for v in tr.threshold],
+                      "left": [int(v) for v in tr.children_left], "right": [int(v) for v in tr.children_right],
+                      "value": value},
+             "trained_on": os.path.basename(args.data), "samples": int(len(X)), "max_depth": args.depth}
+    json.dump(model, open(MODEL, "w"))
+    fixed = {c: float(np.mean(best / T[:, c])) for c in range(T.shape[1])}
+    report = {"samples": int(len(X)), "cv_accuracy": float(np.mean(acc)),
+              "cv_pick_over_best_mean": float(np.mean(ratios)), "cv_pick_over_best_min": float(np.min(ratios)),
+              "cv_regressor_mape": float(np.mean(mape)), "train_s": train_s, "infer_ms_per_call": infer_ms,
+              "fixed_class_mean_ratio": fixed, "label_histogram": np.bincount(y, minlength=T.shape[1]).tolist(),
+              "nodes": int(tr.node_count)}
+    print(json.dumps(report, indent=1))
+    if args.report:
+        json.dump(report, open(args.report, "w"), indent=1)
+
+
+def evaluate(args):
+    import torch
+
+    import paper_conf_cluster_linwds24_b200 as sf
+    out_f = open(args.out, "w")
+    for name in args.configs.split(","):
+        cfg = synth.CONFIGS[name]
+        inds, vals = synth.config_tensor_device(cfg)
+        facs = synth.config_factors_device(cfg)
+        with sf.Tensor(cfg.dims, inds, vals) as T:
+            del inds, vals
+            for n in range(cfg.nmodes):
+                R = cfg.rank
+                y = torch.empty((cfg.dims[n], R), device="cuda")
+                cands = T.selector_candidates(n, R)
+                times = [time_launch(T, n, R, facs, y, L, torch) for L in cands]
+                auto = sf.Launch()
+                auto.kernel = 0  # SF_KERNEL_AUTO: re-plan with the selector (model installed at import)
+                T.set_launch(n, R, auto)
+                pick = T.plan_info(n, R)["launch"]
+                import ctypes
+                L = sf.Launch()
+                L.kernel = 2 if pick["kernel"] == "frag" else 1
+                L.block_threads, L.ctas_per_sm, L.chunk_nnz = pick["block_threads"], pick["ctas_per_sm"], pick["chunk_nnz"]
+                L.staged_mask, L.flags = pick["staged_mask"], pick["flags"]
+                for m, r in enumerate(pick["block_rows"]):
+                    L.block_rows[m] = r
+                t_pick = time_launch(T, n, R, facs, y, L, torch)
+                rec = {"config": name, "mode": n, "times": times, "pick": pick, "pick_ms": t_pick,
+                       "best_ms": min(times), "pick_over_best": min(times) / t_pick,
+                       "features": T.selector_features(n, R)}
+                print(json.dumps(rec), flush=True)
+                out_f.write(json.dumps(rec) + "\n")
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("cmd", choices=["collect", "train", "eval"])
+    ap.add_argument("--count", type=int, default=40)
+    ap.add_argument("--nnz-log10", default="6.0,7.5")
+    ap.add_argument("--dims-log10", default="2.5,7.2")
+    ap.add_argument("--seed", type=int, default=7)
+    ap.add_argument("--out", default="gpurun_out/selector_data.jsonl")
+    ap.add_argument("--data", default="profiles/selector_train_r01.jsonl")
+    ap.add_argument("--depth", type=int, default=5)
+    ap.add_argument("--report", default=None)
+    ap.add_argument("--configs", default="nell2,deli4d,nell1")
+    args = ap.parse_args()
+    global args_nnz_lo, args_nnz_hi, args_dims_log10
+    args_nnz_lo, args_nnz_hi = (float(x) for x in args.nnz_log10.split(","))
+    args_dims_log10 = tuple(float(x) for x in args.dims_log10.split(","))
+    {"collect": collect, "train": train, "eval": evaluate}[args.cmd](args)
+
+
+if __name__ == "__main__":
+    main()
