@@ -186,6 +186,17 @@ typedef enum { SF_ROWS_PACK = 0, SF_ROWS_ADD = 1, SF_ROWS_ZERO = 2 } sf_rows_op_
 sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int count, int op,
                      void* stream);
 
+/* ---- CP-ALS (Algorithm 1) ------------- */
+
+/* Runs up to `iters` ALS sweeps over all modes on this tensor, calling the MTTKRP of the
+ * hot path for line 4 of Alg. 1 (plans are built on demand with the selector).  factors:
+ * nmodes DEVICE pointers, fp32 I_m x rank row-major, in/out (initial guess -> result).
+ * fits: host array of >= iters doubles (may be NULL), fit after each sweep; stops early
+ * when tol > 0 and |fit_k - fit_{k-1}| < tol.  rank <= 64; no shard (nranks must be 1).
+ * Stream-ordered work, synchronizes once per sweep (to read the fit). */
+sf_status sf_cpals(sf_tensor_t t, int rank, float* const* factors, int iters, double tol, double* fits,
+                   int* iters_done, void* stream);
+
 /* ---- diagnostics -------------------------------------------------------- */
 const char* sf_status_string(sf_status s);
 const char* sf_last_error(void);

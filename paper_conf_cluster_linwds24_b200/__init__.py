@@ -97,7 +97,7 @@ EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_
             "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
             "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
-            "sf_selector_candidates", "sf_set_selector_model"]
+            "sf_selector_candidates", "sf_set_selector_model", "sf_cpals"]
 
 
 def lib(build_if_missing: bool = True):
@@ -127,10 +127,11 @@ def lib(build_if_missing: bool = True):
             L.sf_selector_features.argtypes = [P, I, I, P, ctypes.POINTER(I)]
             L.sf_selector_candidates.argtypes = [P, I, I, P, ctypes.POINTER(I)]
             L.sf_set_selector_model.argtypes = [P, P, P, P, P, I, I]
+            L.sf_cpals.argtypes = [P, I, P, I, ctypes.c_double, P, ctypes.POINTER(I), P]
             for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
                        "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
                        "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op", "sf_selector_features",
-                       "sf_selector_candidates", "sf_set_selector_model"]:
+                       "sf_selector_candidates", "sf_set_selector_model", "sf_cpals"]:
                 getattr(L, fn).restype = ctypes.c_int
             L.sf_status_string.argtypes = [I]
             L.sf_status_string.restype = ctypes.c_char_p
@@ -151,7 +152,7 @@ def lib(build_if_missing: bool = True):
 MODEL_PATH = os.path.join(_HERE, "selector_model.json")
 # "rules" (sf_select.cpp, calibrated on sweeps) or "model" (the learned DecisionTree,
 # tools/train_selector.py).  See DESIGN.md §5 for the held-out comparison that sets this.
-DEFAULT_SELECTOR = "rules"
+DEFAULT_SELECTOR = "model"
 
 
 def _install_model(L, path):
@@ -297,6 +298,17 @@ class Tensor:
             ctypes.memmove(ctypes.byref(l), ctypes.byref(arr[i]), ctypes.sizeof(Launch))
             out.append(l)
         return out
+
+    def cp_als(self, factors, iters=10, tol=0.0, stream=None):
+        """CP-ALS (Algorithm 1) in place on device factor tensors; returns the fit per sweep."""
+        import numpy as np
+        rank = int(factors[0].shape[1])
+        fp = (ctypes.c_void_p * self.nmodes)(*[_ptr(f) for f in factors])
+        fits = np.zeros(max(iters, 1), np.float64)
+        done = ctypes.c_int(0)
+        _check(lib().sf_cpals(self._h, rank, fp, int(iters), float(tol), fits.ctypes.data, ctypes.byref(done),
+                              _stream_handle(stream)))
+        return fits[:done.value].tolist()
 
     def mttkrp(self, mode, factors, out, rank=None, stream=None):
         """out <- mode-`mode` MTTKRP (device tensors; stream-ordered)."""

@@ -15,7 +15,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
                 "--expt-relaxed-constexpr", "-Xptxas", "-v", "-I", os.path.join(ROOT, "include")]
-SOURCES = ["sf_api.cu", "sf_plan.cu", "sf_mttkrp.cu", "sf_select.cpp", "sf_frag_r16.cu", "sf_frag_r32.cu", "sf_frag_r64.cu"]
+SOURCES = ["sf_api.cu", "sf_plan.cu", "sf_mttkrp.cu", "sf_select.cpp", "sf_cpals.cu", "sf_frag_r16.cu",
+           "sf_frag_r32.cu", "sf_frag_r64.cu"]
 
 
 def _deps():

@@ -457,6 +457,27 @@ sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int co
   });
 }
 
+sf_status sf_cpals(sf_tensor_t h, int rank, float* const* factors, int iters, double tol, double* fits,
+                   int* iters_done, void* stream) {
+  return guard([&]() -> sf_status {
+    if (!h || !factors || iters < 0) throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, 0, rank);
+    if (t->nranks != 1) throw StatusError{SF_ERR_UNSUPPORTED, "sf_cpals: sharded handles not supported"};
+    for (int m = 0; m < t->nmodes; ++m)
+      if (!factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
+    SF_CUDA(cudaSetDevice(t->device));
+    Plan* plans[SF_MAX_MODES];
+    for (int m = 0; m < t->nmodes; ++m) {
+      if (!get_plan(*t, m, rank)) make_plan(*t, m, rank, nullptr);
+      plans[m] = get_plan(*t, m, rank);
+    }
+    if (iters_done) *iters_done = 0;
+    cpals(*t, rank, factors, iters, tol, fits, iters_done, static_cast<cudaStream_t>(stream), plans);
+    return SF_OK;
+  });
+}
+
 sf_status sf_selector_features(sf_tensor_t h, int mode, int rank, double* x, int* n) {
   return guard([&]() -> sf_status {
     if (!h || !x || !n) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};

@@ -117,6 +117,9 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out);
 void set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
                         const int32_t* right, const int32_t* value, int n_nodes, int n_features);
 size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l);
+// ---- CP-ALS (sf_cpals.cu) ----
+void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, double* fits, int* done,
+           cudaStream_t s, Plan* const* plans);
 // ---- kernels (sf_mttkrp.cu) ----
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
                    cudaStream_t s);

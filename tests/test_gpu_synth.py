@@ -11,7 +11,8 @@ pytestmark = pytest.mark.gpu
 @pytest.mark.parametrize("name", ["tiny", "tiny_skew", "deli4d"])
 def test_device_generator_matches_host(cuda_device, name):
     cfg = synth.CONFIGS[name]
-    lo, hi = 12345, min(cfg.nnz, 12345 + 300_000)
+    lo = min(12345, cfg.nnz // 3)
+    hi = min(cfg.nnz, lo + 300_000)
     hi_ = [a for a in synth.config_tensor(cfg, lo, hi)[0]]
     hv = synth.config_tensor(cfg, lo, hi)[1]
     di, dv = synth.config_tensor_device(cfg, lo=lo, hi=hi)
