@@ -10,6 +10,8 @@
 
 #include <algorithm>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -23,21 +25,67 @@ static thread_local std::string g_err;
 
 void set_error(const std::string& msg) { g_err = msg; }
 
+// Caching device allocator.  cudaMalloc/cudaFree of GB-sized plan arrays cost tens of ms
+// each and cudaFree synchronizes the device; blocks are instead kept in a size-keyed free
+// list and reused (best fit within 2x).  Reuse is stream-safe because every library buffer
+// is produced and consumed on the handle's planning stream, or the device is synchronized
+// first (plan replacement and handle destruction call cudaDeviceSynchronize).
+struct BlockCache {
+  std::mutex mu;
+  std::multimap<size_t, void*> free_blocks;
+  size_t cached = 0;
+  void* get(size_t b, size_t* got) {
+    {
+      std::lock_guard<std::mutex> g(mu);
+      auto it = free_blocks.lower_bound(b);
+      if (it != free_blocks.end() && it->first <= 2 * b + (1u << 20)) {
+        void* q = it->second;
+        *got = it->first;
+        cached -= it->first;
+        free_blocks.erase(it);
+        return q;
+      }
+    }
+    void* q = nullptr;
+    cudaError_t e = cudaMalloc(&q, b);
+    if (e != cudaSuccess) {  // give the cache back to the driver and retry once
+      cudaGetLastError();
+      trim();
+      e = cudaMalloc(&q, b);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        throw CudaError{e, "cudaMalloc"};
+      }
+    }
+    *got = b;
+    return q;
+  }
+  void put(void* q, size_t b) {
+    std::lock_guard<std::mutex> g(mu);
+    free_blocks.emplace(b, q);
+    cached += b;
+  }
+  void trim() {
+    std::lock_guard<std::mutex> g(mu);
+    cudaDeviceSynchronize();
+    for (auto& kv : free_blocks) cudaFree(kv.second);
+    free_blocks.clear();
+    cached = 0;
+  }
+};
+static BlockCache g_cache;
+
 void DevBuf::alloc(size_t b) {
   release();
   if (b == 0) b = 16;
-  void* q = nullptr;
-  cudaError_t e = cudaMalloc(&q, b);
-  if (e != cudaSuccess) {
-    cudaGetLastError();
-    throw CudaError{e, "cudaMalloc"};
-  }
-  p = q;
-  bytes = b;
+  b = (b + 255) & ~(size_t)255;
+  size_t got = 0;
+  p = g_cache.get(b, &got);
+  bytes = got;
 }
 
 void DevBuf::release() {
-  if (p) cudaFree(p);
+  if (p) g_cache.put(p, bytes);
   p = nullptr;
   bytes = 0;
 }
@@ -171,7 +219,8 @@ static Plan* get_plan(Tensor& t, int mode, int rank) {
 static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override_launch) {
   SF_CUDA(cudaSetDevice(t.device));
   sf_features_t f;
-  compute_features(t, mode, &f);
+  DevBuf keys, pos;  // the matricized order, sorted once for features + the plan
+  compute_features(t, mode, &f, &keys, &pos);
   const uint64_t lo = (uint64_t)(((unsigned __int128)t.rank * t.nnz) / t.nranks);
   const uint64_t hi = (uint64_t)(((unsigned __int128)(t.rank + 1) * t.nnz) / t.nranks);
   sf_launch_t l;
@@ -185,13 +234,16 @@ static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override
     throw StatusError{SF_ERR_INVALID_ARG, "launch needs more shared memory than the device has"};
   Plan* p = new Plan();
   try {
-    build_plan(t, *p, mode, rank, l);
+    build_plan(t, *p, mode, rank, l, &keys, &pos);
   } catch (...) {
     delete p;
     throw;
   }
   Plan* old = get_plan(t, mode, rank);
-  delete old;
+  if (old) {
+    SF_CUDA(cudaDeviceSynchronize());  // in-flight sf_mttkrp may still read the old plan
+    delete old;
+  }
   t.plans[{mode, rank}] = p;
 }
 
@@ -271,7 +323,7 @@ sf_status sf_tensor_destroy(sf_tensor_t h) {
     if (!h) return SF_OK;
     Tensor* t = as_tensor(h);
     cudaSetDevice(t->device);
-    cudaStreamSynchronize(t->stream);
+    cudaDeviceSynchronize();  // kernels on caller streams may still read the arrays
     delete t;
     return SF_OK;
   });
@@ -317,7 +369,7 @@ sf_status sf_features(sf_tensor_t h, int mode, sf_features_t* out) {
     Tensor* t = as_tensor(h);
     check_mode_rank(*t, mode, 1);
     SF_CUDA(cudaSetDevice(t->device));
-    compute_features(*t, mode, out);
+    compute_features(*t, mode, out, nullptr, nullptr);
     return SF_OK;
   });
 }
@@ -485,7 +537,7 @@ sf_status sf_selector_features(sf_tensor_t h, int mode, int rank, double* x, int
     check_mode_rank(*t, mode, rank);
     SF_CUDA(cudaSetDevice(t->device));
     sf_features_t f;
-    compute_features(*t, mode, &f);
+    compute_features(*t, mode, &f, nullptr, nullptr);
     const uint64_t lo = (uint64_t)(((unsigned __int128)t->rank * t->nnz) / t->nranks);
     const uint64_t hi = (uint64_t)(((unsigned __int128)(t->rank + 1) * t->nnz) / t->nranks);
     *n = selector_features(*t, f, mode, rank, hi - lo, x);

@@ -85,6 +85,8 @@ struct Tensor {
   size_t smem_optin = 227 * 1024;
   DevBuf ind[SF_MAX_MODES];  // raw COO (input order)
   DevBuf val;
+  DevBuf aos;                // raw COO as AoS records (aos_words per nonzero), built on first plan
+  int aos_words = 0;
   bool have_features[SF_MAX_MODES] = {};
   sf_features_t features[SF_MAX_MODES] = {};
   std::map<std::pair<int, int>, Plan*> plans;  // (mode, rank) -> plan
@@ -105,8 +107,10 @@ inline int secondary_mode(const Tensor& t, int mode) {
 }
 
 // ---- planning (sf_plan.cu) ----
-void compute_features(Tensor& t, int mode, sf_features_t* out);
-void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch);
+// keys/pos (optional): receive the matricized order (sorted keys, input positions) when
+// this call had to sort, so build_plan can reuse it instead of sorting again.
+void compute_features(Tensor& t, int mode, sf_features_t* out, DevBuf* keys, DevBuf* pos);
+void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch, DevBuf* keys, DevBuf* pos);
 // ---- selection (sf_select.cpp) ----
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank,
                           uint64_t nnz_local);

@@ -204,12 +204,16 @@ static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_f
   }
 }
 
-void compute_features(Tensor& t, int mode, sf_features_t* out) {
+void compute_features(Tensor& t, int mode, sf_features_t* out, DevBuf* keys_out, DevBuf* pos_out) {
   if (!t.have_features[mode]) {
     DevBuf keys, pos;
     if (t.nnz) matricized_sort(t, mode, keys, pos);
     features_from_sorted(t, mode, keys.as<uint64_t>(), &t.features[mode]);
     t.have_features[mode] = true;
+    if (keys_out && pos_out) {
+      *keys_out = std::move(keys);
+      *pos_out = std::move(pos);
+    }
   }
   *out = t.features[mode];
 }
@@ -233,6 +237,45 @@ __global__ void tile_key_kernel(TileParams tp, const uint32_t* __restrict__ pos,
       if (tp.staged_mask & (1u << m)) t = t * tp.ntiles[m] + tp.ind[m][e] / tp.block_rows[m];
     tkey[k] = t;
     tpos[k] = e;
+  }
+}
+
+// AoS copy of the raw COO: one record of W words per nonzero (N indices, value, padding),
+// W = 4 / 8 / 16, so the permutation gather reads one 16/32/64-byte record per nonzero
+// (one or two sectors) instead of N+1 scattered 4-byte words.
+struct AosParams {
+  const uint32_t* ind[SF_MAX_MODES];
+  const float* val;
+  uint32_t* aos;
+  int nmodes, W;
+};
+
+__global__ void build_aos_kernel(AosParams a, uint64_t n) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    uint32_t* r = a.aos + e * a.W;
+    for (int m = 0; m < a.nmodes; ++m) r[m] = a.ind[m][e];
+    r[a.nmodes] = __float_as_uint(a.val[e]);
+  }
+}
+
+template <int W>
+__global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
+                                  uint64_t n, int nmodes, uint32_t* const* __restrict__ dst,
+                                  float* __restrict__ vdst) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint4* rec = reinterpret_cast<const uint4*>(aos + (uint64_t)perm[k] * W);
+    uint32_t w[W];
+#pragma unroll
+    for (int q = 0; q < W / 4; ++q) {
+      const uint4 v = __ldg(rec + q);
+      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
+    }
+#pragma unroll
+    for (int m = 0; m < W - 1; ++m)
+      if (m < nmodes) dst[m][k] = w[m];
+    vdst[k] = __uint_as_float(w[nmodes < W ? nmodes : 0]);
   }
 }
 
@@ -291,7 +334,8 @@ __global__ void chunk_scatter_kernel(const uint32_t* __restrict__ flag, const ui
 
 __global__ void set_u32_kernel(uint32_t* p, uint32_t v) { *p = v; }
 
-void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch) {
+void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch, DevBuf* keys_in,
+                DevBuf* pos_in) {
   cudaEvent_t ev0, ev1;
   SF_CUDA(cudaEventCreate(&ev0));
   SF_CUDA(cudaEventCreate(&ev1));
@@ -308,7 +352,12 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   if (nl >= (1ull << 32)) throw StatusError{SF_ERR_UNSUPPORTED, "shard nnz must be < 2^32"};
 
   DevBuf keys, pos0;
-  if (n) matricized_sort(t, mode, keys, pos0);
+  if (keys_in && pos_in && keys_in->p && pos_in->p) {  // reuse the features' sort
+    keys = std::move(*keys_in);
+    pos0 = std::move(*pos_in);
+  } else if (n) {
+    matricized_sort(t, mode, keys, pos0);
+  }
   if (!t.have_features[mode]) {
     features_from_sorted(t, mode, keys.as<uint64_t>(), &t.features[mode]);
     t.have_features[mode] = true;
@@ -380,9 +429,34 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   g.vdst = p.val.as<float>();
   g.nmodes = N;
   if (nl) {
-    gather_kernel<<<grid_for(nl), 256, 0, t.stream>>>(g, perm.as<uint32_t>(), nl);
+    // AoS record copy of the raw COO (built once per tensor, reused by every mode's plan)
+    const int W = (N + 1 <= 4) ? 4 : (N + 1 <= 8 ? 8 : 16);
+    if (!t.aos.p) {
+      t.aos.alloc((size_t)n * W * 4 + 64);
+      AosParams a{};
+      for (int m = 0; m < N; ++m) a.ind[m] = t.ind[m].as<uint32_t>();
+      a.val = t.val.as<float>();
+      a.aos = t.aos.as<uint32_t>();
+      a.nmodes = N;
+      a.W = W;
+      build_aos_kernel<<<grid_for(n), 256, 0, t.stream>>>(a, n);
+      count_launch();
+      SF_CUDA(cudaGetLastError());
+      t.aos_words = W;
+    }
+    DevBuf dptr(sizeof(uint32_t*) * SF_MAX_MODES);
+    uint32_t* hptr[SF_MAX_MODES] = {};
+    for (int m = 0; m < N; ++m) hptr[m] = g.dst[m];
+    SF_CUDA(cudaMemcpyAsync(dptr.p, hptr, sizeof(hptr), cudaMemcpyHostToDevice, t.stream));
+    uint32_t* const* dd = reinterpret_cast<uint32_t* const*>(dptr.p);
+    switch (W) {
+      case 4: gather_aos_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+      case 8: gather_aos_kernel<8><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+      default: gather_aos_kernel<16><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+    }
     count_launch();
     SF_CUDA(cudaGetLastError());
+    SF_CUDA(cudaStreamSynchronize(t.stream));  // dptr's host source must outlive the copy
   }
   p.perm = std::move(perm);
 
