@@ -76,6 +76,7 @@ typedef struct {
 } sf_launch_t;
 #define SF_LAUNCH_PREFETCH_L2 1u
 #define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
+#define SF_LAUNCH_NO_CARRY 8u /* FRAG: flush each stretch's last run (no cross-stretch carry) */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation
                                        (ld.global.nc.L1::no_allocate.v8.f32; measured faster) */
 
@@ -133,6 +134,11 @@ sf_status sf_set_shard(sf_tensor_t t, int nranks, int rank);
 /* Sort (matricized order, then tiles), build fragments/chunks, compute features and
  * select the launch for (mode, rank).  Idempotent; synchronizes the device. */
 sf_status sf_plan(sf_tensor_t t, int mode, int rank);
+/* Free the plan of (mode, rank) (device memory returns to the library's block cache);
+ * a later sf_mttkrp needs sf_plan again.  Synchronizes the device. */
+sf_status sf_plan_release(sf_tensor_t t, int mode, int rank);
+/* Return every cached device block to the driver (cudaFree).  Synchronizes the device. */
+sf_status sf_trim_cache(void);
 /* Override the selector (sweeps, Fig. 4) and re-plan. */
 sf_status sf_set_launch(sf_tensor_t t, int mode, int rank, const sf_launch_t* launch);
 /* Features only (no plan needed). Synchronizes. */

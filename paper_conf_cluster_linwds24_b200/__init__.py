@@ -97,7 +97,8 @@ EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_
             "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
             "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
-            "sf_selector_candidates", "sf_set_selector_model", "sf_cpals"]
+            "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
+            "sf_trim_cache"]
 
 
 def lib(build_if_missing: bool = True):
@@ -128,10 +129,13 @@ def lib(build_if_missing: bool = True):
             L.sf_selector_candidates.argtypes = [P, I, I, P, ctypes.POINTER(I)]
             L.sf_set_selector_model.argtypes = [P, P, P, P, P, I, I]
             L.sf_cpals.argtypes = [P, I, P, I, ctypes.c_double, P, ctypes.POINTER(I), P]
+            L.sf_plan_release.argtypes = [P, I, I]
+            L.sf_trim_cache.argtypes = []
             for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
                        "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
                        "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op", "sf_selector_features",
-                       "sf_selector_candidates", "sf_set_selector_model", "sf_cpals"]:
+                       "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
+            "sf_trim_cache"]:
                 getattr(L, fn).restype = ctypes.c_int
             L.sf_status_string.argtypes = [I]
             L.sf_status_string.restype = ctypes.c_char_p
@@ -215,6 +219,11 @@ def _stream_handle(stream):
     return stream.cuda_stream
 
 
+def trim_cache():
+    """Return the library's cached device blocks to the driver."""
+    _check(lib().sf_trim_cache())
+
+
 def kernel_launches() -> int:
     return int(lib().sf_kernel_launches())
 
@@ -259,6 +268,9 @@ class Tensor:
 
     def plan(self, mode, rank):
         _check(lib().sf_plan(self._h, int(mode), int(rank)))
+
+    def plan_release(self, mode, rank):
+        _check(lib().sf_plan_release(self._h, int(mode), int(rank)))
 
     def set_launch(self, mode, rank, launch: Launch):
         _check(lib().sf_set_launch(self._h, int(mode), int(rank), ctypes.byref(launch)))

@@ -353,6 +353,29 @@ sf_status sf_plan(sf_tensor_t h, int mode, int rank) {
   });
 }
 
+sf_status sf_plan_release(sf_tensor_t h, int mode, int rank) {
+  return guard([&]() -> sf_status {
+    if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    auto it = t->plans.find({mode, rank});
+    if (it != t->plans.end()) {
+      SF_CUDA(cudaSetDevice(t->device));
+      SF_CUDA(cudaDeviceSynchronize());
+      delete it->second;
+      t->plans.erase(it);
+    }
+    return SF_OK;
+  });
+}
+
+sf_status sf_trim_cache(void) {
+  return guard([&]() -> sf_status {
+    g_cache.trim();
+    return SF_OK;
+  });
+}
+
 sf_status sf_set_launch(sf_tensor_t h, int mode, int rank, const sf_launch_t* launch) {
   return guard([&]() -> sf_status {
     if (!h || !launch) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};

@@ -46,7 +46,7 @@ struct FragParams {
   uint32_t stage_words;               // words per field per pipeline stage
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
   uint32_t row_end;                   // this shard's rows end (exclusive)
-  uint32_t prefetch;                  // launch flags: 1 L2 prefetch
+  uint32_t prefetch;                  // launch flags: 1 L2 prefetch, 8 no carry
 };
 
 constexpr int kFragStages = 2;
@@ -240,6 +240,14 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
   for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]);
   uint32_t fac_phase = 0;
   uint32_t it = 0;  // chunks this warp has consumed (stage = it % 2, parity = (it / 2) & 1)
+  // A7 carry: a lane group keeps its open run (row `cur`, partial acc) across its
+  // consecutive stretches, so a heavy row receives one atomic per (CTA, group) instead of
+  // one per stretch (shorter fp32 atomic chains: SURVEY F-c; measured on amazon mode 1).
+  bool carry = false;
+  uint32_t cur = 0;
+  float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
+  float* const out0 = p.out + 4 * c0;
+  float* const out1 = out0 + 4;
 
   uint32_t seg = j0;
   while (seg < j1) {
@@ -302,8 +310,6 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
         const uint32_t* sIdx[G];
 #pragma unroll
         for (int q = 0; q < G; ++q) sIdx[q] = reinterpret_cast<const uint32_t*>(sb + (size_t)p.slot_mode[q] * SW);
-        float* out0 = p.out + 4 * c0;
-        float* out1 = out0 + 4;
         // gather slot q of nonzero kk (staged: shared memory, else global via L1/L2)
         auto gather = [&](int q, uint32_t kk) -> F8 {
           const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
@@ -334,8 +340,6 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
             }
           }
         }
-        uint32_t cur = sOut[k0];
-        float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
         // A5 (owner mode, unstaged plans only): runs wholly inside this stretch are
         // STORED (this group owns the row); the stretch's first/last run is atomically
         // added when it continues into the neighbouring stretch (those rows were zeroed by
@@ -344,20 +348,16 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
         // flush is an atomic.
         bool shared = true;       // current run may be shared with another stretch/tile
         bool last_shared = true;  // the stretch's last run continues past k1
+        const uint32_t first = sOut[k0];
+        bool first_shared = true;
+        uint32_t before = 0xFFFFFFFFu;
         if constexpr (S == 0) {
           if (p.owner) {
             const uint32_t P0 = b + k0, P1 = b + k1;
             const uint32_t* gOut = p.ind[p.mode];
-            const uint32_t first = sOut[k0];
-            const uint32_t before = (P0 > 0) ? __ldg(gOut + P0 - 1) : 0xFFFFFFFFu;
-            shared = (P0 > 0) && before == first;
+            before = (P0 > 0) ? __ldg(gOut + P0 - 1) : 0xFFFFFFFFu;
+            first_shared = (P0 > 0) && before == first;
             last_shared = (P1 < p.nnz) && __ldg(gOut + P1) == sOut[k1 - 1];
-            if (!shared && P0 > 0)  // gap rows (before, first) belong to this group
-              for (uint32_t r = before + 1; r < first; ++r) {
-                if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
-                                              make_float4(0.f, 0.f, 0.f, 0.f));
-                else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
-              }
           }
         }
         auto flush_run = [&](bool atomic) {
@@ -371,6 +371,24 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
           acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
           acc1 = acc0;
         };
+        if (carry && first != cur) {  // the carried run ended before this stretch
+          flush_run(true);
+          carry = false;
+        }
+        if (carry) {
+          shared = true;  // continuing a run begun in an earlier stretch
+        } else {
+          cur = first;
+          shared = first_shared;
+          if constexpr (S == 0) {
+            if (p.owner && !first_shared && b + k0 > 0)  // gap rows (before, first) are ours
+              for (uint32_t r = before + 1; r < first; ++r) {
+                if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
+                                              make_float4(0.f, 0.f, 0.f, 0.f));
+                else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
+              }
+          }
+        }
         // run edge inside the stretch: close `cur`, zero the gap up to the next row i
         auto flush = [&]() { flush_run(shared); };
         auto advance = [&](uint32_t i) {
@@ -439,12 +457,23 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
           f4fma_(acc0, vb, pr.a);
           if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
         }
-        flush_run(shared || last_shared);
+        // carry only a run that filled the whole stretch (a heavy row); shorter runs that
+        // merely cross the boundary are flushed now (cheaper, and their chains are short)
+        if (last_shared && first == cur && !(p.prefetch & 8u)) {
+          carry = true;  // the run continues past this stretch: keep accumulating
+        } else {
+          flush_run(shared || last_shared);  // a run crossing into the next stretch is shared
+          carry = false;
+        }
       }
       __syncwarp();  // every lane is done reading stage st
       if (lane == 0 && j + 2u * nwarps < seg_end) issue(j + 2u * nwarps, st);
     }
     seg = seg_end;
+  }
+  if (carry) {  // close the run still open at the end of this CTA's range
+    red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
+    if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
   }
 }
 

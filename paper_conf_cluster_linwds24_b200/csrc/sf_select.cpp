@@ -114,6 +114,7 @@ static sf_launch_t select_rules(const Tensor& t, const sf_features_t& f, int mod
     if (best >= 0) {
       l.staged_mask = 1u << best;
       l.block_rows[best] = kBlockRows;
+      l.flags |= SF_LAUNCH_NO_CARRY;
     }
   }
   normalize_launch(t, mode, rank, l);
@@ -185,6 +186,7 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out) {
     if (stage_mode >= 0) {
       l.staged_mask = 1u << stage_mode;
       l.block_rows[stage_mode] = rows;
+      l.flags |= SF_LAUNCH_NO_CARRY;  // tiled runs are short; the carry costs ~4 % there
     }
     normalize_launch(t, mode, rank, l);
     out[n++] = l;
