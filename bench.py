@@ -209,19 +209,24 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     N, R = cfg.nmodes, cfg.rank
 
-    # ---- synthetic input (every rank holds the full raw COO, §8(e) v1) ----
+    # ---- synthetic input (every rank holds the full raw COO, §8(e) v1), generated in HBM by
+    # the device twin of the seeded generator; pinned host copies feed the e2e leg ----
     t_gen = time.perf_counter()
-    inds, vals = synth.config_tensor(cfg)
-    facs = synth.config_factors(cfg)
+    d_inds, d_vals = synth.config_tensor_device(cfg, device=dev)
+    d_facs = synth.config_factors_device(cfg, device=dev)
+    h_inds = [a.cpu().pin_memory() for a in d_inds]
+    h_vals = d_vals.cpu().pin_memory()
+    h_facs = [f.cpu().pin_memory() for f in d_facs]
+    inds = [a.numpy().view(np.uint32) for a in h_inds]
+    vals = h_vals.numpy()
+    facs = [f.numpy() for f in h_facs]
     t_gen = time.perf_counter() - t_gen
-    h_inds = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
-    h_vals = torch.from_numpy(vals).pin_memory()
-    h_facs = [torch.from_numpy(f).pin_memory() for f in facs]
-    d_facs = [f.to(dev) for f in h_facs]
     stream = torch.cuda.Stream(device=dev)
 
     # ---- resident tensor + plans ----
-    T = sf.Tensor(cfg.dims, h_inds, h_vals)
+    T = sf.Tensor(cfg.dims, d_inds, d_vals)
+    del d_inds, d_vals
+    torch.cuda.empty_cache()
     if world > 1:
         T.set_shard(world, rank)
     overrides = {}

@@ -65,6 +65,7 @@ def main():
     ap.add_argument("--modes", default=None)
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--only-staged", default=None, help="restrict to this staged set, e.g. '1:256'")
     args = ap.parse_args()
     import torch
 
@@ -90,6 +91,11 @@ def main():
         results = []
         t0 = time.time()
         for g in grid(cfg.dims, n, R, args.quick):
+            if args.only_staged is not None:
+                want = {} if args.only_staged == "none" else {int(a): int(b) for a, b in
+                                                              (x.split(":") for x in args.only_staged.split(","))}
+                if g.get("kernel") != 2 or g.get("staged") != want:
+                    continue
             L = sf.Launch.make(**g)
             ms, err = time_launch(T, n, R, facs, out, L, sf, torch)
             rec = {"mode": n, "launch": g, "ms": ms, "err": err,

@@ -123,7 +123,24 @@ CONFIGS = {
                   "BASELINE.json configs[3]: nell-1-shaped, R=32"),
     "amazon": _cfg(5, "amazon", (4821207, 1774269, 1805187), 1_741_809_018, 16, (0.8, 0.8, 1.0),
                    "BASELINE.json configs[4]: amazon-reviews-shaped, R=16"),
+    # the other PAPER.md Table III tensors (L256-267) as synthetic shapes
+    # (FROSTT exact dims; rank not stated by the paper: R = 16; Zipf exponents proposals)
+    "vast": _cfg(6, "vast", (165427, 11374, 2), 26_021_945, 16, (0.5, 0.5, 0.0),
+                 "Table III vast-shaped 165K x 11K x 2, 26M nnz"),
+    "flickr3d": _cfg(7, "flickr3d", (319686, 28153045, 1607191), 112_890_310, 16, (1.0, 1.0, 1.0),
+                     "Table III flickr-3d-shaped 320K x 28M x 2M, 113M nnz"),
+    "deli3d": _cfg(8, "deli3d", (532924, 17262471, 2480308), 140_126_181, 16, (1.0, 1.0, 1.0),
+                   "Table III deli-3d-shaped 533K x 17M x 3M, 140M nnz"),
+    "uber": _cfg(9, "uber", (183, 24, 1140, 1717), 3_309_490, 16, (0.3, 0.3, 0.5, 0.5),
+                 "Table III uber-shaped 183 x 24 x 1140 x 1717, 3M nnz"),
+    "nips": _cfg(10, "nips", (2482, 2862, 14036, 17), 3_101_609, 16, (0.8, 0.8, 0.8, 0.3),
+                 "Table III nips-shaped 2K x 3K x 14K x 17, 3M nnz"),
+    "enron": _cfg(11, "enron", (6066, 5699, 244268, 1176), 54_202_099, 16, (1.0, 1.0, 0.8, 0.5),
+                  "Table III enron-shaped 6K x 6K x 244K x 1K, 54M nnz"),
+    "flickr4d": _cfg(12, "flickr4d", (319686, 28153045, 1607191, 731), 112_890_310, 16, (1.0, 1.0, 1.0, 0.3),
+                     "Table III flickr-4d-shaped 320K x 28M x 2M x 731, 113M nnz"),
 }
+TABLE_III = ["vast", "nell2", "flickr3d", "deli3d", "nell1", "uber", "nips", "enron", "flickr4d", "deli4d"]
 
 
 def tables_for(dims, zipf):

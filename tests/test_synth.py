@@ -55,8 +55,9 @@ def test_skew_is_heavy_headed():
 
 
 def test_configs_match_table_III_density():
-    """PAPER.md Table III (L256-267): nell-2 2.4e-5, nell-1 9.1e-13, deli-4d 4.3e-15."""
-    want = {"nell2": 2.4e-5, "nell1": 9.1e-13, "deli4d": 4.3e-15}
+    """PAPER.md Table III (L256-267) densities (reading R13: exponent minus signs restored)."""
+    want = {"nell2": 2.4e-5, "nell1": 9.1e-13, "deli4d": 4.3e-15, "vast": 6.9e-3, "flickr3d": 7.8e-12,
+            "deli3d": 6.1e-12, "uber": 3.9e-4, "nips": 1.8e-6, "enron": 5.5e-9, "flickr4d": 1.1e-14}
     for name, dens in want.items():
         c = synth.CONFIGS[name]
         d = c.nnz / float(np.prod([float(x) for x in c.dims]))
