@@ -1,0 +1,91 @@
+#!/usr/bin/env python
+"""segments x streams study of the paper's pipeline (§IV-C
+L201-229, Fig. 11 "fix the number of segments to 4 ... fix the number of CUDA
+streams to 4"), on B200 with synthetic tensors shaped like the paper's workloads.
+
+For a host-resident (pinned) COO tensor and one mode:
+  T_h2d      the COO upload alone (cudaMemcpy of the N+1 arrays)
+  T_(1,1)    sf_mttkrp_streamed with 1 segment on 1 stream (no overlap)
+  T_compute  = T_(1,1) - T_h2d
+  T_(S,K)    sf_mttkrp_streamed with S segments over K streams
+  overlap    = (T_h2d + T_compute - T_(S,K)) / min(T_h2d, T_compute)
+and, for comparison, the resident path (create + plan + fragment MTTKRP) end to end.
+"""
+from __future__ import annotations
+
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+
+def main():
+    import torch
+
+    import paper_conf_cluster_linwds24_b200 as sf
+    names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["vast", "nell2"]
+    out = {}
+    for name in names:
+        cfg = synth.CONFIGS[name]
+        d_inds, d_vals = synth.config_tensor_device(cfg)
+        h_inds = [a.cpu().pin_memory() for a in d_inds]
+        h_vals = d_vals.cpu().pin_memory()
+        del d_inds, d_vals
+        facs = synth.config_factors_device(cfg)
+        n = 0
+        R = cfg.rank
+        y = torch.empty((cfg.dims[n], R), device="cuda")
+        dev_bufs = [torch.empty_like(a, device="cuda") for a in h_inds] + [torch.empty_like(h_vals, device="cuda")]
+
+        def wall(fn, reps=5):
+            fn()
+            torch.cuda.synchronize()
+            ts = []
+            for _ in range(reps):
+                t0 = time.perf_counter()
+                fn()
+                torch.cuda.synchronize()
+                ts.append(time.perf_counter() - t0)
+            return float(np.median(ts)) * 1e3
+
+        def h2d():
+            for dbuf, h in zip(dev_bufs, h_inds + [h_vals]):
+                dbuf.copy_(h, non_blocking=True)
+
+        t_h2d = wall(h2d)
+        grid = {}
+        for S in (1, 2, 4, 8, 16, 32):
+            for K in (1, 2, 4, 8):
+                if K > S:
+                    continue
+                grid[f"{S}x{K}"] = wall(lambda: sf.mttkrp_streamed(cfg.dims, h_inds, h_vals, facs, n, y, S, K))
+        t11 = grid["1x1"]
+        t_comp = max(t11 - t_h2d, 1e-6)
+        ov = {k: (t_h2d + t_comp - v) / min(t_h2d, t_comp) for k, v in grid.items()}
+
+        def resident():
+            with sf.Tensor(cfg.dims, h_inds, h_vals, segments=8, streams=4) as T:
+                T.plan(n, R)
+                T.mttkrp(n, facs, y)
+                torch.cuda.synchronize()
+        t_res = wall(resident, reps=3)
+        best = min(grid, key=grid.get)
+        out[name] = {"nnz": cfg.nnz, "bytes_h2d": int(sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4),
+                     "t_h2d_ms": t_h2d, "h2d_GBps": (sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4) / t_h2d / 1e6,
+                     "t_compute_ms": t_comp, "t_streamed_ms": grid, "overlap_ratio": ov,
+                     "best": best, "speedup_best_vs_1x1": t11 / grid[best],
+                     "t_resident_path_ms": t_res, "mode": n}
+        print(json.dumps({name: out[name]}), flush=True)
+    path = os.path.join(ROOT, "gpurun_out", "stream_study.json")
+    json.dump(out, open(path, "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()
