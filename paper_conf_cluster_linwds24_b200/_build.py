@@ -8,7 +8,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
-SO = os.path.join(HERE, "libscalfrag.so")
+SO = os.environ.get("SF_LIB_PATH") or os.path.join(HERE, "libscalfrag.so")  # override: A/B experiments
 BUILD = os.path.join(HERE, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 

@@ -53,7 +53,7 @@ def grid(dims, n, R, quick):
         opts = {m: sorted(set(row_opts + ([dims[m]] if dims[m] <= 2048 else []))) for m in st}
         rows_choices = [()] if not st else itertools.product(*[opts[m] for m in st])
         for rows in rows_choices:
-            for C, th, fl in itertools.product(chunks, threads, (2, 10)):
+            for C, th, fl in itertools.product(chunks, threads, (2,) if not st else (10,)):
                 yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl,
                        "staged": {m: min(r, dims[m]) for m, r in zip(st, rows)}}
     yield {"kernel": 1}
