@@ -203,10 +203,17 @@ def main():
     import paper_conf_cluster_linwds24_b200 as sf
     from paper_conf_cluster_linwds24_b200 import dist as sfdist
 
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+    # SF_SAME_GPU=1 (tests only): every rank on cuda:0 and gloo for the collectives -- lets
+    # the N>1 path (shards + boundary exchange + max over ranks) run on a 1-GPU box.
+    same_gpu = os.environ.get("SF_SAME_GPU") == "1"
+    local_dev = 0 if same_gpu else local_rank
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if same_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     N, R = cfg.nmodes, cfg.rank
 
     # ---- synthetic input (every rank holds the full raw COO, §8(e) v1), generated in HBM by
@@ -242,7 +249,12 @@ def main():
         plan_ms[n] = T.plan_info(n, R)["plan_ms"]
     infos = {n: T.plan_info(n, R) for n in range(N)}
     outs = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
-    exch = sfdist.BoundaryExchange(world, rank, R, dev) if world > 1 else None
+    exch = sfdist.BoundaryExchange(world, rank, R, dev, host_staging=same_gpu) if world > 1 else None
+
+    def max_over_ranks(x):
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if same_gpu else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
 
     def step(ev=None):
         for n in range(N):
@@ -262,7 +274,7 @@ def main():
            for _ in range(args.steps)]
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
-    clk = ClockSampler(local_rank)
+    clk = ClockSampler(local_dev)
     clk.start()
     time.sleep(0.3)
     launches0 = sf.kernel_launches()
@@ -280,9 +292,7 @@ def main():
     clocks = clk.stop()
     ms_total = t0.elapsed_time(t1)
     if world > 1:
-        tt = torch.tensor([ms_total], device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms_total = float(tt.item())
+        ms_total = max_over_ranks(ms_total)
     ms_step = ms_total / args.steps
     flops_step = flops_per_mode(cfg) * N
     value = flops_step / (ms_step * 1e-3) / 1e9
@@ -342,9 +352,7 @@ def main():
         torch.cuda.synchronize(dev)
         e2e_ms = (time.perf_counter() - s0) / args.e2e_steps * 1e3
         if world > 1:
-            tt = torch.tensor([e2e_ms], device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            e2e_ms = float(tt.item())
+            e2e_ms = max_over_ranks(e2e_ms)
         e2e = {"value": flops_step / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms,
                "steps": args.e2e_steps,

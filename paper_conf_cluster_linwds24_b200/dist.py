@@ -57,9 +57,12 @@ def owner_maps(ranges):
 class BoundaryExchange:
     """Caches the owner maps per (row_begin, row_end) and runs steps 1-4."""
 
-    def __init__(self, world, rank, R, device, rows_op=None, group=None):
+    def __init__(self, world, rank, R, device, rows_op=None, group=None, host_staging=False):
+        """host_staging: run the all_gather on CPU copies (gloo), for multi-rank tests on
+        one GPU where NCCL cannot be used (two ranks may not share a device)."""
         self.world, self.rank, self.R, self.device = world, rank, R, device
         self.group = group
+        self.host_staging = host_staging
         if rows_op is None:
             from . import rows_op as _rows_op
             rows_op = _rows_op
@@ -72,7 +75,8 @@ class BoundaryExchange:
     def _maps(self, row_begin, row_end):
         key = (int(row_begin), int(row_end))
         if key not in self._cache:
-            mine = torch.tensor([key[0], key[1]], dtype=torch.int64, device=self.device)
+            cdev = "cpu" if self.host_staging else self.device
+            mine = torch.tensor([key[0], key[1]], dtype=torch.int64, device=cdev)
             allr = [torch.empty_like(mine) for _ in range(self.world)]
             dist.all_gather(allr, mine, group=self.group)
             ranges = [tuple(int(x) for x in t.cpu().tolist()) for t in allr]
@@ -95,7 +99,15 @@ class BoundaryExchange:
         ctx = torch.cuda.stream(stream) if (stream is not None and Y.is_cuda) else _null()
         with ctx:
             self.rows_op(Y, pack, self.send, 0, stream)
-            dist.all_gather(self._recv_list, self.send, group=self.group)
+            if self.host_staging:
+                if Y.is_cuda:
+                    torch.cuda.current_stream().synchronize()
+                hs = self.send.cpu()
+                hr = [torch.empty_like(hs) for _ in range(self.world)]
+                dist.all_gather(hr, hs, group=self.group)
+                self.recv.copy_(torch.cat(hr, 0))
+            else:
+                dist.all_gather(self._recv_list, self.send, group=self.group)
             self.rows_op(Y, zero, None, 2, stream)
             self.rows_op(Y, tgt, self.recv, 1, stream)
         return Y
