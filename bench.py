@@ -315,6 +315,22 @@ def main():
         except Exception:
             traffic = None
 
+    # ---- the same step with re-planning (A2-A4 on the device-resident raw COO) ----
+    # Planning is a one-time cost per (mode, rank) in CP-ALS; reported beside `value` so the
+    # whole §8(a) path (sort + tiles + features + selection + kernel) is measured too.
+    auto = sf.Launch()
+    auto.kernel = 0
+    torch.cuda.synchronize(dev)
+    p0 = time.perf_counter()
+    for n in range(N):
+        T.set_launch(n, R, auto)  # SF_KERNEL_AUTO: re-plan with the selector
+        T.mttkrp(n, d_facs, outs[n], stream=stream)
+    torch.cuda.synchronize(dev)
+    plan_step_ms = (time.perf_counter() - p0) * 1e3
+    if world > 1:
+        plan_step_ms = max_over_ranks(plan_step_ms)
+    infos = {n: T.plan_info(n, R) for n in range(N)}
+
     # ---- e2e through the public API from pinned host buffers ----
     e2e = None
     if not args.no_e2e:
@@ -387,6 +403,10 @@ def main():
                                   "launch": infos[n]["launch"], "num_tiles": infos[n]["num_tiles"],
                                   "num_chunks": infos[n]["num_chunks"]}
                          for n in range(N)},
+            "plan_step": {"ms": plan_step_ms, "value": flops_step / (plan_step_ms * 1e-3) / 1e9,
+                          "unit": "GFLOP/s",
+                          "includes": "per mode: sf_plan (matricized sort, features, selection, tiles, "
+                                      "chunks) + sf_mttkrp, device-resident raw COO, host wall clock"},
             "gen_s": t_gen,
         }
         print(json.dumps(line), flush=True)

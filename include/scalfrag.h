@@ -70,11 +70,8 @@ typedef struct {
   uint32_t staged_mask;  /* FRAG: bit m set => factor m is staged in shared memory by
                             blocks of block_rows[m] rows (a "tensor block") */
   uint32_t block_rows[SF_MAX_MODES];
-  uint32_t flags;        /* FRAG: SF_LAUNCH_PREFETCH_L2 = prefetch each stretch's global
-                            factor rows into L2 before gathering (memory-level parallelism
-                            without registers) */
+  uint32_t flags;        /* FRAG: SF_LAUNCH_* bits below */
 } sf_launch_t;
-#define SF_LAUNCH_PREFETCH_L2 1u
 #define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
 #define SF_LAUNCH_NO_CARRY 8u /* FRAG: flush each stretch's last run (no cross-stretch carry) */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation

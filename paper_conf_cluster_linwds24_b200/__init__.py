@@ -23,7 +23,7 @@ _lib = None
 SF_MAX_MODES = 8
 SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
-LAUNCH_PREFETCH_L2 = 1
+LAUNCH_L1_NO_ALLOCATE, LAUNCH_NO_OWNER_STORES, LAUNCH_NO_CARRY = 2, 4, 8
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",
@@ -51,7 +51,7 @@ class Launch(ctypes.Structure):
     @classmethod
     def make(cls, kernel=KERNEL_FRAG, block_threads=512, ctas_per_sm=0, chunk_nnz=128,
              staged=None, flags=0):
-        """staged: {mode: block_rows}; flags: LAUNCH_PREFETCH_L2"""
+        """staged: {mode: block_rows}; flags: LAUNCH_* bits (include/scalfrag.h)"""
         l = cls()
         l.flags = flags
         l.kernel, l.block_threads, l.ctas_per_sm, l.chunk_nnz = kernel, block_threads, ctas_per_sm, chunk_nnz

@@ -46,13 +46,10 @@ struct FragParams {
   uint32_t stage_words;               // words per field per pipeline stage
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
   uint32_t row_end;                   // this shard's rows end (exclusive)
-  uint32_t prefetch;                  // launch flags: 1 L2 prefetch, 8 no carry
+  uint32_t flags;                     // launch flags (SF_LAUNCH_NO_CARRY)
 };
 
 constexpr int kFragStages = 2;
-#ifndef SF_LDG256_OP
-#define SF_LDG256_OP "ld.global.nc.v8.f32"
-#endif
 constexpr int kFragUnroll = 4;
 
 // Lane-group stretch of a chunk of n nonzeros (shared with the A5 boundary pre-pass):
@@ -84,29 +81,12 @@ __device__ __forceinline__ uint32_t su32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-__device__ __forceinline__ float4 lds128(uint32_t addr) {
-  float4 v;
-  asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "r"(addr));
-  return v;
-}
-
 __device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
 
-__device__ __forceinline__ void ldg256(const float4* p, float4& a, float4& b) {
-  asm(SF_LDG256_OP " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
-      : "l"(p));
-}
 __device__ __forceinline__ void ldg256_na(const float4* p, float4& a, float4& b) {
   asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
       : "l"(p));
-}
-
-__device__ __forceinline__ void prefetch_l2(const void* p) {
-  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -329,23 +309,6 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
           }
           return r;
         };
-        // Memory-level parallelism without registers: request every global row of this
-        // stretch into L2 up front (one 32-byte sector per lane), then gather.
-        if constexpr (G - S > 0) {
-          if ((p.prefetch & 1u) && (VEC == 8 || (lane_in_group & 1) == 0)) {
-            for (uint32_t kk = k0; kk < k1; ++kk) {
-#pragma unroll
-              for (int q = S; q < G; ++q)
-                prefetch_l2(gbase[q - S] + (size_t)sIdx[q][kk] * R4 + c0);
-            }
-          }
-        }
-        // A5 (owner mode, unstaged plans only): runs wholly inside this stretch are
-        // STORED (this group owns the row); the stretch's first/last run is atomically
-        // added when it continues into the neighbouring stretch (those rows were zeroed by
-        // the boundary pre-pass); empty rows between runs are zeroed by the group that
-        // owns the run after the gap.  Otherwise (staged tiles) Y was memset and every
-        // flush is an atomic.
         bool shared = true;       // current run may be shared with another stretch/tile
         bool last_shared = true;  // the stretch's last run continues past k1
         const uint32_t first = sOut[k0];
@@ -459,7 +422,7 @@ __global__ void __launch_bounds__(1024) frag_kernel(const FragParams p) {
         }
         // carry only a run that filled the whole stretch (a heavy row); shorter runs that
         // merely cross the boundary are flushed now (cheaper, and their chains are short)
-        if (last_shared && first == cur && !(p.prefetch & 8u)) {
+        if (last_shared && first == cur && !(p.flags & SF_LAUNCH_NO_CARRY)) {
           carry = true;  // the run continues past this stretch: keep accumulating
         } else {
           flush_run(shared || last_shared);  // a run crossing into the next stretch is shared

@@ -297,7 +297,7 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   fp.nnz = (uint32_t)p.nnz_local;
   fp.mode = n;
   fp.stage_words = (uint32_t)p.launch.chunk_nnz + 8;
-  fp.prefetch = p.launch.flags & (SF_LAUNCH_PREFETCH_L2 | SF_LAUNCH_NO_CARRY);
+  fp.flags = p.launch.flags;
   fp.owner = owner ? 1u : 0u;
   fp.row_end = (uint32_t)p.row_end;
   // slots: staged modes first (ascending mode id = tile-id fold order), then the rest

@@ -287,15 +287,6 @@ struct GatherParams {
   int nmodes;
 };
 
-__global__ void gather_kernel(GatherParams g, const uint32_t* __restrict__ perm, uint64_t n) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    const uint32_t e = perm[k];
-    for (int m = 0; m < g.nmodes; ++m) g.dst[m][k] = g.src[m][e];
-    g.vdst[k] = g.vsrc[e];
-  }
-}
-
 // Chunk start flags: k starts a chunk iff (k - tile_start(k)) % C == 0.
 __global__ void tile_start_kernel(const uint64_t* __restrict__ tkey, uint64_t n, uint32_t* __restrict__ ts,
                                   unsigned long long* __restrict__ ntiles) {

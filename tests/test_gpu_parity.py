@@ -215,3 +215,17 @@ def test_kernel_launch_counter(cuda_device):
     cfg, inds, vals, facs = _cfg_data("tiny")
     G.run(cfg.dims, inds, vals, facs, cfg.rank, modes=[0])
     assert sf.kernel_launches() > before
+
+
+@pytest.mark.parametrize("dims,R", [((4, 5, 3, 6, 2, 3), 4), ((3, 4, 2, 5, 3, 2, 4, 2), 3),
+                                    ((50, 1, 40), 32), ((1, 70, 60), 16), ((20, 30, 25), 128)])
+def test_generic_paths_and_degenerate_dims(cuda_device, dims, R):
+    """N = 6..8 and R = 128 run the generic COO kernel; size-1 modes; exact integers."""
+    nnz = 1500
+    inds, vals = synth.gen_coo(dims, nnz, 3, val_kind="int")
+    facs = synth.gen_factors(dims, R, 4, "int")
+    Y, _ = G.run(dims, inds, vals, facs, R)
+    for n in range(len(dims)):
+        Yo, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
+        assert np.max(S) < 2 ** 24
+        assert np.array_equal(Y[n].astype(np.float64), Yo), n
