@@ -69,6 +69,8 @@ struct Plan {
   // kernel-order arrays (SoA): sorted indices of every mode + values + input position
   DevBuf ind[SF_MAX_MODES];
   DevBuf val;
+  DevBuf rec;           // frag3 plans: kernel-order records in slot order (rec_words each)
+  int rec_words = 0;    // 0: SoA arrays (ind/val) instead of records
   DevBuf perm;          // uint32 input position per sorted slot
   DevBuf chunk_begin;   // uint32[num_chunks + 1]
   DevBuf chunk_tile;    // uint64[num_chunks]
@@ -106,6 +108,33 @@ inline int secondary_mode(const Tensor& t, int mode) {
   return s;
 }
 
+// ---- frag3 layout helpers (shared by the planner, the selector and the kernel) ----
+template <int N>
+struct RecWords {
+  static constexpr int W = (N + 1 <= 4) ? 4 : 8;
+};
+
+__host__ __device__ inline int rec_words_for(int N) { return (N + 1 <= 4) ? 4 : 8; }
+
+// Region stride (words) of one group's K records: W*K + pad with stride/4 odd, so the
+// GPW groups' record k (read in lockstep) fall into distinct 16-byte bank quads.
+__host__ __device__ __forceinline__ uint32_t frag3_region_words(uint32_t K, uint32_t W) {
+  const uint32_t base = K * W;
+  return ((base / 4u) % 2u == 0u) ? base + 4u : base + 8u;
+}
+
+// Records per group per stage for a launch's chunk_nnz (nonzeros per warp per stage).
+__host__ __device__ __forceinline__ uint32_t frag3_K(uint32_t chunk_nnz, uint32_t GPW) {
+  uint32_t K = chunk_nnz / GPW;
+  return K < 4u ? 4u : K;
+}
+
+// Lane groups per warp of the fragment kernels for rank R (LaneMap<R> in sf_frag.cuh).
+inline int frag_groups_per_warp(int R) {
+  const int lpn = R >= 32 ? R / 8 : R / 4;
+  return lpn >= 1 && lpn <= 32 ? 32 / lpn : 1;
+}
+
 // ---- planning (sf_plan.cu) ----
 // keys/pos (optional): receive the matricized order (sorted keys, input positions) when
 // this call had to sort, so build_plan can reuse it instead of sorting again.
@@ -132,6 +161,11 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
                 cudaStream_t s);
 int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem);
 bool frag_supported(int nmodes, int rank);
+// Fragment-kernel implementation: 3 = record-packed group-contiguous frag3_kernel (default),
+// 2 = SoA chunk-stretch frag_kernel (env SF_FRAG_IMPL=2, kept for A/B measurements).
+int frag_impl();
+// gathered slot order of a plan: staged modes ascending, then the other gathered modes
+int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode);
 void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s);
 void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
                       uint32_t* const* inds, int* d_flag, cudaStream_t s);

@@ -28,6 +28,8 @@
 #include <cstdio>
 
 #include "sf_frag.cuh"
+#include "sf_frag3.cuh"
+#include <cstdlib>
 #include "sf_internal.h"
 
 namespace sf {
@@ -251,6 +253,95 @@ static void frag_launch(int N, int R, int S, const FragParams& fp, int grid, int
   }
 }
 
+int frag_impl() {
+  static const int impl = [] {
+    const char* e = std::getenv("SF_FRAG_IMPL");
+    return (e && std::atoi(e) == 2) ? 2 : 3;
+  }();
+  return impl;
+}
+
+int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode) {
+  int q = 0;
+  for (int m = 0; m < nmodes; ++m)
+    if (m != mode && (staged_mask & (1u << m))) slot_mode[q++] = m;
+  const int S = q;
+  for (int m = 0; m < nmodes; ++m)
+    if (m != mode && !(staged_mask & (1u << m))) slot_mode[q++] = m;
+  return S;
+}
+
+static int frag3_occ(int N, int R, int S, int threads, size_t smem) {
+  switch (R) {
+    case 16: return frag3_occ_r16(N, S, threads, smem);
+    case 32: return frag3_occ_r32(N, S, threads, smem);
+    case 64: return frag3_occ_r64(N, S, threads, smem);
+    default: return 0;
+  }
+}
+
+// frag3 path (record plans): A5 owner pre-pass on the frag3 group partition, then the kernel.
+static void launch_frag3(const Tensor& t, const Plan& p, const float* const* factors, float* out,
+                         cudaStream_t s, bool owner) {
+  const int N = t.nmodes, R = p.rank, n = p.mode;
+  Frag3Params fp{};
+  for (int m = 0; m < N; ++m) {
+    fp.fac[m] = factors[m];
+    fp.dims[m] = (uint32_t)t.dims[m];
+  }
+  fp.rec = p.rec.as<uint32_t>();
+  fp.out = out;
+  fp.chunk_begin = p.chunk_begin.as<uint32_t>();
+  fp.chunk_tile = p.chunk_tile.as<uint64_t>();
+  fp.num_chunks = (uint32_t)p.num_chunks;
+  fp.nnz = (uint32_t)p.nnz_local;
+  const uint32_t gpw = (uint32_t)frag_groups_per_warp(R);
+  fp.K = frag3_K((uint32_t)p.launch.chunk_nnz, gpw);
+  fp.W = (uint32_t)p.rec_words;
+  fp.owner = owner ? 1u : 0u;
+  const int S = frag_slot_order(N, n, p.launch.staged_mask, fp.slot_mode);
+  uint32_t off = 0;
+  for (int q = 0; q < S; ++q) {
+    const int m = fp.slot_mode[q];
+    fp.block_rows[q] = p.launch.block_rows[m];
+    fp.ntiles[q] = (uint32_t)((t.dims[m] + fp.block_rows[q] - 1) / fp.block_rows[q]);
+    fp.fac_off[q] = off;
+    off += fp.block_rows[q] * (uint32_t)R;
+  }
+  const size_t smem = frag_smem_bytes(t, n, R, p.launch);
+  const int threads = p.launch.block_threads;
+  int per_sm = p.launch.ctas_per_sm;
+  const int occ = frag3_occ(N, R, S, threads, smem);
+  if (occ <= 0) throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: launch does not fit an SM"};
+  if (per_sm <= 0 || per_sm > occ) per_sm = occ;
+  int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
+  grid = std::max(grid, 1);
+  if (owner) {
+    const uint32_t groups = (uint32_t)(threads / 32) * gpw;
+    switch (R) {
+      case 16: boundary_zero3_r16(fp, (uint32_t)grid, groups, out, s); break;
+      case 32: boundary_zero3_r32(fp, (uint32_t)grid, groups, out, s); break;
+      default: boundary_zero3_r64(fp, (uint32_t)grid, groups, out, s); break;
+    }
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+  }
+  switch (R) {
+    case 16: frag3_launch_r16(N, S, fp, grid, threads, smem, s); break;
+    case 32: frag3_launch_r32(N, S, fp, grid, threads, smem, s); break;
+    case 64: frag3_launch_r64(N, S, fp, grid, threads, smem, s); break;
+    default: throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: unsupported rank"};
+  }
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    char msg[256];
+    snprintf(msg, sizeof msg, "frag3_kernel<%d,%d,%d> launch grid=%d threads=%d smem=%zu occ=%d: %s", N, R, S,
+             grid, threads, smem, occ, cudaGetErrorString(e));
+    throw StatusError{SF_ERR_CUDA, msg};
+  }
+}
+
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
                    cudaStream_t s) {
   const int N = t.nmodes, R = p.rank, n = p.mode;
@@ -262,6 +353,10 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   const size_t row_bytes = sizeof(float) * (size_t)R;
   if (!owner) {
     SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * t.dims[n], s));
+  } else if (p.rec_words) {  // frag3: rows outside the shard; the pre-pass runs in launch_frag3
+    if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
+    if (p.row_end < t.dims[n])
+      SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (t.dims[n] - p.row_end), s));
   } else {
     if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
     if (p.row_end < t.dims[n])
@@ -277,6 +372,7 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
     SF_CUDA(cudaGetLastError());
   }
   if (p.nnz_local == 0) return;
+  if (frag && p.rec_words) return launch_frag3(t, p, factors, out, s, owner);
   if (!frag) {
     uint32_t* ind[SF_MAX_MODES];
     for (int m = 0; m < N; ++m) ind[m] = p.ind[m].as<uint32_t>();

@@ -279,6 +279,38 @@ __global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32
   }
 }
 
+// frag3 records: kernel-order record k = [raw field fmap[0], ..., fmap[WK-1]] of the raw
+// AoS record perm[k] (fmap < 0: zero padding).  Slot order: i_n, gathered slots, value.
+struct RecParams {
+  int fmap[8];
+};
+
+template <int WR, int WK>
+__global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
+                                  uint64_t n, RecParams rp, uint32_t* __restrict__ rec) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)perm[k] * WR);
+    uint32_t w[WR];
+#pragma unroll
+    for (int q = 0; q < WR / 4; ++q) {
+      const uint4 v = __ldg(src + q);
+      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
+    }
+    uint32_t o[WK];
+#pragma unroll
+    for (int d = 0; d < WK; ++d) {
+      uint32_t x = 0;
+#pragma unroll
+      for (int q = 0; q < WR; ++q) x = (rp.fmap[d] == q) ? w[q] : x;
+      o[d] = x;
+    }
+    uint4* dst = reinterpret_cast<uint4*>(rec + k * WK);
+#pragma unroll
+    for (int q = 0; q < WK / 4; ++q) dst[q] = make_uint4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+  }
+}
+
 struct GatherParams {
   const uint32_t* src[SF_MAX_MODES];
   uint32_t* dst[SF_MAX_MODES];
@@ -406,48 +438,76 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     }
   }
 
-  // Gather the kernel-order SoA arrays (padded for aligned bulk copies).
-  GatherParams g{};
-  for (int m = 0; m < N; ++m) {
-    p.ind[m].alloc(nl * 4 + kPadBytes);
-    SF_CUDA(cudaMemsetAsync(p.ind[m].p, 0, nl * 4 + kPadBytes, t.stream));
-    g.src[m] = t.ind[m].as<uint32_t>();
-    g.dst[m] = p.ind[m].as<uint32_t>();
-  }
-  p.val.alloc(nl * 4 + kPadBytes);
-  SF_CUDA(cudaMemsetAsync(p.val.p, 0, nl * 4 + kPadBytes, t.stream));
-  g.vsrc = t.val.as<float>();
-  g.vdst = p.val.as<float>();
-  g.nmodes = N;
-  if (nl) {
-    // AoS record copy of the raw COO (built once per tensor, reused by every mode's plan)
-    const int W = (N + 1 <= 4) ? 4 : (N + 1 <= 8 ? 8 : 16);
-    if (!t.aos.p) {
-      t.aos.alloc((size_t)n * W * 4 + 64);
-      AosParams a{};
-      for (int m = 0; m < N; ++m) a.ind[m] = t.ind[m].as<uint32_t>();
-      a.val = t.val.as<float>();
-      a.aos = t.aos.as<uint32_t>();
-      a.nmodes = N;
-      a.W = W;
-      build_aos_kernel<<<grid_for(n), 256, 0, t.stream>>>(a, n);
-      count_launch();
-      SF_CUDA(cudaGetLastError());
-      t.aos_words = W;
-    }
-    DevBuf dptr(sizeof(uint32_t*) * SF_MAX_MODES);
-    uint32_t* hptr[SF_MAX_MODES] = {};
-    for (int m = 0; m < N; ++m) hptr[m] = g.dst[m];
-    SF_CUDA(cudaMemcpyAsync(dptr.p, hptr, sizeof(hptr), cudaMemcpyHostToDevice, t.stream));
-    uint32_t* const* dd = reinterpret_cast<uint32_t* const*>(dptr.p);
-    switch (W) {
-      case 4: gather_aos_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
-      case 8: gather_aos_kernel<8><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
-      default: gather_aos_kernel<16><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
-    }
+  // AoS record copy of the raw COO (built once per tensor, reused by every mode's plan)
+  const int WR = (N + 1 <= 4) ? 4 : (N + 1 <= 8 ? 8 : 16);
+  if (nl && !t.aos.p) {
+    t.aos.alloc((size_t)n * WR * 4 + 64);
+    AosParams a{};
+    for (int m = 0; m < N; ++m) a.ind[m] = t.ind[m].as<uint32_t>();
+    a.val = t.val.as<float>();
+    a.aos = t.aos.as<uint32_t>();
+    a.nmodes = N;
+    a.W = WR;
+    build_aos_kernel<<<grid_for(n), 256, 0, t.stream>>>(a, n);
     count_launch();
     SF_CUDA(cudaGetLastError());
-    SF_CUDA(cudaStreamSynchronize(t.stream));  // dptr's host source must outlive the copy
+    t.aos_words = WR;
+  }
+  const bool use_rec = launch.kernel == SF_KERNEL_FRAG && frag_supported(N, rank) && frag_impl() == 3;
+  p.rec_words = 0;
+  if (use_rec) {
+    // frag3 records in slot order [i_n, staged slots, other gathered slots, value, 0...]
+    const int WK = rec_words_for(N);
+    p.rec_words = WK;
+    p.rec.alloc(nl * WK * 4 + kPadBytes);
+    SF_CUDA(cudaMemsetAsync(p.rec.as<uint32_t>() + nl * WK, 0, kPadBytes, t.stream));
+    RecParams rp{};
+    for (int d = 0; d < 8; ++d) rp.fmap[d] = -1;
+    int slot_mode[SF_MAX_MODES];
+    frag_slot_order(N, mode, launch.staged_mask, slot_mode);
+    rp.fmap[0] = mode;
+    for (int q = 0; q < N - 1; ++q) rp.fmap[1 + q] = slot_mode[q];
+    rp.fmap[N] = N;  // value word of the raw record
+    if (nl) {
+      const uint32_t* aos = t.aos.as<uint32_t>();
+      const uint32_t* pm = perm.as<uint32_t>();
+      uint32_t* rec = p.rec.as<uint32_t>();
+      if (WR == 4 && WK == 4) gather_rec_kernel<4, 4><<<grid_for(nl), 256, 0, t.stream>>>(aos, pm, nl, rp, rec);
+      else if (WR == 8 && WK == 8) gather_rec_kernel<8, 8><<<grid_for(nl), 256, 0, t.stream>>>(aos, pm, nl, rp, rec);
+      else throw StatusError{SF_ERR_UNSUPPORTED, "frag3 records: unsupported record width"};
+      count_launch();
+      SF_CUDA(cudaGetLastError());
+    }
+  } else {
+    // Gather the kernel-order SoA arrays (padded for aligned bulk copies).
+    GatherParams g{};
+    for (int m = 0; m < N; ++m) {
+      p.ind[m].alloc(nl * 4 + kPadBytes);
+      SF_CUDA(cudaMemsetAsync(p.ind[m].p, 0, nl * 4 + kPadBytes, t.stream));
+      g.src[m] = t.ind[m].as<uint32_t>();
+      g.dst[m] = p.ind[m].as<uint32_t>();
+    }
+    p.val.alloc(nl * 4 + kPadBytes);
+    SF_CUDA(cudaMemsetAsync(p.val.p, 0, nl * 4 + kPadBytes, t.stream));
+    g.vsrc = t.val.as<float>();
+    g.vdst = p.val.as<float>();
+    g.nmodes = N;
+    if (nl) {
+      const int W = WR;
+      DevBuf dptr(sizeof(uint32_t*) * SF_MAX_MODES);
+      uint32_t* hptr[SF_MAX_MODES] = {};
+      for (int m = 0; m < N; ++m) hptr[m] = g.dst[m];
+      SF_CUDA(cudaMemcpyAsync(dptr.p, hptr, sizeof(hptr), cudaMemcpyHostToDevice, t.stream));
+      uint32_t* const* dd = reinterpret_cast<uint32_t* const*>(dptr.p);
+      switch (W) {
+        case 4: gather_aos_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+        case 8: gather_aos_kernel<8><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+        default: gather_aos_kernel<16><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
+      }
+      count_launch();
+      SF_CUDA(cudaGetLastError());
+      SF_CUDA(cudaStreamSynchronize(t.stream));  // dptr's host source must outlive the copy
+    }
   }
   p.perm = std::move(perm);
 

@@ -27,7 +27,13 @@ size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l
   (void)mode;
   const size_t nwarps = (size_t)std::max(1, l.block_threads / 32);
   size_t b = ((2 * nwarps + 1) * 8 + 127) & ~(size_t)127;
-  b += nwarps * kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
+  if (frag_impl() == 3) {  // frag3: per warp 2 stages x GPW regions of K records
+    const uint32_t gpw = (uint32_t)frag_groups_per_warp(rank);
+    const uint32_t K = frag3_K((uint32_t)l.chunk_nnz, gpw);
+    b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)rec_words_for(t.nmodes)) * 4;
+  } else {
+    b += nwarps * kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
+  }
   for (int m = 0; m < t.nmodes; ++m)
     if (l.staged_mask & (1u << m)) b += (size_t)l.block_rows[m] * rank * 4;
   return b;

@@ -44,7 +44,7 @@ def time_launch(T, n, R, facs, out, L, sf, torch, reps=5):
 def grid(dims, n, R, quick):
     others = [m for m in range(len(dims)) if m != n]
     row_opts = [128, 256, 384, 512, 775] if not quick else [256, 512]
-    chunks = [64, 128, 256] if not quick else [128]
+    chunks = [64, 128, 256, 512] if not quick else [128]
     threads = [256, 512, 1024] if not quick else [512]
     staged_sets = [()]
     for k in range(1, len(others) + 1):
