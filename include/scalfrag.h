@@ -74,6 +74,8 @@ typedef struct {
 } sf_launch_t;
 #define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
 #define SF_LAUNCH_NO_CARRY 8u /* FRAG: flush each stretch's last run (no cross-stretch carry) */
+#define SF_LAUNCH_DETERMINISTIC 32u /* FRAG: A7 two-pass carry combine instead of atomics; forces an
+                                       unstaged owner-store plan; Y is bitwise reproducible run to run */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation
                                        (ld.global.nc.L1::no_allocate.v8.f32; measured faster) */
 
@@ -82,7 +84,7 @@ typedef struct {
   uint64_t nnz;
   uint64_t dim;               /* I_n */
   uint64_t num_slices;        /* non-empty rows of mode n */
-  uint64_t num_fibers;        /* distinct (i_n, i_s) pairs, s = highest mode != n */
+  uint64_t num_fibers;        /* distinct (i_n, i_s) pairs, s = secondary (smallest gathered) mode */
   uint64_t max_nnz_per_slice;
   uint64_t max_nnz_per_fiber;
   uint64_t sum_sq_nnz_per_slice;

@@ -24,6 +24,7 @@ SF_MAX_MODES = 8
 SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
 LAUNCH_L1_NO_ALLOCATE, LAUNCH_NO_OWNER_STORES, LAUNCH_NO_CARRY = 2, 4, 8
+LAUNCH_DETERMINISTIC = 32
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",
@@ -266,8 +267,13 @@ class Tensor:
     def set_shard(self, nranks, rank):
         _check(lib().sf_set_shard(self._h, int(nranks), int(rank)))
 
-    def plan(self, mode, rank):
-        _check(lib().sf_plan(self._h, int(mode), int(rank)))
+    def plan(self, mode, rank, deterministic=False):
+        """sf_plan (selector's launch); deterministic=True plans the A7 two-pass carry
+        combine instead (unstaged owner-store fragment plan, bitwise reproducible Y)."""
+        if deterministic:
+            self.set_launch(mode, rank, Launch.make(kernel=KERNEL_FRAG, flags=LAUNCH_DETERMINISTIC))
+        else:
+            _check(lib().sf_plan(self._h, int(mode), int(rank)))
 
     def plan_release(self, mode, rank):
         _check(lib().sf_plan_release(self._h, int(mode), int(rank)))

@@ -57,6 +57,11 @@ struct Frag3Params {
   uint32_t K;                         // records per group per stage
   uint32_t W;                         // words per record (== RecWords<N>::W)
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
+  // A7 deterministic option (owner mode only): shared runs go to per-group carry slots
+  // (head = 2*gid, tail = 2*gid+1, gid = blockIdx.x * groups + group) instead of atomics;
+  // frag3_combine_kernel then adds them per row in slot order.
+  uint32_t* carry_row;                // [2 * grid * groups], 0xFFFFFFFF = empty (memset per launch)
+  float* carry_val;                   // [2 * grid * groups * R]
 };
 
 namespace detail {
@@ -205,8 +210,33 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     bool shared = first_shared;
     uint32_t cur = 0;
     float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
+    auto gather = [&](int q, uint32_t row_idx) -> F8 {
+      const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
+      const size_t row = (size_t)row_idx * R4;
+      F8 r;
+      if constexpr (VEC == 8) {
+        if (q < S) {
+          const float4 x = base[row + c0 + par];
+          const float4 y = base[row + c0 + 1 - par];
+          r.a = par ? y : x;
+          r.b = par ? x : y;
+        } else {
+          ldg256_na(base + row + c0, r.a, r.b);
+        }
+      } else {
+        r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
+      }
+      return r;
+    };
+    bool advanced = false;  // the first run of the sub-range has been closed
     auto flush_run = [&](bool atomic) {
-      if (atomic) {
+      if (atomic && p.carry_row) {  // deterministic: park the partial in this group's slot
+        const size_t slot = 2 * ((size_t)blockIdx.x * Gam + gam) + (advanced ? 1 : 0);
+        if (lane_in_group == 0) p.carry_row[slot] = cur;
+        float* dst = p.carry_val + slot * R + 4 * c0;
+        if constexpr (VEC == 8) st256(dst, acc0, acc1);
+        else st128(dst, acc0);
+      } else if (atomic) {
         red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
         if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
       } else {
@@ -225,6 +255,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     };
     auto advance = [&](uint32_t i) {  // run edge inside the sub-range: close `cur`, open i
       flush_run(shared);
+      advanced = true;
       if constexpr (S == 0) {
         if (p.owner) {
           zero_rows(cur, i);
@@ -247,24 +278,6 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
             if (p.owner && !first_shared && gs > 0) zero_rows(before, cur);  // gap rows are ours
           }
         }
-        auto gather = [&](int q, uint32_t row_idx) -> F8 {
-          const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
-          const size_t row = (size_t)row_idx * R4;
-          F8 r;
-          if constexpr (VEC == 8) {
-            if (q < S) {
-              const float4 x = base[row + c0 + par];
-              const float4 y = base[row + c0 + 1 - par];
-              r.a = par ? y : x;
-              r.b = par ? x : y;
-            } else {
-              ldg256_na(base + row + c0, r.a, r.b);
-            }
-          } else {
-            r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
-          }
-          return r;
-        };
         // record k of this group: [i_n, g_0 .. g_{G-1}, v]
         auto load_rec = [&](uint32_t k, uint32_t& i, uint32_t (&g)[G], float& v) {
           const uint32_t* rp = reg + (size_t)k * W;
@@ -355,6 +368,35 @@ __global__ void boundary_zero3_kernel(const uint32_t* __restrict__ chunk_begin, 
     float4* y = reinterpret_cast<float4*>(out + (size_t)r * R);
 #pragma unroll
     for (int q = 0; q < R / 4; ++q) y[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+}
+
+// A7 deterministic combine: one warp per carry slot; the first non-empty slot of a row
+// sums that row's slots in slot order (= nonzero order) and stores the row.
+static __global__ void frag3_combine_kernel(const uint32_t* __restrict__ carry_row, const float* __restrict__ carry_val,
+                                     uint64_t nslots, int R, float* __restrict__ out) {
+  const uint64_t warps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  for (uint64_t k = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < nslots; k += warps) {
+    const uint32_t r = carry_row[k];
+    if (r == 0xFFFFFFFFu) continue;
+    uint64_t prev = k;
+    uint32_t pr = 0xFFFFFFFFu;
+    while (prev > 0) {
+      pr = carry_row[--prev];
+      if (pr != 0xFFFFFFFFu) break;
+    }
+    if (pr == r) continue;  // not the first slot of row r
+    for (int c = lane; c < R; c += 32) {
+      float sum = 0.f;
+      for (uint64_t q = k; q < nslots; ++q) {
+        const uint32_t rq = carry_row[q];
+        if (rq == 0xFFFFFFFFu) continue;
+        if (rq != r) break;
+        sum += carry_val[q * R + c];
+      }
+      out[(size_t)r * R + c] = sum;
+    }
   }
 }
 

@@ -74,6 +74,7 @@ struct Plan {
   DevBuf perm;          // uint32 input position per sorted slot
   DevBuf chunk_begin;   // uint32[num_chunks + 1]
   DevBuf chunk_tile;    // uint64[num_chunks]
+  mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
   size_t device_bytes() const;
 };
 

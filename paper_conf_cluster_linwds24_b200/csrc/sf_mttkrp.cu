@@ -308,16 +308,25 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     fp.fac_off[q] = off;
     off += fp.block_rows[q] * (uint32_t)R;
   }
-  const size_t smem = frag_smem_bytes(t, n, R, p.launch);
-  const int threads = p.launch.block_threads;
-  int per_sm = p.launch.ctas_per_sm;
+  const sf_launch_t& l = p.launch;
+  const size_t smem = frag_smem_bytes(t, n, R, l);
+  const int threads = l.block_threads;
+  int per_sm = l.ctas_per_sm;
   const int occ = frag3_occ(N, R, S, threads, smem);
   if (occ <= 0) throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: launch does not fit an SM"};
   if (per_sm <= 0 || per_sm > occ) per_sm = occ;
   int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
   grid = std::max(grid, 1);
-  if (owner) {
-    const uint32_t groups = (uint32_t)(threads / 32) * gpw;
+  const uint32_t groups = (uint32_t)(threads / 32) * gpw;
+  const bool det = owner && (l.flags & SF_LAUNCH_DETERMINISTIC);
+  const uint64_t nslots = 2ull * (uint64_t)grid * groups;
+  if (det) {  // A7 deterministic option: carry slots instead of atomics (no pre-zero needed)
+    const size_t need = nslots * 4 + 16 + nslots * (size_t)R * 4;
+    if (p.carry.bytes < need) { p.carry.release(); p.carry.alloc(need); }
+    fp.carry_row = p.carry.as<uint32_t>();
+    fp.carry_val = reinterpret_cast<float*>(p.carry.as<unsigned char>() + ((nslots * 4 + 15) & ~(size_t)15));
+    SF_CUDA(cudaMemsetAsync(fp.carry_row, 0xFF, nslots * 4, s));
+  } else if (owner) {
     switch (R) {
       case 16: boundary_zero3_r16(fp, (uint32_t)grid, groups, out, s); break;
       case 32: boundary_zero3_r32(fp, (uint32_t)grid, groups, out, s); break;
@@ -339,6 +348,12 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     snprintf(msg, sizeof msg, "frag3_kernel<%d,%d,%d> launch grid=%d threads=%d smem=%zu occ=%d: %s", N, R, S,
              grid, threads, smem, occ, cudaGetErrorString(e));
     throw StatusError{SF_ERR_CUDA, msg};
+  }
+  if (det) {
+    const int cgrid = (int)std::max<uint64_t>(1, std::min<uint64_t>((nslots * 32 + 255) / 256, 148 * 16));
+    frag3_combine_kernel<<<cgrid, 256, 0, s>>>(fp.carry_row, fp.carry_val, nslots, R, out);
+    count_launch();
+    SF_CUDA(cudaGetLastError());
   }
 }
 

@@ -58,6 +58,11 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   }
   for (int m = N; m < SF_MAX_MODES; ++m) l.block_rows[m] = 0;
   l.staged_mask = (l.kernel == SF_KERNEL_FRAG) ? mask : 0u;
+  if (l.flags & SF_LAUNCH_DETERMINISTIC) {  // A7 option: unstaged owner-store plan (no atomics)
+    l.staged_mask = 0u;
+    for (int m = 0; m < SF_MAX_MODES; ++m) l.block_rows[m] = 0;
+    l.flags &= ~SF_LAUNCH_NO_OWNER_STORES;
+  }
 }
 
 // Selector rules, calibrated on the sweeps in profiles/:
