@@ -9,12 +9,13 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 SO = os.environ.get("SF_LIB_PATH") or os.path.join(HERE, "libscalfrag.so")  # override: A/B experiments
-BUILD = os.path.join(HERE, "build")
+BUILD = os.environ.get("SF_BUILD_DIR") or os.path.join(HERE, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
                 "--expt-relaxed-constexpr", "-Xptxas", "-v", "-I", os.path.join(ROOT, "include")]
+FLAGS += os.environ.get("SF_NVCC_EXTRA", "").split()  # A/B builds (with SF_LIB_PATH), e.g. -DSF_R16_VEC=8
 SOURCES = ["sf_api.cu", "sf_plan.cu", "sf_mttkrp.cu", "sf_select.cpp", "sf_cpals.cu", "sf_frag_r16.cu",
            "sf_frag_r32.cu", "sf_frag_r64.cu"]
 

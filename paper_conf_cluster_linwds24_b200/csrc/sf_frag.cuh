@@ -129,7 +129,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 // VEC = 4: lane t owns chunk t.
 template <int R>
 struct LaneMap {
-  static constexpr int VEC = (R >= 32) ? 8 : 4;
+  static constexpr int VEC = (R >= 32) ? 8 : 4;  // R = 16 with VEC = 8: 15-30 % slower (profiles/r01_frag3)
   static constexpr int LPN = R / VEC;
 };
 

@@ -9,6 +9,9 @@
 //      [i_n, g_0, ..., g_{N-2}, v, pad] (W = 4 for N <= 3, 8 for N <= 7), so a lane group
 //      reads its nonzero with one (W = 4) or two 128-bit shared loads instead of N+1
 //      32-bit loads, and one TMA bulk copy moves a group's K records per stage.
+//      PK (N >= 4 with sum_m bits(I_m) <= 96): the N indices are bit-packed into words
+//      0..2 (field f at bit p.boff[f], width from p.bmask[f]; i_n at bit 0) and v is
+//      word 3, so N = 4, 5 records stay 16 bytes (the SoA layout streams 4(N+1)).
 //   2. Group-contiguous work.  Each tile segment of a CTA's range (the CTA range is
 //      nnz-balanced as before) is cut into Gamma = warps x groups equal contiguous
 //      sub-ranges, one per lane group; a group walks its sub-range stage by stage, so a
@@ -55,7 +58,15 @@ struct Frag3Params {
   uint32_t dims[SF_MAX_MODES];        // per mode
   uint32_t fac_off[SF_MAX_MODES];     // per staged slot: float offset of its block in smem
   uint32_t K;                         // records per group per stage
-  uint32_t W;                         // words per record (== RecWords<N>::W)
+  uint32_t W;                         // words per record (== RecWords<N, PK>::W)
+  uint32_t boff[SF_MAX_MODES];        // PK: bit offset of field f (slot order, f = 0 is i_n)
+  uint32_t bmask[SF_MAX_MODES];       // PK: (1 << width) - 1 of field f
+  uint32_t out_mask;                  // mask applied to word 0 to read i_n (PK: bmask[0])
+  // TEX gathers: global slots q with bit q of texmask read their factor rows through the
+  // texture pipeline (tex1Dfetch<float4> on tex[q]) instead of LDG -- a second data path
+  // into registers next to the LSU one, which binds with L2-resident factors.
+  uint32_t texmask;
+  unsigned long long tex[SF_MAX_MODES];
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
   // A7 deterministic option (owner mode only): shared runs go to per-group carry slots
   // (head = 2*gid, tail = 2*gid+1, gid = blockIdx.x * groups + group) instead of atomics;
@@ -75,7 +86,16 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ uint4 lds128(const uint32_t* p) { return *reinterpret_cast<const uint4*>(p); }
 }  // namespace detail
 
-template <int N, int R, int S>
+// Field f of a packed record (words w0..w2): bits [off, off + width) -- a field never
+// spans more than two consecutive words (width <= 32).
+__device__ __forceinline__ uint32_t pk_field(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t off, uint32_t mask) {
+  const uint32_t wi = off >> 5, sh = off & 31u;
+  const uint32_t lo = wi == 0 ? w0 : (wi == 1 ? w1 : w2);
+  const uint32_t hi = wi == 0 ? w1 : (wi == 1 ? w2 : 0u);
+  return __funnelshift_r(lo, hi, sh) & mask;
+}
+
+template <int N, int R, int S, bool PK>
 __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   using namespace detail;
   using LM = LaneMap<R>;
@@ -83,7 +103,8 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   constexpr int LPN = LM::LPN;  // lanes per nonzero
   constexpr int GPW = 32 / LPN; // lane groups per warp
   constexpr int G = N - 1;      // gathered slots
-  constexpr int W = RecWords<N>::W;
+  constexpr int W = PK ? 4 : RecWords<N>::W;
+  static_assert(!PK || N >= 4, "packed records are for N >= 4");
   constexpr int RB = R * 4;     // bytes per factor row
   constexpr int R4 = R / 4;     // float4 per factor row
   constexpr int U = (VEC == 8) ? 2 : kFragUnroll;  // batch (register budget: 64 at 1024 thr)
@@ -196,10 +217,12 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     uint32_t before = 0xFFFFFFFFu;
     if constexpr (S == 0) {
       if (p.owner && gs < ge) {
-        before = (gs > 0) ? __ldg(p.rec + (size_t)(gs - 1) * W) : 0xFFFFFFFFu;
-        const uint32_t first_g = __ldg(p.rec + (size_t)gs * W);
+        const uint32_t om = p.out_mask;
+        before = (gs > 0) ? (__ldg(p.rec + (size_t)(gs - 1) * W) & om) : 0xFFFFFFFFu;
+        const uint32_t first_g = __ldg(p.rec + (size_t)gs * W) & om;
         first_shared = (gs > 0) && before == first_g;
-        last_shared = (ge < p.nnz) && __ldg(p.rec + (size_t)ge * W) == __ldg(p.rec + (size_t)(ge - 1) * W);
+        last_shared = (ge < p.nnz) &&
+                      (__ldg(p.rec + (size_t)ge * W) & om) == (__ldg(p.rec + (size_t)(ge - 1) * W) & om);
       }
     }
     if constexpr (S > 0) {
@@ -220,11 +243,17 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           const float4 y = base[row + c0 + 1 - par];
           r.a = par ? y : x;
           r.b = par ? x : y;
+        } else if (p.texmask & (1u << q)) {
+          const cudaTextureObject_t tx = (cudaTextureObject_t)p.tex[q];
+          r.a = tex1Dfetch<float4>(tx, (int)(row + c0));
+          r.b = tex1Dfetch<float4>(tx, (int)(row + c0 + 1));
         } else {
           ldg256_na(base + row + c0, r.a, r.b);
         }
       } else {
-        r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
+        if (q < S) r.a = base[row + c0];
+        else if (p.texmask & (1u << q)) r.a = tex1Dfetch<float4>((cudaTextureObject_t)p.tex[q], (int)(row + c0));
+        else r.a = ldg128(base + row + c0);
       }
       return r;
     };
@@ -273,7 +302,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
       const uint32_t n = (s0 < ge) ? min(K, ge - s0) : 0u;
       if (n > 0) {
         if (t == 0) {  // open the sub-range's first run
-          cur = reg[0];
+          cur = reg[0] & p.out_mask;
           if constexpr (S == 0) {
             if (p.owner && !first_shared && gs > 0) zero_rows(before, cur);  // gap rows are ours
           }
@@ -288,10 +317,17 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
             const uint4 w1 = lds128(rp + 4);
             w[4] = w1.x; w[5] = w1.y; w[6] = w1.z; w[7] = w1.w;
           }
-          i = w[0];
+          if constexpr (PK) {
+            i = w[0] & p.out_mask;  // i_n at bit 0
 #pragma unroll
-          for (int q = 0; q < G; ++q) g[q] = w[1 + q];
-          v = __uint_as_float(w[N]);
+            for (int q = 0; q < G; ++q) g[q] = pk_field(w[0], w[1], w[2], p.boff[1 + q], p.bmask[1 + q]);
+            v = __uint_as_float(w[3]);
+          } else {
+            i = w[0];
+#pragma unroll
+            for (int q = 0; q < G; ++q) g[q] = w[1 + q];
+            v = __uint_as_float(w[N]);
+          }
         };
         uint32_t k = 0;
         for (; k + U <= n; k += U) {
@@ -351,7 +387,8 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
 template <int R>
 __global__ void boundary_zero3_kernel(const uint32_t* __restrict__ chunk_begin, uint32_t num_chunks,
                                       uint32_t nnz, uint32_t ctas, uint32_t groups_per_cta,
-                                      const uint32_t* __restrict__ rec, uint32_t W, float* __restrict__ out) {
+                                      const uint32_t* __restrict__ rec, uint32_t W, uint32_t om,
+                                      float* __restrict__ out) {
   const uint64_t total = (uint64_t)ctas * groups_per_cta;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
@@ -363,8 +400,8 @@ __global__ void boundary_zero3_kernel(const uint32_t* __restrict__ chunk_begin, 
     const uint32_t pos = frag3_group_begin(a, b - a, gam, groups_per_cta);
     const uint32_t end = frag3_group_begin(a, b - a, gam + 1, groups_per_cta);
     if (pos >= end || pos == 0) continue;
-    const uint32_t r = rec[(size_t)pos * W];
-    if (rec[(size_t)(pos - 1) * W] != r) continue;
+    const uint32_t r = rec[(size_t)pos * W] & om;
+    if ((rec[(size_t)(pos - 1) * W] & om) != r) continue;
     float4* y = reinterpret_cast<float4*>(out + (size_t)r * R);
 #pragma unroll
     for (int q = 0; q < R / 4; ++q) y[q] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -412,14 +449,14 @@ void boundary_zero3_r64(const Frag3Params& fp, uint32_t ctas, uint32_t groups, f
 
 template <int N, int R, int S>
 void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s) {
-  auto k = frag3_kernel<N, R, S>;
+  auto k = fp.W == 4 && N >= 4 ? frag3_kernel<N, R, S, (N >= 4)> : frag3_kernel<N, R, S, false>;
   SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   k<<<grid, threads, smem, s>>>(fp);
 }
 
 template <int N, int R, int S>
 int frag3_occ_one(int threads, size_t smem) {
-  auto k = frag3_kernel<N, R, S>;
+  auto k = frag3_kernel<N, R, S, false>;
   SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int nb = 0;
   SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));
@@ -441,7 +478,7 @@ int frag3_occ_one(int threads, size_t smem) {
     const uint64_t total = (uint64_t)ctas * groups;                                                      \
     const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((total + 255) / 256, 148 * 16));     \
     boundary_zero3_kernel<R><<<grid, 256, 0, s>>>(fp.chunk_begin, fp.num_chunks, fp.nnz, ctas, groups,  \
-                                                  fp.rec, fp.W, out);                   \
+                                                  fp.rec, fp.W, fp.out_mask, out);      \
   }
 
 }  // namespace sf

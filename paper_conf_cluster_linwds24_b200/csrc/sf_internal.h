@@ -75,6 +75,9 @@ struct Plan {
   DevBuf chunk_begin;   // uint32[num_chunks + 1]
   DevBuf chunk_tile;    // uint64[num_chunks]
   mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
+  bool rec_packed = false;               // frag3 PK records (N >= 4, indices bit-packed)
+  uint32_t rec_boff[SF_MAX_MODES] = {};  // PK: bit offset of field f (slot order)
+  uint32_t rec_bmask[SF_MAX_MODES] = {}; // PK: width mask of field f
   size_t device_bytes() const;
 };
 
@@ -94,8 +97,34 @@ struct Tensor {
   sf_features_t features[SF_MAX_MODES] = {};
   std::map<std::pair<int, int>, Plan*> plans;  // (mode, rank) -> plan
   cudaStream_t stream = nullptr;               // internal stream for planning
+  // texture objects over caller factors (frag3 TEX gathers), keyed by (pointer, bytes)
+  struct TexEntry {
+    const void* ptr;
+    size_t bytes;
+    unsigned long long obj;
+    uint64_t last_use;
+  };
+  mutable std::vector<TexEntry> tex_cache;
+  mutable uint64_t tex_clock = 0;
   ~Tensor();
 };
+
+// Packed 16-byte records for N >= 4 (frag3 PK): all N indices fit 96 bits.
+inline int index_bits(uint64_t dim) {  // bits to hold 0 .. dim-1 (>= 1)
+  int b = 0;
+  for (uint64_t x = dim > 0 ? dim - 1 : 0; x; x >>= 1) ++b;
+  return b > 0 ? b : 1;
+}
+inline bool rec_packable(const Tensor& t) {
+  if (t.nmodes < 4) return false;
+  int b = 0;
+  for (int m = 0; m < t.nmodes; ++m) b += index_bits(t.dims[m]);
+  return b <= 96;
+}
+// Words per frag3 record for this tensor: 4 (N <= 3, or N >= 4 packed), else 8.
+inline int tensor_rec_words(const Tensor& t) {
+  return (t.nmodes + 1 <= 4 || rec_packable(t)) ? 4 : 8;
+}
 
 // Secondary sort key of mode n (reading R10): the gathered mode with the
 // smallest dimension (ties: the higher mode index) -- the (i_n, i_s) fibers with the most
@@ -116,6 +145,7 @@ struct RecWords {
 };
 
 __host__ __device__ inline int rec_words_for(int N) { return (N + 1 <= 4) ? 4 : 8; }
+
 
 // Region stride (words) of one group's K records: W*K + pad with stride/4 odd, so the
 // GPW groups' record k (read in lockstep) fall into distinct 16-byte bank quads.

@@ -280,6 +280,32 @@ static int frag3_occ(int N, int R, int S, int threads, size_t smem) {
   }
 }
 
+// Texture object over a caller factor (cached per tensor by pointer and size; LRU of 16).
+static unsigned long long factor_texture(const Tensor& t, const float* ptr, size_t bytes) {
+  for (auto& e : t.tex_cache)
+    if (e.ptr == ptr && e.bytes == bytes) {
+      e.last_use = ++t.tex_clock;
+      return e.obj;
+    }
+  if (t.tex_cache.size() >= 16) {
+    auto it = std::min_element(t.tex_cache.begin(), t.tex_cache.end(),
+                               [](const Tensor::TexEntry& a, const Tensor::TexEntry& b) { return a.last_use < b.last_use; });
+    cudaDestroyTextureObject((cudaTextureObject_t)it->obj);
+    t.tex_cache.erase(it);
+  }
+  cudaResourceDesc rd{};
+  rd.resType = cudaResourceTypeLinear;
+  rd.res.linear.devPtr = const_cast<float*>(ptr);
+  rd.res.linear.desc = cudaCreateChannelDesc<float4>();
+  rd.res.linear.sizeInBytes = bytes;
+  cudaTextureDesc td{};
+  td.readMode = cudaReadModeElementType;
+  cudaTextureObject_t obj = 0;
+  SF_CUDA(cudaCreateTextureObject(&obj, &rd, &td, nullptr));
+  t.tex_cache.push_back({ptr, bytes, (unsigned long long)obj, ++t.tex_clock});
+  return (unsigned long long)obj;
+}
+
 // frag3 path (record plans): A5 owner pre-pass on the frag3 group partition, then the kernel.
 static void launch_frag3(const Tensor& t, const Plan& p, const float* const* factors, float* out,
                          cudaStream_t s, bool owner) {
@@ -298,8 +324,25 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   const uint32_t gpw = (uint32_t)frag_groups_per_warp(R);
   fp.K = frag3_K((uint32_t)p.launch.chunk_nnz, gpw);
   fp.W = (uint32_t)p.rec_words;
+  fp.out_mask = p.rec_packed ? p.rec_bmask[0] : 0xFFFFFFFFu;
+  for (int f = 0; f < SF_MAX_MODES; ++f) {
+    fp.boff[f] = p.rec_boff[f];
+    fp.bmask[f] = p.rec_bmask[f];
+  }
   fp.owner = owner ? 1u : 0u;
   const int S = frag_slot_order(N, n, p.launch.staged_mask, fp.slot_mode);
+  // SF_LAUNCH_TEX: the last global slot gathers through the texture pipeline
+  bool tex = (p.launch.flags & SF_LAUNCH_TEX) != 0;
+  if (const char* e = std::getenv("SF_TEX")) tex = std::atoi(e) != 0;  // A/B override
+  fp.texmask = 0;
+  if (tex && S < N - 1) {
+    const int q = N - 2, m = fp.slot_mode[q];
+    const size_t texels = (size_t)t.dims[m] * (size_t)R / 4;
+    if (texels <= (1ull << 28) && R % 4 == 0) {
+      fp.tex[q] = factor_texture(t, factors[m], texels * 16);
+      fp.texmask = 1u << q;
+    }
+  }
   uint32_t off = 0;
   for (int q = 0; q < S; ++q) {
     const int m = fp.slot_mode[q];

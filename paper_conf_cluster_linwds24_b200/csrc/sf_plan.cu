@@ -281,8 +281,12 @@ __global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32
 
 // frag3 records: kernel-order record k = [raw field fmap[0], ..., fmap[WK-1]] of the raw
 // AoS record perm[k] (fmap < 0: zero padding).  Slot order: i_n, gathered slots, value.
+// Packed (nfields > 0): fields f < nfields (raw word fmap[f]) are OR-ed in at bit boff[f]
+// of words 0..2, and word 3 = raw word fmap[nfields] (the value).
 struct RecParams {
   int fmap[8];
+  int nfields;
+  uint32_t boff[8];
 };
 
 template <int WR, int WK>
@@ -304,6 +308,21 @@ __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32
 #pragma unroll
       for (int q = 0; q < WR; ++q) x = (rp.fmap[d] == q) ? w[q] : x;
       o[d] = x;
+    }
+    if (WK == 8 && rp.nfields > 0) {  // packed 16-byte record
+      uint32_t o0 = 0, o1 = 0, o2 = 0;
+#pragma unroll
+      for (int f = 0; f < 8; ++f) {
+        if (f >= rp.nfields) break;
+        const uint32_t x = o[f < WK ? f : 0], off = rp.boff[f], wi = off >> 5, sh = off & 31u;
+        const uint32_t lo = x << sh, hi = sh ? (x >> (32u - sh)) : 0u;
+        if (wi == 0) { o0 |= lo; o1 |= hi; } else if (wi == 1) { o1 |= lo; o2 |= hi; } else { o2 |= lo; }
+      }
+      uint32_t val = 0;
+#pragma unroll
+      for (int f = 0; f < WK; ++f) val = (f == rp.nfields) ? o[f] : val;
+      reinterpret_cast<uint4*>(rec)[k] = make_uint4(o0, o1, o2, val);
+      continue;
     }
     uint4* dst = reinterpret_cast<uint4*>(rec + k * WK);
 #pragma unroll
@@ -457,8 +476,10 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   p.rec_words = 0;
   if (use_rec) {
     // frag3 records in slot order [i_n, staged slots, other gathered slots, value, 0...]
-    const int WK = rec_words_for(N);
+    const bool packed = N >= 4 && rec_packable(t);
+    const int WK = packed ? 4 : rec_words_for(N);
     p.rec_words = WK;
+    p.rec_packed = packed;
     p.rec.alloc(nl * WK * 4 + kPadBytes);
     SF_CUDA(cudaMemsetAsync(p.rec.as<uint32_t>() + nl * WK, 0, kPadBytes, t.stream));
     RecParams rp{};
@@ -468,12 +489,26 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     rp.fmap[0] = mode;
     for (int q = 0; q < N - 1; ++q) rp.fmap[1 + q] = slot_mode[q];
     rp.fmap[N] = N;  // value word of the raw record
+    rp.nfields = 0;
+    if (packed) {  // fields in slot order, i_n at bit 0
+      uint32_t off = 0;
+      for (int f = 0; f < N; ++f) {
+        const int b = index_bits(t.dims[rp.fmap[f]]);
+        rp.boff[f] = off;
+        p.rec_boff[f] = off;
+        p.rec_bmask[f] = (b >= 32) ? 0xFFFFFFFFu : ((1u << b) - 1u);
+        off += (uint32_t)b;
+      }
+      rp.nfields = N;
+    }
     if (nl) {
       const uint32_t* aos = t.aos.as<uint32_t>();
       const uint32_t* pm = perm.as<uint32_t>();
       uint32_t* rec = p.rec.as<uint32_t>();
       if (WR == 4 && WK == 4) gather_rec_kernel<4, 4><<<grid_for(nl), 256, 0, t.stream>>>(aos, pm, nl, rp, rec);
       else if (WR == 8 && WK == 8) gather_rec_kernel<8, 8><<<grid_for(nl), 256, 0, t.stream>>>(aos, pm, nl, rp, rec);
+      else if (WR == 8 && WK == 4 && packed)
+        gather_rec_kernel<8, 8><<<grid_for(nl), 256, 0, t.stream>>>(aos, pm, nl, rp, rec);
       else throw StatusError{SF_ERR_UNSUPPORTED, "frag3 records: unsupported record width"};
       count_launch();
       SF_CUDA(cudaGetLastError());

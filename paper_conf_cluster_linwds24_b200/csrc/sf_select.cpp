@@ -30,7 +30,7 @@ size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l
   if (frag_impl() == 3) {  // frag3: per warp 2 stages x GPW regions of K records
     const uint32_t gpw = (uint32_t)frag_groups_per_warp(rank);
     const uint32_t K = frag3_K((uint32_t)l.chunk_nnz, gpw);
-    b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)rec_words_for(t.nmodes)) * 4;
+    b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)tensor_rec_words(t)) * 4;
   } else {
     b += nwarps * kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
   }
