@@ -16,7 +16,7 @@ Contract (one JSON line on rank 0):
 * e2e: the same metric through the public C ABI from PINNED HOST buffers:
   sf_tensor_create (segmented H2D + validate) + factor H2D + sf_plan (all modes)
   + sf_mttkrp (all modes) + D2H of every Y, every step.
-* roofline: dominant kernel = frag_kernel; algorithmic bytes per launch =
+* roofline: dominant kernel = frag3_kernel; algorithmic bytes per launch =
   4(N+1)*nnz + 4R*sum_m I_m, over its event-timed duration.
 * cpu_baseline: the oracle (oracle/oracle.c, fp64, 1 thread) on a bounded sample.
 """
@@ -392,7 +392,7 @@ def main():
             "config": workload_config(cfg, world),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
-                         "kernel": "frag_kernel", "peak_src": peaks["src"],
+                         "kernel": "frag3_kernel", "peak_src": peaks["src"],
                          "bytes_per_launch": bytes_launch, "launch_ms": mean_launch_ms},
             "cpu_baseline": cpu,
             "e2e": e2e,

@@ -73,9 +73,7 @@ typedef struct {
   uint32_t flags;        /* FRAG: SF_LAUNCH_* bits below */
 } sf_launch_t;
 #define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
-#define SF_LAUNCH_NO_CARRY 8u /* FRAG: flush each stretch's last run (no cross-stretch carry) */
-#define SF_LAUNCH_TEX 64u /* FRAG: the last globally gathered factor is read through the texture
-                              pipeline (a second data path into registers; factors <= 2^28 float4) */
+#define SF_LAUNCH_NO_CARRY 8u /* legacy (round-1 stretch kernel); ignored: frag3 flushes once per run */
 #define SF_LAUNCH_DETERMINISTIC 32u /* FRAG: A7 two-pass carry combine instead of atomics; forces an
                                        unstaged owner-store plan; Y is bitwise reproducible run to run */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation

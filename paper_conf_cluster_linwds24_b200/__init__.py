@@ -24,7 +24,7 @@ SF_MAX_MODES = 8
 SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
 LAUNCH_L1_NO_ALLOCATE, LAUNCH_NO_OWNER_STORES, LAUNCH_NO_CARRY = 2, 4, 8
-LAUNCH_DETERMINISTIC, LAUNCH_TEX = 32, 64
+LAUNCH_DETERMINISTIC = 32
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",

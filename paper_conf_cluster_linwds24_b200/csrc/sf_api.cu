@@ -97,8 +97,6 @@ size_t Plan::device_bytes() const {
 }
 
 Tensor::~Tensor() {
-  for (auto& e : tex_cache) cudaDestroyTextureObject((cudaTextureObject_t)e.obj);
-  tex_cache.clear();
   for (auto& kv : plans) delete kv.second;
   plans.clear();
   if (stream) cudaStreamDestroy(stream);

@@ -2,7 +2,7 @@
 //
 // Y(i_n(e), :) += v_e * prod_{m != n} A_m(i_m(e), :)   (Eq. (4))
 //
-// Same method as frag_kernel (sf_frag.cuh), with two changes that cut L1TEX work per
+// Same method as the round-1 SoA frag_kernel (chunks of 128 nonzeros cut into 8 stretches), with two changes that cut L1TEX work per
 // nonzero -- the resource that binds on sm_100a when the factors are L2-resident
 // (profiles/r01_ncu_full_nell2.json: l1tex 92 %, DRAM 16 %):
 //   1. Records.  The plan stores each nonzero as one W-word record in *slot order*
@@ -62,11 +62,6 @@ struct Frag3Params {
   uint32_t boff[SF_MAX_MODES];        // PK: bit offset of field f (slot order, f = 0 is i_n)
   uint32_t bmask[SF_MAX_MODES];       // PK: (1 << width) - 1 of field f
   uint32_t out_mask;                  // mask applied to word 0 to read i_n (PK: bmask[0])
-  // TEX gathers: global slots q with bit q of texmask read their factor rows through the
-  // texture pipeline (tex1Dfetch<float4> on tex[q]) instead of LDG -- a second data path
-  // into registers next to the LSU one, which binds with L2-resident factors.
-  uint32_t texmask;
-  unsigned long long tex[SF_MAX_MODES];
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
   // A7 deterministic option (owner mode only): shared runs go to per-group carry slots
   // (head = 2*gid, tail = 2*gid+1, gid = blockIdx.x * groups + group) instead of atomics;
@@ -243,17 +238,11 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           const float4 y = base[row + c0 + 1 - par];
           r.a = par ? y : x;
           r.b = par ? x : y;
-        } else if (p.texmask & (1u << q)) {
-          const cudaTextureObject_t tx = (cudaTextureObject_t)p.tex[q];
-          r.a = tex1Dfetch<float4>(tx, (int)(row + c0));
-          r.b = tex1Dfetch<float4>(tx, (int)(row + c0 + 1));
         } else {
           ldg256_na(base + row + c0, r.a, r.b);
         }
       } else {
-        if (q < S) r.a = base[row + c0];
-        else if (p.texmask & (1u << q)) r.a = tex1Dfetch<float4>((cudaTextureObject_t)p.tex[q], (int)(row + c0));
-        else r.a = ldg128(base + row + c0);
+        r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
       }
       return r;
     };

@@ -97,15 +97,6 @@ struct Tensor {
   sf_features_t features[SF_MAX_MODES] = {};
   std::map<std::pair<int, int>, Plan*> plans;  // (mode, rank) -> plan
   cudaStream_t stream = nullptr;               // internal stream for planning
-  // texture objects over caller factors (frag3 TEX gathers), keyed by (pointer, bytes)
-  struct TexEntry {
-    const void* ptr;
-    size_t bytes;
-    unsigned long long obj;
-    uint64_t last_use;
-  };
-  mutable std::vector<TexEntry> tex_cache;
-  mutable uint64_t tex_clock = 0;
   ~Tensor();
 };
 
@@ -190,11 +181,7 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
 void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* const* inds,
                 const float* vals, const float* const* factors, int rank, int mode, float* out,
                 cudaStream_t s);
-int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem);
 bool frag_supported(int nmodes, int rank);
-// Fragment-kernel implementation: 3 = record-packed group-contiguous frag3_kernel (default),
-// 2 = SoA chunk-stretch frag_kernel (env SF_FRAG_IMPL=2, kept for A/B measurements).
-int frag_impl();
 // gathered slot order of a plan: staged modes ascending, then the other gathered modes
 int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode);
 void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s);

@@ -12,24 +12,19 @@
 //
 // coo_kernel  (SF_KERNEL_COO): raw input order, one vector atomic
 //   (red.global.add.v4.f32) per nonzero per group.  Baseline + streamed path.
-// frag_kernel (SF_KERNEL_FRAG): persistent CTAs walk chunks of the planned order
-//   (tile, i_n, i_s).  Each chunk's N+1 SoA fields are staged into shared memory by
-//   1-D TMA bulk copies (cp.async.bulk + mbarrier, double buffered).  Factors of
-//   "staged" modes are copied block-wise into shared memory once per tile (the
-//   paper's "times_mat in shared memory") and gathered from there;
-//   other modes are gathered from global memory (L2).  Each lane group walks a
-//   contiguous stretch of the chunk, accumulating in registers while i_n is
-//   unchanged (segmented reduction over sorted runs) and flushing one vector
-//   atomic per run edge -- global atomics fire only at run / fragment boundaries
-//   (north_star; "requirement for atomic operations").
+// frag3_kernel (SF_KERNEL_FRAG, sf_frag3.cuh): persistent CTAs walk the planned order
+//   (tile, i_n, i_s) of packed records; each lane group owns a contiguous sub-range,
+//   stages its records into shared memory by 1-D TMA bulk copies (cp.async.bulk +
+//   mbarrier, double buffered), gathers "staged" factor blocks from shared memory (the
+//   paper's "times_mat in shared memory") and the others from L2, and
+//   accumulates in registers while i_n is unchanged, flushing once per run -- global
+//   atomics fire only at run / sub-range boundaries (north_star).
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdio>
 
-#include "sf_frag.cuh"
 #include "sf_frag3.cuh"
-#include <cstdlib>
 #include "sf_internal.h"
 
 namespace sf {
@@ -230,37 +225,6 @@ bool frag_supported(int nmodes, int rank) {
   return nmodes >= 2 && nmodes <= 5 && (rank == 16 || rank == 32 || rank == 64);
 }
 
-static int frag_occ(int N, int R, int S, int threads, size_t smem) {
-  switch (R) {
-    case 16: return frag_occ_r16(N, S, threads, smem);
-    case 32: return frag_occ_r32(N, S, threads, smem);
-    case 64: return frag_occ_r64(N, S, threads, smem);
-    default: return 0;
-  }
-}
-
-int frag_max_ctas_per_sm(int nmodes, int rank, int threads, size_t smem) {
-  return frag_occ(nmodes, rank, 0, threads, smem);
-}
-
-static void frag_launch(int N, int R, int S, const FragParams& fp, int grid, int threads, size_t smem,
-                        cudaStream_t s) {
-  switch (R) {
-    case 16: return frag_launch_r16(N, S, fp, grid, threads, smem, s);
-    case 32: return frag_launch_r32(N, S, fp, grid, threads, smem, s);
-    case 64: return frag_launch_r64(N, S, fp, grid, threads, smem, s);
-    default: throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: unsupported rank"};
-  }
-}
-
-int frag_impl() {
-  static const int impl = [] {
-    const char* e = std::getenv("SF_FRAG_IMPL");
-    return (e && std::atoi(e) == 2) ? 2 : 3;
-  }();
-  return impl;
-}
-
 int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode) {
   int q = 0;
   for (int m = 0; m < nmodes; ++m)
@@ -278,32 +242,6 @@ static int frag3_occ(int N, int R, int S, int threads, size_t smem) {
     case 64: return frag3_occ_r64(N, S, threads, smem);
     default: return 0;
   }
-}
-
-// Texture object over a caller factor (cached per tensor by pointer and size; LRU of 16).
-static unsigned long long factor_texture(const Tensor& t, const float* ptr, size_t bytes) {
-  for (auto& e : t.tex_cache)
-    if (e.ptr == ptr && e.bytes == bytes) {
-      e.last_use = ++t.tex_clock;
-      return e.obj;
-    }
-  if (t.tex_cache.size() >= 16) {
-    auto it = std::min_element(t.tex_cache.begin(), t.tex_cache.end(),
-                               [](const Tensor::TexEntry& a, const Tensor::TexEntry& b) { return a.last_use < b.last_use; });
-    cudaDestroyTextureObject((cudaTextureObject_t)it->obj);
-    t.tex_cache.erase(it);
-  }
-  cudaResourceDesc rd{};
-  rd.resType = cudaResourceTypeLinear;
-  rd.res.linear.devPtr = const_cast<float*>(ptr);
-  rd.res.linear.desc = cudaCreateChannelDesc<float4>();
-  rd.res.linear.sizeInBytes = bytes;
-  cudaTextureDesc td{};
-  td.readMode = cudaReadModeElementType;
-  cudaTextureObject_t obj = 0;
-  SF_CUDA(cudaCreateTextureObject(&obj, &rd, &td, nullptr));
-  t.tex_cache.push_back({ptr, bytes, (unsigned long long)obj, ++t.tex_clock});
-  return (unsigned long long)obj;
 }
 
 // frag3 path (record plans): A5 owner pre-pass on the frag3 group partition, then the kernel.
@@ -331,18 +269,6 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   }
   fp.owner = owner ? 1u : 0u;
   const int S = frag_slot_order(N, n, p.launch.staged_mask, fp.slot_mode);
-  // SF_LAUNCH_TEX: the last global slot gathers through the texture pipeline
-  bool tex = (p.launch.flags & SF_LAUNCH_TEX) != 0;
-  if (const char* e = std::getenv("SF_TEX")) tex = std::atoi(e) != 0;  // A/B override
-  fp.texmask = 0;
-  if (tex && S < N - 1) {
-    const int q = N - 2, m = fp.slot_mode[q];
-    const size_t texels = (size_t)t.dims[m] * (size_t)R / 4;
-    if (texels <= (1ull << 28) && R % 4 == 0) {
-      fp.tex[q] = factor_texture(t, factors[m], texels * 16);
-      fp.texmask = 1u << q;
-    }
-  }
   uint32_t off = 0;
   for (int q = 0; q < S; ++q) {
     const int m = fp.slot_mode[q];
@@ -403,90 +329,25 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
 void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
                    cudaStream_t s) {
   const int N = t.nmodes, R = p.rank, n = p.mode;
-  const bool frag = p.launch.kernel == SF_KERNEL_FRAG && frag_supported(N, R);
+  const bool frag = p.launch.kernel == SF_KERNEL_FRAG && frag_supported(N, R) && p.rec_words;
   // A5: unstaged fragment plans run in owner mode (whole runs stored, gaps zeroed by
-  // their owner, only run-crossing rows pre-zeroed); everything else zeroes Y and adds.
+  // their owner, only run-crossing rows pre-zeroed by launch_frag3); everything else
+  // zeroes Y and adds.
   const bool owner = frag && p.launch.staged_mask == 0 && p.nnz_local > 0 &&
                      !(p.launch.flags & SF_LAUNCH_NO_OWNER_STORES);
   const size_t row_bytes = sizeof(float) * (size_t)R;
   if (!owner) {
     SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * t.dims[n], s));
-  } else if (p.rec_words) {  // frag3: rows outside the shard; the pre-pass runs in launch_frag3
+  } else {  // rows outside this shard's row range
     if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
     if (p.row_end < t.dims[n])
       SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (t.dims[n] - p.row_end), s));
-  } else {
-    if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
-    if (p.row_end < t.dims[n])
-      SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (t.dims[n] - p.row_end), s));
-    const uint32_t* cb = p.chunk_begin.as<uint32_t>();
-    const uint32_t* rows = p.ind[n].as<uint32_t>();
-    switch (R) {
-      case 16: boundary_zero_r16(cb, (uint32_t)p.num_chunks, rows, out, s); break;
-      case 32: boundary_zero_r32(cb, (uint32_t)p.num_chunks, rows, out, s); break;
-      default: boundary_zero_r64(cb, (uint32_t)p.num_chunks, rows, out, s); break;
-    }
-    count_launch();
-    SF_CUDA(cudaGetLastError());
   }
   if (p.nnz_local == 0) return;
-  if (frag && p.rec_words) return launch_frag3(t, p, factors, out, s, owner);
-  if (!frag) {
-    uint32_t* ind[SF_MAX_MODES];
-    for (int m = 0; m < N; ++m) ind[m] = p.ind[m].as<uint32_t>();
-    launch_coo(N, t.dims, p.nnz_local, ind, p.val.as<float>(), factors, R, n, out, s);
-    return;
-  }
-  FragParams fp{};
-  for (int m = 0; m < N; ++m) {
-    fp.ind[m] = p.ind[m].as<uint32_t>();
-    fp.fac[m] = factors[m];
-    fp.dims[m] = (uint32_t)t.dims[m];
-  }
-  fp.val = p.val.as<float>();
-  fp.out = out;
-  fp.chunk_begin = p.chunk_begin.as<uint32_t>();
-  fp.chunk_tile = p.chunk_tile.as<uint64_t>();
-  fp.num_chunks = (uint32_t)p.num_chunks;
-  fp.nnz = (uint32_t)p.nnz_local;
-  fp.mode = n;
-  fp.stage_words = (uint32_t)p.launch.chunk_nnz + 8;
-  fp.flags = p.launch.flags;
-  fp.owner = owner ? 1u : 0u;
-  fp.row_end = (uint32_t)p.row_end;
-  // slots: staged modes first (ascending mode id = tile-id fold order), then the rest
-  int S = 0, q = 0;
-  uint32_t off = 0;
-  for (int m = 0; m < N; ++m)
-    if (m != n && (p.launch.staged_mask & (1u << m))) {
-      fp.slot_mode[q] = m;
-      fp.block_rows[q] = p.launch.block_rows[m];
-      fp.ntiles[q] = (uint32_t)((t.dims[m] + fp.block_rows[q] - 1) / fp.block_rows[q]);
-      fp.fac_off[q] = off;
-      off += fp.block_rows[q] * (uint32_t)R;
-      ++q;
-      ++S;
-    }
-  for (int m = 0; m < N; ++m)
-    if (m != n && !(p.launch.staged_mask & (1u << m))) fp.slot_mode[q++] = m;
-
-  const size_t smem = frag_smem_bytes(t, n, R, p.launch);
-  const int threads = p.launch.block_threads;
-  int per_sm = p.launch.ctas_per_sm;
-  const int occ = frag_occ(N, R, S, threads, smem);
-  if (occ <= 0) throw StatusError{SF_ERR_UNSUPPORTED, "frag kernel: launch does not fit an SM"};
-  if (per_sm <= 0 || per_sm > occ) per_sm = occ;
-  int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
-  grid = std::max(grid, 1);
-  frag_launch(N, R, S, fp, grid, threads, smem, s);
-  count_launch();
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) {
-    char msg[256];
-    snprintf(msg, sizeof msg, "frag_kernel<%d,%d> launch grid=%d threads=%d smem=%zu occ=%d: %s", N, R, grid,
-             threads, smem, occ, cudaGetErrorString(e));
-    throw StatusError{SF_ERR_CUDA, msg};
-  }
+  if (frag) return launch_frag3(t, p, factors, out, s, owner);
+  uint32_t* ind[SF_MAX_MODES];
+  for (int m = 0; m < N; ++m) ind[m] = p.ind[m].as<uint32_t>();
+  launch_coo(N, t.dims, p.nnz_local, ind, p.val.as<float>(), factors, R, n, out, s);
 }
 
 }  // namespace sf

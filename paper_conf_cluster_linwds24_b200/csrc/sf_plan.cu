@@ -472,7 +472,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     SF_CUDA(cudaGetLastError());
     t.aos_words = WR;
   }
-  const bool use_rec = launch.kernel == SF_KERNEL_FRAG && frag_supported(N, rank) && frag_impl() == 3;
+  const bool use_rec = launch.kernel == SF_KERNEL_FRAG && frag_supported(N, rank);
   p.rec_words = 0;
   if (use_rec) {
     // frag3 records in slot order [i_n, staged slots, other gathered slots, value, 0...]

@@ -19,21 +19,19 @@
 
 namespace sf {
 
-static constexpr int kStagesHost = 2;  // must match frag_kernel's kStages
+static constexpr int kStagesHost = 2;  // must match kFragStages (sf_frag.cuh)
 
-// Shared memory of frag_kernel: mbarriers (2 per warp + 1), one double-buffered stage
-// ring of (N+1) x (C+8) words per warp (C = chunk_nnz, a per-warp chunk), factor blocks.
+// Shared memory of frag3_kernel: mbarriers (2 per warp + 1), per warp a double-buffered
+// stage of GPW regions of K = C / GPW records (C = chunk_nnz, nonzeros per warp per
+// stage), and the staged factor blocks.
 size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l) {
   (void)mode;
   const size_t nwarps = (size_t)std::max(1, l.block_threads / 32);
   size_t b = ((2 * nwarps + 1) * 8 + 127) & ~(size_t)127;
-  if (frag_impl() == 3) {  // frag3: per warp 2 stages x GPW regions of K records
-    const uint32_t gpw = (uint32_t)frag_groups_per_warp(rank);
-    const uint32_t K = frag3_K((uint32_t)l.chunk_nnz, gpw);
-    b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)tensor_rec_words(t)) * 4;
-  } else {
-    b += nwarps * kStagesHost * (t.nmodes + 1) * ((size_t)l.chunk_nnz + 8) * 4;
-  }
+  // frag3: per warp 2 stages x GPW regions of K records
+  const uint32_t gpw = (uint32_t)frag_groups_per_warp(rank);
+  const uint32_t K = frag3_K((uint32_t)l.chunk_nnz, gpw);
+  b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)tensor_rec_words(t)) * 4;
   for (int m = 0; m < t.nmodes; ++m)
     if (l.staged_mask & (1u << m)) b += (size_t)l.block_rows[m] * rank * 4;
   return b;
@@ -125,7 +123,6 @@ static sf_launch_t select_rules(const Tensor& t, const sf_features_t& f, int mod
     if (best >= 0) {
       l.staged_mask = 1u << best;
       l.block_rows[best] = kBlockRows;
-      l.flags |= SF_LAUNCH_NO_CARRY;
     }
   }
   normalize_launch(t, mode, rank, l);
@@ -197,7 +194,6 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out) {
     if (stage_mode >= 0) {
       l.staged_mask = 1u << stage_mode;
       l.block_rows[stage_mode] = rows;
-      l.flags |= SF_LAUNCH_NO_CARRY;  // tiled runs are short; the carry costs ~4 % there
     }
     normalize_launch(t, mode, rank, l);
     out[n++] = l;

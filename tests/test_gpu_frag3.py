@@ -109,20 +109,3 @@ def test_record_packing_boundaries(cuda_device, dims):
             Yo, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
             assert np.max(S) < 2 ** 24
             assert np.array_equal(Y[n].astype(np.float64), Yo), (dims, n, staged)
-
-
-@pytest.mark.parametrize("R", [16, 32, 64])
-@pytest.mark.parametrize("dims", [(100, 80, 60), (10, 12, 14, 16), (5, 6, 4, 3, 7)])
-def test_texture_gathers(cuda_device, R, dims):
-    """SF_LAUNCH_TEX: the last global slot read with tex1Dfetch -- same values as LDG."""
-    inds, vals = synth.gen_coo(dims, 3001, 71, zipf=(0.8,) * len(dims), val_kind="int")
-    facs = synth.gen_factors(dims, R, 72, "int")
-    for staged in (False, True):
-        def L(n):
-            st = {} if not staged else {min(m for m in range(len(dims)) if m != n): 5}
-            return sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged=st, flags=sf.LAUNCH_TEX)
-        Y, _ = G.run(dims, inds, vals, facs, R, launch=L)
-        for n in range(len(dims)):
-            Yo, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
-            assert np.max(S) < 2 ** 24
-            assert np.array_equal(Y[n].astype(np.float64), Yo), (n, staged)
