@@ -227,6 +227,18 @@ struct TileParams {
   int nmodes;
 };
 
+// Single staged mode == the secondary key s: the tile id is (key % I_s) / block_rows, read
+// from the (sequential) matricized keys instead of a random 4-byte gather of i_s.
+__global__ void tile_key_from_keys_kernel(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ pos,
+                                          uint64_t n, uint64_t Is, uint32_t block_rows,
+                                          uint64_t* __restrict__ tkey, uint32_t* __restrict__ tpos) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    tkey[k] = (keys[k] % Is) / block_rows;
+    tpos[k] = pos[k];
+  }
+}
+
 __global__ void tile_key_kernel(TileParams tp, const uint32_t* __restrict__ pos, uint64_t n,
                                 uint64_t* __restrict__ tkey, uint32_t* __restrict__ tpos) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -416,7 +428,8 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     p.row_begin = kb / t.dims[s];
     p.row_end = ke / t.dims[s] + 1;
   }
-  keys.release();
+  const bool staged_is_secondary = launch.kernel == SF_KERNEL_FRAG && launch.staged_mask == (1u << s);
+  if (!staged_is_secondary) keys.release();  // else kept for the tile keys
 
   // Kernel order (positions into the raw COO).
   const bool staged = (launch.kernel == SF_KERNEL_FRAG) && launch.staged_mask != 0;
@@ -436,11 +449,17 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       tp.staged_mask = launch.staged_mask;
       tp.nmodes = N;
       DevBuf k0(nl * 8 + 16), k1(nl * 8 + 16), p1(nl * 4 + kPadBytes);
-      tile_key_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tp, pos0.as<uint32_t>() + lo, nl, k0.as<uint64_t>(),
-                                                         perm.as<uint32_t>());
+      if (staged_is_secondary)
+        tile_key_from_keys_kernel<<<grid_for(nl), 256, 0, t.stream>>>(
+            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, t.dims[s], launch.block_rows[s],
+            k0.as<uint64_t>(), perm.as<uint32_t>());
+      else
+        tile_key_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tp, pos0.as<uint32_t>() + lo, nl, k0.as<uint64_t>(),
+                                                           perm.as<uint32_t>());
       count_launch();
       SF_CUDA(cudaGetLastError());
       pos0.release();
+      keys.release();
       const int end_bit = std::max(1, bitlen(total_tiles - 1));
       cub::DoubleBuffer<uint64_t> dk(k0.as<uint64_t>(), k1.as<uint64_t>());
       cub::DoubleBuffer<uint32_t> dv(perm.as<uint32_t>(), p1.as<uint32_t>());
