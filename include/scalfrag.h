@@ -76,6 +76,16 @@ typedef struct {
 #define SF_LAUNCH_NO_CARRY 8u /* legacy (round-1 stretch kernel); ignored: frag3 flushes once per run */
 #define SF_LAUNCH_DETERMINISTIC 32u /* FRAG: A7 two-pass carry combine instead of atomics; forces an
                                        unstaged owner-store plan; Y is bitwise reproducible run to run */
+#define SF_LAUNCH_L2_TILES 64u /* FRAG: the staged_mask modes are NOT copied into shared memory; they
+                                 only tile the order (tile = block of block_rows[m] rows, PAPER.md L34
+                                 "tensor blocks") and every CTA sweeps the tiles in the same order,
+                                 taking 1/grid of each, so the factor rows gathered at any moment
+                                 are one block that stays L2-resident (for factors >> L2).  Forces
+                                 memset + atomics (no owner stores); ignored with DETERMINISTIC. */
+#define SF_LAUNCH_COMPACT 128u /* FRAG, N = 3, non-owner plans: 8-byte records (gathered indices + run
+                                  delta, value; i_n per slot in a side array) where the fields fit
+                                  30 bits.  Halves the record stream, but measured 9 % slower on
+                                  nell-2 (+19 % issued instructions for the decode): opt-in. */
 #define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation
                                        (ld.global.nc.L1::no_allocate.v8.f32; measured faster) */
 

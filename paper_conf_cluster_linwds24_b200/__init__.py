@@ -25,6 +25,8 @@ SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
 LAUNCH_L1_NO_ALLOCATE, LAUNCH_NO_OWNER_STORES, LAUNCH_NO_CARRY = 2, 4, 8
 LAUNCH_DETERMINISTIC = 32
+LAUNCH_L2_TILES = 64
+LAUNCH_COMPACT = 128
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",

@@ -46,6 +46,7 @@ __device__ __forceinline__ uint32_t frag3_lower_chunk(const uint32_t* cb, uint32
 
 struct Frag3Params {
   const uint32_t* rec;                // kernel-order records (slot order), W words each
+  const uint32_t* rowid;              // CR records: i_n per kernel-order slot
   const float* fac[SF_MAX_MODES];     // by mode
   float* out;
   const uint32_t* chunk_begin;        // num_chunks + 1
@@ -63,6 +64,8 @@ struct Frag3Params {
   uint32_t bmask[SF_MAX_MODES];       // PK: (1 << width) - 1 of field f
   uint32_t out_mask;                  // mask applied to word 0 to read i_n (PK: bmask[0])
   uint32_t owner;                     // A5: unstaged plans store whole runs, zero gaps (no memset)
+  uint32_t l2tiles;                   // SF_LAUNCH_L2_TILES: every CTA takes 1/grid of every tile, in tile
+                                      // order (S == 0: the tiled modes are gathered from L2)
   // A7 deterministic option (owner mode only): shared runs go to per-group carry slots
   // (head = 2*gid, tail = 2*gid+1, gid = blockIdx.x * groups + group) instead of atomics;
   // frag3_combine_kernel then adds them per row in slot order.
@@ -90,7 +93,15 @@ __device__ __forceinline__ uint32_t pk_field(uint32_t w0, uint32_t w1, uint32_t 
   return __funnelshift_r(lo, hi, sh) & mask;
 }
 
-template <int N, int R, int S, bool PK>
+// Record formats (RF): kRecPlain [i_n, g_0 .. g_{N-2}, v, 0..] (W = 4 or 8); kRecPacked
+// (N >= 4: N bit fields in words 0..2, v in word 3); kRecCompact (non-owner N = 3 plans
+// whose gathered fields leave >= 2 of 32 bits: word 0 = fields (staged slots: the row inside
+// the tile's block) | the run delta d in the top bits (boff[0], mask bmask[0] = E):
+// d = 0 inside a run, i_n - i_n(prev) in [1, E) at a run start, E = "read p.rowid" (tile
+// starts, big jumps); word 1 = v.  A group reads p.rowid once per sub-range start.
+constexpr int kRecPlain = 0, kRecPacked = 1, kRecCompact = 2;
+
+template <int N, int R, int S, int RF>
 __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   using namespace detail;
   using LM = LaneMap<R>;
@@ -98,7 +109,9 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   constexpr int LPN = LM::LPN;  // lanes per nonzero
   constexpr int GPW = 32 / LPN; // lane groups per warp
   constexpr int G = N - 1;      // gathered slots
-  constexpr int W = PK ? 4 : RecWords<N>::W;
+  constexpr bool PK = RF == kRecPacked;
+  constexpr bool CR = RF == kRecCompact;
+  constexpr int W = CR ? 2 : (PK ? 4 : RecWords<N>::W);
   static_assert(!PK || N >= 4, "packed records are for N >= 4");
   constexpr int RB = R * 4;     // bytes per factor row
   constexpr int R4 = R / 4;     // float4 per factor row
@@ -116,7 +129,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   const bool leader = lane_in_group == 0;
 
   const uint32_t K = p.K;
-  const uint32_t RS = frag3_region_words(K, W);
+  const uint32_t RS = CR ? frag3_cr_region_words(K) : frag3_region_words(K, W);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);
   const uint32_t bar_bytes = ((2u * nwarps + 1u) * 8u + 127u) & ~127u;
   uint32_t* ring = reinterpret_cast<uint32_t*>(smem_raw + bar_bytes) + (size_t)warp * kFragStages * GPW * RS;
@@ -125,8 +138,12 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   uint64_t* fbar = bars + 2 * nwarps;
 
   const uint64_t grid = gridDim.x;
-  const uint32_t j0 = frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)blockIdx.x * p.nnz) / grid);
-  const uint32_t j1 = frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)(blockIdx.x + 1) * p.nnz) / grid);
+  // CTA range: nnz-balanced chunks [j0, j1) of the plan order, or (L2 tiles) every chunk,
+  // of which each tile segment contributes its blockIdx.x-th 1/grid share.
+  const bool l2t = (S == 0) && p.l2tiles;
+  const uint32_t j0 = l2t ? 0u : frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)blockIdx.x * p.nnz) / grid);
+  const uint32_t j1 = l2t ? p.num_chunks
+                          : frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)(blockIdx.x + 1) * p.nnz) / grid);
   if (j0 >= j1) return;
 
   if (lane == 0) {
@@ -152,6 +169,15 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   uint32_t seg = j0;
   while (seg < j1) {
     uint32_t seg_end = j1;
+    if (S == 0 && l2t) {  // this tile's chunks [seg, seg_end)
+      const uint64_t tile = __ldg(p.chunk_tile + seg);
+      uint32_t lo = seg + 1, hi = j1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (__ldg(p.chunk_tile + mid) == tile) lo = mid + 1; else hi = mid;
+      }
+      seg_end = lo;
+    }
     if constexpr (S > 0) {
       const uint64_t tile = __ldg(p.chunk_tile + seg);
       uint32_t lo = seg + 1, hi = j1;  // first chunk with a different (larger) tile
@@ -181,24 +207,37 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
         }
       }
 #pragma unroll
-      for (int q = 0; q < S; ++q)
-        sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (ptrdiff_t)row0[q] * R4;
+      for (int q = 0; q < S; ++q)  // CR records carry the row inside the block
+        sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (CR ? (ptrdiff_t)0 : (ptrdiff_t)row0[q] * R4);
     }
     // this group's sub-range [gs, ge) of the tile segment [a, b)
-    const uint32_t a = __ldg(p.chunk_begin + seg), b = __ldg(p.chunk_begin + seg_end);
+    uint32_t a = __ldg(p.chunk_begin + seg), b = __ldg(p.chunk_begin + seg_end);
+    if (l2t) {  // this CTA's share of the tile
+      const uint32_t len = b - a;
+      b = a + (uint32_t)(((uint64_t)(blockIdx.x + 1) * len) / grid);
+      a = a + (uint32_t)(((uint64_t)blockIdx.x * len) / grid);
+    }
     const uint32_t gs = frag3_group_begin(a, b - a, gam, Gam);
     const uint32_t ge = frag3_group_begin(a, b - a, gam + 1, Gam);
     const uint32_t T = (__reduce_max_sync(0xFFFFFFFFu, ge - gs) + K - 1) / K;  // stages of this warp
     uint32_t* const my_region0 = ring + (size_t)group * RS;
+    // CR: stages are copied from the 16-byte-aligned record at or before s0; every stage
+    // start s0 = gs + t*K has the parity of gs (K is even), so record k sits at k + o
+    const uint32_t o = CR ? (gs & 1u) : 0u;
 
     // stage t of this warp into ring slot st: every group leader copies its own records
     auto issue = [&](uint32_t t, int st) {
       if (leader) {
         const uint32_t s0 = gs + t * K;
         if (s0 < ge) {
-          const uint32_t bytes = min(K, ge - s0) * (uint32_t)(W * 4);
+          uint32_t first = s0, cnt = min(K, ge - s0);
+          if constexpr (CR) {
+            first = s0 & ~1u;
+            cnt = ((s0 + cnt + 1u) & ~1u) - first;
+          }
+          const uint32_t bytes = cnt * (uint32_t)(W * 4);
           mbar_expect_tx_only(&wbar[st], bytes);
-          bulk_g2s(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)s0 * W, bytes, &wbar[st]);
+          bulk_g2s(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
         }
       }
       __syncwarp();
@@ -287,17 +326,35 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
       const int st = (int)(it % kFragStages);
       mbar_wait(&wbar[st], (it / kFragStages) & 1u);
       const uint32_t* reg = my_region0 + (size_t)st * GPW * RS;
+      const uint32_t* reg_o = reg + 2 * o;  // CR: record 0 of this stage
       const uint32_t s0 = gs + t * K;
       const uint32_t n = (s0 < ge) ? min(K, ge - s0) : 0u;
       if (n > 0) {
         if (t == 0) {  // open the sub-range's first run
-          cur = reg[0] & p.out_mask;
+          if constexpr (CR) {
+            // start one run early so the first record's delta d0 lands on rowid[gs]: its
+            // flush of the still-empty accumulator is harmless (adds zeros to a valid row)
+            const uint32_t d0 = reg[2 * o] >> p.boff[0];
+            cur = __ldg(p.rowid + gs);
+            if (d0 != 0u && d0 != p.bmask[0]) cur -= d0;
+          } else {
+            cur = reg[0] & p.out_mask;
+          }
           if constexpr (S == 0) {
             if (p.owner && !first_shared && gs > 0) zero_rows(before, cur);  // gap rows are ours
           }
         }
         // record k of this group: [i_n, g_0 .. g_{G-1}, v]
+        // CR: i = the run delta d (0: same run)
         auto load_rec = [&](uint32_t k, uint32_t& i, uint32_t (&g)[G], float& v) {
+          if constexpr (CR) {
+            const uint2 w = *reinterpret_cast<const uint2*>(reg_o + (size_t)k * 2);
+            i = w.x >> p.boff[0];
+#pragma unroll
+            for (int q = 0; q < G; ++q) g[q] = (w.x >> p.boff[1 + q]) & p.bmask[1 + q];
+            v = __uint_as_float(w.y);
+            return;
+          }
           const uint32_t* rp = reg + (size_t)k * W;
           const uint4 w0 = lds128(rp);
           uint32_t w[W];
@@ -340,7 +397,16 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (ii[u] != cur) advance(ii[u]);
+            if constexpr (CR) {
+              if (ii[u]) {
+                flush_run(shared);
+                advanced = true;
+                if (ii[u] == p.bmask[0]) cur = __ldg(p.rowid + s0 + k + u);
+                else cur += ii[u];
+              }
+            } else if (ii[u] != cur) {
+              advance(ii[u]);
+            }
             const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
             f4fma_(acc0, vb, pr[u].a);
             if constexpr (VEC == 8) f4fma_(acc1, vb, pr[u].b);
@@ -357,7 +423,16 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
             f4mul_(pr.a, x.a);
             if constexpr (VEC == 8) f4mul_(pr.b, x.b);
           }
-          if (i != cur) advance(i);
+          if constexpr (CR) {
+            if (i) {
+              flush_run(shared);
+              advanced = true;
+              if (i == p.bmask[0]) cur = __ldg(p.rowid + s0 + k);
+              else cur += i;
+            }
+          } else if (i != cur) {
+            advance(i);
+          }
           const float4 vb = make_float4(v, v, v, v);
           f4fma_(acc0, vb, pr.a);
           if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
@@ -438,14 +513,20 @@ void boundary_zero3_r64(const Frag3Params& fp, uint32_t ctas, uint32_t groups, f
 
 template <int N, int R, int S>
 void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s) {
-  auto k = fp.W == 4 && N >= 4 ? frag3_kernel<N, R, S, (N >= 4)> : frag3_kernel<N, R, S, false>;
+  auto k = frag3_kernel<N, R, S, kRecPlain>;
+  if constexpr (N >= 4) {
+    if (fp.W == 4) k = frag3_kernel<N, R, S, kRecPacked>;
+  }
+  if constexpr (N == 3) {
+    if (fp.W == 2) k = frag3_kernel<N, R, S, kRecCompact>;
+  }
   SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   k<<<grid, threads, smem, s>>>(fp);
 }
 
 template <int N, int R, int S>
 int frag3_occ_one(int threads, size_t smem) {
-  auto k = frag3_kernel<N, R, S, false>;
+  auto k = frag3_kernel<N, R, S, kRecPlain>;
   SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int nb = 0;
   SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));

@@ -76,6 +76,9 @@ struct Plan {
   DevBuf chunk_tile;    // uint64[num_chunks]
   mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
   bool rec_packed = false;               // frag3 PK records (N >= 4, indices bit-packed)
+  bool rec_compact = false;              // frag3 CR records: 8 bytes [gathered fields | run-start
+                                         // bit 31, v]; i_n per slot in `rowid` (non-owner plans)
+  DevBuf rowid;                          // CR: uint32 i_n per kernel-order slot
   uint32_t rec_boff[SF_MAX_MODES] = {};  // PK: bit offset of field f (slot order)
   uint32_t rec_bmask[SF_MAX_MODES] = {}; // PK: width mask of field f
   size_t device_bytes() const;
@@ -145,6 +148,13 @@ __host__ __device__ __forceinline__ uint32_t frag3_region_words(uint32_t K, uint
   return ((base / 4u) % 2u == 0u) ? base + 4u : base + 8u;
 }
 
+// CR (8-byte records): a group's stage holds K records copied from a 16-byte-aligned
+// start, i.e. up to K + 2 records; stride/4 odd as above.
+__host__ __device__ __forceinline__ uint32_t frag3_cr_region_words(uint32_t K) {
+  const uint32_t base = 2u * K + 4u;
+  return ((base / 4u) % 2u == 0u) ? base + 4u : base;
+}
+
 // Records per group per stage for a launch's chunk_nnz (nonzeros per warp per stage).
 __host__ __device__ __forceinline__ uint32_t frag3_K(uint32_t chunk_nnz, uint32_t GPW) {
   uint32_t K = chunk_nnz / GPW;
@@ -184,6 +194,10 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
 bool frag_supported(int nmodes, int rank);
 // gathered slot order of a plan: staged modes ascending, then the other gathered modes
 int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode);
+// modes whose factor blocks are copied into shared memory (L2-tiled plans stage none)
+inline uint32_t smem_staged_mask(const sf_launch_t& l) {
+  return (l.flags & SF_LAUNCH_L2_TILES) ? 0u : l.staged_mask;
+}
 void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s);
 void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
                       uint32_t* const* inds, int* d_flag, cudaStream_t s);

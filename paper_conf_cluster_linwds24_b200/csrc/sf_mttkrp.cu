@@ -254,6 +254,7 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     fp.dims[m] = (uint32_t)t.dims[m];
   }
   fp.rec = p.rec.as<uint32_t>();
+  fp.rowid = p.rowid.as<uint32_t>();
   fp.out = out;
   fp.chunk_begin = p.chunk_begin.as<uint32_t>();
   fp.chunk_tile = p.chunk_tile.as<uint64_t>();
@@ -261,6 +262,7 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   fp.nnz = (uint32_t)p.nnz_local;
   const uint32_t gpw = (uint32_t)frag_groups_per_warp(R);
   fp.K = frag3_K((uint32_t)p.launch.chunk_nnz, gpw);
+  if (p.rec_compact) fp.K &= ~1u;  // CR stages keep the parity of the sub-range start (K even)
   fp.W = (uint32_t)p.rec_words;
   fp.out_mask = p.rec_packed ? p.rec_bmask[0] : 0xFFFFFFFFu;
   for (int f = 0; f < SF_MAX_MODES; ++f) {
@@ -268,7 +270,8 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     fp.bmask[f] = p.rec_bmask[f];
   }
   fp.owner = owner ? 1u : 0u;
-  const int S = frag_slot_order(N, n, p.launch.staged_mask, fp.slot_mode);
+  const int S = frag_slot_order(N, n, smem_staged_mask(p.launch), fp.slot_mode);
+  fp.l2tiles = (p.launch.flags & SF_LAUNCH_L2_TILES) ? 1u : 0u;
   uint32_t off = 0;
   for (int q = 0; q < S; ++q) {
     const int m = fp.slot_mode[q];

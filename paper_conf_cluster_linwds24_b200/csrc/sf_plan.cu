@@ -342,6 +342,61 @@ __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32
   }
 }
 
+// CR records (8 bytes): word 0 = the gathered slots' indices bit-packed (staged slots: row
+// inside the block, idx % block_rows), word 1 = v; rowid[k] = i_n.  cr_delta_kernel then
+// writes the run delta d into the top bits (sf_frag3.cuh kRecCompact).
+struct CrParams {
+  int in_word;               // raw AoS word of i_n
+  int nslots;                // gathered slots (N - 1)
+  int slot_word[SF_MAX_MODES];
+  uint32_t slot_mod[SF_MAX_MODES];  // 0 = full index, else block rows (staged slot)
+  uint32_t boff[SF_MAX_MODES];
+  int val_word;
+};
+
+template <int WR>
+__global__ void gather_rec_cr_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
+                                     uint64_t n, CrParams cp, uint32_t* __restrict__ rec,
+                                     uint32_t* __restrict__ rowid) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)perm[k] * WR);
+    uint32_t w[WR];
+#pragma unroll
+    for (int q = 0; q < WR / 4; ++q) {
+      const uint4 v = __ldg(src + q);
+      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
+    }
+    auto word = [&](int i) {
+      uint32_t x = 0;
+#pragma unroll
+      for (int q = 0; q < WR; ++q) x = (i == q) ? w[q] : x;
+      return x;
+    };
+    uint32_t x = 0;
+    for (int q = 0; q < cp.nslots; ++q) {
+      uint32_t idx = word(cp.slot_word[q]);
+      if (cp.slot_mod[q]) idx %= cp.slot_mod[q];
+      x |= idx << cp.boff[q];
+    }
+    reinterpret_cast<uint2*>(rec)[k] = make_uint2(x, word(cp.val_word));
+    rowid[k] = word(cp.in_word);
+  }
+}
+
+__global__ void cr_delta_kernel(const uint32_t* __restrict__ rowid, uint64_t n, uint32_t shift, uint32_t esc,
+                                uint32_t* __restrict__ rec) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    uint32_t d = esc;
+    if (k > 0) {
+      const uint32_t a = rowid[k - 1], b = rowid[k];
+      d = (b == a) ? 0u : ((b > a && b - a < esc) ? b - a : esc);
+    }
+    rec[2 * k] |= d << shift;
+  }
+}
+
 struct GatherParams {
   const uint32_t* src[SF_MAX_MODES];
   uint32_t* dst[SF_MAX_MODES];
@@ -493,7 +548,61 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   }
   const bool use_rec = launch.kernel == SF_KERNEL_FRAG && frag_supported(N, rank);
   p.rec_words = 0;
-  if (use_rec) {
+  p.rec_compact = false;
+  p.rowid.release();
+  // CR records: non-owner plans (staged or L2-tiled or NO_OWNER_STORES; the owner path
+  // needs i_n at every run edge) with N = 3 whose gathered fields leave >= 2 bits for d.
+  bool compact = false;
+  int cr_bits[SF_MAX_MODES] = {};
+  if (use_rec && N == 3 && (launch.flags & SF_LAUNCH_COMPACT) && !(launch.flags & SF_LAUNCH_DETERMINISTIC) &&
+      (launch.staged_mask != 0 || (launch.flags & SF_LAUNCH_NO_OWNER_STORES))) {
+    int slot_mode[SF_MAX_MODES];
+    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
+    int total = 0;
+    for (int q = 0; q < N - 1; ++q) {
+      const int m = slot_mode[q];
+      const bool in_smem = smem_staged_mask(launch) & (1u << m);
+      cr_bits[q] = index_bits(in_smem ? (uint64_t)launch.block_rows[m] : t.dims[m]);
+      total += cr_bits[q];
+    }
+    compact = total <= 30;
+  }
+  if (use_rec && compact) {
+    int slot_mode[SF_MAX_MODES];
+    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
+    p.rec_words = 2;
+    p.rec_compact = true;
+    p.rec.alloc(nl * 8 + kPadBytes);
+    p.rowid.alloc(nl * 4 + kPadBytes);
+    SF_CUDA(cudaMemsetAsync(p.rec.as<uint32_t>() + nl * 2, 0, kPadBytes, t.stream));
+    CrParams cp{};
+    cp.in_word = mode;
+    cp.nslots = N - 1;
+    cp.val_word = N;
+    uint32_t off = 0;
+    int total = 0;
+    for (int q = 0; q < N - 1; ++q) total += cr_bits[q];
+    const uint32_t dbits = (uint32_t)std::min(16, 32 - total);
+    p.rec_boff[0] = 32u - dbits;        // run delta d in the top dbits bits
+    p.rec_bmask[0] = (1u << dbits) - 1u;  // escape value E
+    for (int q = 0; q < N - 1; ++q) {
+      const int m = slot_mode[q];
+      cp.slot_word[q] = m;
+      cp.slot_mod[q] = (smem_staged_mask(launch) & (1u << m)) ? launch.block_rows[m] : 0u;
+      cp.boff[q] = off;
+      p.rec_boff[1 + q] = off;
+      p.rec_bmask[1 + q] = (1u << cr_bits[q]) - 1u;
+      off += (uint32_t)cr_bits[q];
+    }
+    if (nl) {
+      gather_rec_cr_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, cp,
+                                                                p.rec.as<uint32_t>(), p.rowid.as<uint32_t>());
+      cr_delta_kernel<<<grid_for(nl), 256, 0, t.stream>>>(p.rowid.as<uint32_t>(), nl, p.rec_boff[0], p.rec_bmask[0],
+                                                          p.rec.as<uint32_t>());
+      count_launch(2);
+      SF_CUDA(cudaGetLastError());
+    }
+  } else if (use_rec) {
     // frag3 records in slot order [i_n, staged slots, other gathered slots, value, 0...]
     const bool packed = N >= 4 && rec_packable(t);
     const int WK = packed ? 4 : rec_words_for(N);
@@ -504,7 +613,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     RecParams rp{};
     for (int d = 0; d < 8; ++d) rp.fmap[d] = -1;
     int slot_mode[SF_MAX_MODES];
-    frag_slot_order(N, mode, launch.staged_mask, slot_mode);
+    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
     rp.fmap[0] = mode;
     for (int q = 0; q < N - 1; ++q) rp.fmap[1 + q] = slot_mode[q];
     rp.fmap[N] = N;  // value word of the raw record

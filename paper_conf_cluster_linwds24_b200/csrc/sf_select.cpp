@@ -14,6 +14,7 @@
 // block sizes; the chunk length C; threads per CTA.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "sf_internal.h"
 
@@ -32,8 +33,9 @@ size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l
   const uint32_t gpw = (uint32_t)frag_groups_per_warp(rank);
   const uint32_t K = frag3_K((uint32_t)l.chunk_nnz, gpw);
   b += nwarps * kStagesHost * gpw * (size_t)frag3_region_words(K, (uint32_t)tensor_rec_words(t)) * 4;
-  for (int m = 0; m < t.nmodes; ++m)
-    if (l.staged_mask & (1u << m)) b += (size_t)l.block_rows[m] * rank * 4;
+  if (!(l.flags & SF_LAUNCH_L2_TILES))
+    for (int m = 0; m < t.nmodes; ++m)
+      if (l.staged_mask & (1u << m)) b += (size_t)l.block_rows[m] * rank * 4;
   return b;
 }
 
@@ -59,8 +61,9 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   if (l.flags & SF_LAUNCH_DETERMINISTIC) {  // A7 option: unstaged owner-store plan (no atomics)
     l.staged_mask = 0u;
     for (int m = 0; m < SF_MAX_MODES; ++m) l.block_rows[m] = 0;
-    l.flags &= ~SF_LAUNCH_NO_OWNER_STORES;
+    l.flags &= ~(SF_LAUNCH_NO_OWNER_STORES | SF_LAUNCH_L2_TILES);
   }
+  if (l.staged_mask == 0u) l.flags &= ~SF_LAUNCH_L2_TILES;
 }
 
 // Selector rules, calibrated on the sweeps in profiles/:
@@ -244,7 +247,63 @@ static int tree_predict(const double* x, int nx) {
   return -1;
 }
 
+// ---------------------------------------------------------------------------
+// L2-tile refinement (SF_LAUNCH_L2_TILES; DESIGN.md §5 "L2 tiles").  When the pick is an
+// unstaged plan (the hyper-sparse regime: factors >> L2, gathers DRAM-latency bound), tile
+// the order by 64 MB row blocks of the LARGEST gathered factor of >= 64 MB, so at any moment
+// every CTA gathers that factor from one L2-resident block -- unless re-visiting Y once per
+// (tile, row) costs too much: rho = T * touched(T) / nnz <= 0.25, touched(T) = the expected
+// rows of Y a tile touches, sum_b slices_b (1 - exp(-1.44 * 2^b / T)) over the log2
+// slice-length histogram (PAPER.md L195 features); rho = 0 when Y fits in 32 MB (its
+// re-visits hit L2).  Calibrated on tools/l2tile_study.py over the BASELINE.json and Table III
+// shapes (profiles/r01s3_l2tiles.jsonl): the rule's pick is within 2.4 % of the best tiled
+// option on average (worst 20 %), 1.1-2.1x over the unstaged plan where it tiles.
+static constexpr double kL2BlockBytes = 64.0 * 1024 * 1024;
+static constexpr double kL2MinFactorBytes = 64.0 * 1024 * 1024;
+static constexpr double kL2MaxRevisit = 0.25;
+static constexpr double kL2YInCache = 32.0 * 1024 * 1024;
+
+static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local,
+                           sf_launch_t& l) {
+  if (l.kernel != SF_KERNEL_FRAG || l.staged_mask != 0 || (l.flags & SF_LAUNCH_DETERMINISTIC) || nnz_local == 0 ||
+      f.nnz == 0)
+    return;
+  const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
+  int best = -1;
+  double bestF = 0;
+  for (int m = 0; m < t.nmodes; ++m) {
+    if (m == mode) continue;
+    const double F = (double)t.dims[m] * RB;
+    if (F < kL2MinFactorBytes || F <= bestF) continue;
+    const double T = std::ceil(F / kL2BlockBytes);
+    double rho = 0;
+    if (Yb > kL2YInCache) {
+      double touched = 0;
+      for (int b = 0; b < SF_HIST_BINS; ++b)
+        touched += (double)f.slice_hist[b] * (1.0 - std::exp(-1.44 * std::ldexp(1.0, b) / T));
+      rho = T * touched / (double)f.nnz;
+    }
+    if (rho > kL2MaxRevisit) continue;
+    best = m;
+    bestF = F;
+  }
+  if (best < 0) return;
+  sf_launch_t c = l;
+  c.staged_mask = 1u << best;
+  c.block_rows[best] = (uint32_t)std::max(1.0, kL2BlockBytes / RB);
+  c.flags = (c.flags | SF_LAUNCH_L2_TILES) & ~SF_LAUNCH_NO_OWNER_STORES;
+  normalize_launch(t, mode, rank, c);
+  if (frag_smem_bytes(t, mode, rank, c) <= t.smem_optin) l = c;
+}
+
+static bool l2_refine_enabled() {
+  const char* e = std::getenv("SF_L2_TILES");  // "0": keep the selector's unstaged pick (A/B)
+  return !(e && e[0] == '0');
+}
+
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local) {
+  sf_launch_t l{};
+  bool picked = false;
   if (g_have_model && frag_supported(t.nmodes, rank) && nnz_local > 0) {
     double x[32];
     const int nx = selector_features(t, f, mode, rank, nnz_local, x);
@@ -252,10 +311,15 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
       const int c = tree_predict(x, nx);
       sf_launch_t cand[16];
       const int nc = selector_candidates(t, mode, rank, cand);
-      if (c >= 0 && c < nc && frag_smem_bytes(t, mode, rank, cand[c]) <= t.smem_optin) return cand[c];
+      if (c >= 0 && c < nc && frag_smem_bytes(t, mode, rank, cand[c]) <= t.smem_optin) {
+        l = cand[c];
+        picked = true;
+      }
     }
   }
-  return select_rules(t, f, mode, rank, nnz_local);
+  if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
+  if (l2_refine_enabled()) l2_tile_refine(t, f, mode, rank, nnz_local, l);
+  return l;
 }
 
 }  // namespace sf

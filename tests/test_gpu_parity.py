@@ -46,6 +46,17 @@ def _launches(dims, n):
     yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, block_threads=1024, staged={others[0]: 7})
     yield sf.Launch.make(kernel=FRAG, chunk_nnz=256, block_threads=128, ctas_per_sm=1,
                          staged={others[-1]: dims[others[-1]]})
+    # L2 tiles (SF_LAUNCH_L2_TILES): tiled order, no shared-memory staging, every CTA takes a
+    # share of every tile; one and two tiled modes, ragged last block
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=32, staged={others[-1]: max(1, dims[others[-1]] // 4 + 1)},
+                         flags=sf.LAUNCH_L2_TILES)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, block_threads=256,
+                         staged={m: max(1, dims[m] // 3 + 1) for m in others}, flags=sf.LAUNCH_L2_TILES)
+    # compact 8-byte records (SF_LAUNCH_COMPACT, N = 3 non-owner plans): staged, L2 tiles, unstaged
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=48, staged={others[0]: 7}, flags=sf.LAUNCH_COMPACT)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={others[-1]: max(1, dims[others[-1]] // 4 + 1)},
+                         flags=sf.LAUNCH_COMPACT | sf.LAUNCH_L2_TILES)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=sf.LAUNCH_COMPACT | sf.LAUNCH_NO_OWNER_STORES)
 
 
 @pytest.mark.parametrize("name", ["tiny", "tiny_skew"])
@@ -66,11 +77,11 @@ def test_ranks_and_orders(cuda_device, R, dims):
     nnz = 3001  # ragged
     inds, vals = synth.gen_coo(dims, nnz, 99, zipf=(0.8,) * len(dims), val_kind="signed")
     facs = synth.gen_factors(dims, R, 77, "signed")
-    for staged in (False, True):
+    for staged, flags in ((False, 0), (True, 0), (True, sf.LAUNCH_L2_TILES), (True, sf.LAUNCH_COMPACT)):
         def L(n):
             if not staged:
                 return sf.Launch.make(kernel=FRAG, chunk_nnz=100)
-            return sf.Launch.make(kernel=FRAG, chunk_nnz=100,
+            return sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=flags,
                                   staged={m: max(1, dims[m] // 2) for m in range(len(dims)) if m != n})
         Y, _ = G.run(dims, inds, vals, facs, R, launch=L)
         for n in range(len(dims)):
@@ -103,8 +114,9 @@ def test_plan_bit_exact_vs_oracle(cuda_device):
                 assert f[k] == of[k], k
             assert f["slice_hist"] == list(of["slice_hist"])
             others = [m for m in range(3) if m != n]
-            for staged in ({}, {others[0]: 13}, {others[0]: 40, others[1]: 7}):
-                L = sf.Launch.make(kernel=FRAG, chunk_nnz=100, staged=staged)
+            for staged, flags in (({}, 0), ({others[0]: 13}, 0), ({others[0]: 40, others[1]: 7}, 0),
+                                  ({others[1]: 50}, sf.LAUNCH_L2_TILES)):
+                L = sf.Launch.make(kernel=FRAG, chunk_nnz=100, staged=staged, flags=flags)
                 t.set_launch(n, 16, L)
                 perm, chunks = t.plan_export(n, 16)
                 ref = oplan.plan_order(dims, inds, n, tuple(sorted(staged)), staged)
