@@ -11,6 +11,9 @@
 #include <algorithm>
 #include <cstring>
 #include <map>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <mutex>
 #include <new>
 #include <string>
@@ -24,6 +27,18 @@ std::atomic<uint64_t> g_launches{0};
 static thread_local std::string g_err;
 
 void set_error(const std::string& msg) { g_err = msg; }
+
+void trace_mark(const char* phase) {
+  static const bool on = [] {
+    const char* e = std::getenv("SF_PLAN_TRACE");
+    return e && e[0] == '1';
+  }();
+  if (!on) return;
+  static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
+  const auto now = std::chrono::steady_clock::now();
+  fprintf(stderr, "[sf trace] %-24s +%.3f ms\n", phase, std::chrono::duration<double, std::milli>(now - last).count());
+  last = now;
+}
 
 // Caching device allocator.  cudaMalloc/cudaFree of GB-sized plan arrays cost tens of ms
 // each and cudaFree synchronizes the device; blocks are instead kept in a size-keyed free
@@ -217,10 +232,12 @@ static Plan* get_plan(Tensor& t, int mode, int rank) {
 }
 
 static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override_launch) {
+  trace_mark("plan: enter");
   SF_CUDA(cudaSetDevice(t.device));
   sf_features_t f;
   DevBuf keys, pos;  // the matricized order, sorted once for features + the plan
   compute_features(t, mode, &f, &keys, &pos);
+  trace_mark("plan: features");
   const uint64_t lo = (uint64_t)(((unsigned __int128)t.rank * t.nnz) / t.nranks);
   const uint64_t hi = (uint64_t)(((unsigned __int128)(t.rank + 1) * t.nnz) / t.nranks);
   sf_launch_t l;
@@ -232,9 +249,11 @@ static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override
   }
   if (l.kernel == SF_KERNEL_FRAG && frag_smem_bytes(t, mode, rank, l) > t.smem_optin)
     throw StatusError{SF_ERR_INVALID_ARG, "launch needs more shared memory than the device has"};
+  trace_mark("plan: select");
   Plan* p = new Plan();
   try {
     build_plan(t, *p, mode, rank, l, &keys, &pos);
+    trace_mark("plan: build");
   } catch (...) {
     delete p;
     throw;

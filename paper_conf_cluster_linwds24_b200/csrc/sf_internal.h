@@ -14,6 +14,9 @@
 
 namespace sf {
 
+// SF_PLAN_TRACE=1: host wall-clock phase marks of sf_plan on stderr (profiling aid).
+void trace_mark(const char* phase);
+
 // Thread-local error detail + status plumbing.
 void set_error(const std::string& msg);
 extern std::atomic<uint64_t> g_launches;

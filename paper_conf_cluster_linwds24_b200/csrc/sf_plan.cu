@@ -405,43 +405,36 @@ struct GatherParams {
   int nmodes;
 };
 
-// Chunk start flags: k starts a chunk iff (k - tile_start(k)) % C == 0.
-__global__ void tile_start_kernel(const uint64_t* __restrict__ tkey, uint64_t n, uint32_t* __restrict__ ts,
-                                  unsigned long long* __restrict__ ntiles) {
+// Chunks of tile t: nch[t] = ceil(cnt[t] / C) (0 past the encoded runs: cnt was zeroed).
+__global__ void chunk_count_kernel(const uint32_t* __restrict__ cnt, uint64_t ntiles, uint32_t C,
+                                   uint32_t* __restrict__ nch) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned long long c = 0;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    const bool st = (k == 0) || (tkey ? tkey[k] != tkey[k - 1] : false);
-    ts[k] = st ? (uint32_t)k : 0u;
-    c += st;
-  }
-  typedef cub::BlockReduce<unsigned long long, 256> BR;
-  __shared__ typename BR::TempStorage tmp;
-  unsigned long long a = BR(tmp).Sum(c);
-  if (threadIdx.x == 0) atomicAdd(ntiles, a);
+  for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += stride)
+    nch[t] = (cnt[t] + C - 1) / C;
 }
 
-__global__ void chunk_flag_kernel(const uint32_t* __restrict__ ts, uint64_t n, uint32_t C,
-                                  uint32_t* __restrict__ flag) {
+// chunk j (< nchunks) of tile t (coff[t] <= j < coff[t+1], binary search over the nr tiles):
+// begins at tstart[t] + (j - coff[t]) * C, tile id uniq[t]; cbegin[nchunks] = n.  Without
+// tiles (uniq == nullptr) every chunk is j * C of tile 0.
+__global__ void chunk_fill_kernel(const uint64_t* __restrict__ uniq, const uint32_t* __restrict__ tstart,
+                                  const uint32_t* __restrict__ coff, const void* unused, uint32_t nr, uint32_t C,
+                                  uint64_t n, uint64_t nchunks, uint32_t* __restrict__ cbegin,
+                                  uint64_t* __restrict__ ctile) {
+  (void)unused;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride)
-    flag[k] = (((uint32_t)k - ts[k]) % C == 0u) ? 1u : 0u;
-}
-
-__global__ void chunk_scatter_kernel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ excl,
-                                     const uint64_t* __restrict__ tkey, uint64_t n,
-                                     uint32_t* __restrict__ cbegin, uint64_t* __restrict__ ctile) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    if (flag[k]) {
-      const uint32_t j = excl[k];
-      cbegin[j] = (uint32_t)k;
-      ctile[j] = tkey ? tkey[k] : 0ull;
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j <= nchunks; j += stride) {
+    if (j == nchunks) { cbegin[j] = (uint32_t)n; continue; }
+    if (!uniq) { cbegin[j] = (uint32_t)(j * C); ctile[j] = 0; continue; }
+    uint32_t lo = 0, hi = nr;  // last tile with coff <= j
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (coff[mid] <= j) lo = mid; else hi = mid;
     }
+    cbegin[j] = tstart[lo] + (uint32_t)(j - coff[lo]) * C;
+    ctile[j] = uniq[lo];
   }
 }
 
-__global__ void set_u32_kernel(uint32_t* p, uint32_t v) { *p = v; }
 
 void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launch, DevBuf* keys_in,
                 DevBuf* pos_in) {
@@ -472,6 +465,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     t.have_features[mode] = true;
   }
   p.feat = t.features[mode];
+  trace_mark("build: sorted");
 
   const int s = secondary_mode(t, mode);
   p.row_begin = p.row_end = 0;
@@ -483,6 +477,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     p.row_begin = kb / t.dims[s];
     p.row_end = ke / t.dims[s] + 1;
   }
+  trace_mark("build: shard range");
   const bool staged_is_secondary = launch.kernel == SF_KERNEL_FRAG && launch.staged_mask == (1u << s);
   if (!staged_is_secondary) keys.release();  // else kept for the tile keys
 
@@ -531,6 +526,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     }
   }
 
+  trace_mark("build: tile order");
   // AoS record copy of the raw COO (built once per tensor, reused by every mode's plan)
   const int WR = (N + 1 <= 4) ? 4 : (N + 1 <= 8 ? 8 : 16);
   if (nl && !t.aos.p) {
@@ -673,45 +669,64 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     }
   }
   p.perm = std::move(perm);
+  trace_mark("build: records");
 
   // Chunks.
   p.num_chunks = 0;
   p.num_tiles = 0;
   if (nl) {
+    // Per tile (run of equal tile keys in kernel order): its start, its nonzero count and
+    // ceil(count / C) chunks; chunk j of tile t begins at start_t + (j - first_chunk_t) * C.
+    // O(num_tiles + num_chunks) after one run-length encode of the tile keys.
     const uint32_t C = (uint32_t)std::max(1, launch.chunk_nnz);
-    DevBuf ts(nl * 4 + 16), flag(nl * 4 + 16), excl(nl * 4 + 16), cnt(16);
-    SF_CUDA(cudaMemsetAsync(cnt.p, 0, 16, t.stream));
-    const uint64_t* tk = staged ? tkeys.as<uint64_t>() : nullptr;
-    tile_start_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tk, nl, ts.as<uint32_t>(), cnt.as<unsigned long long>());
-    count_launch();
-    size_t temp = 0;
-    SF_CUDA(cub::DeviceScan::InclusiveScan(nullptr, temp, ts.as<uint32_t>(), ts.as<uint32_t>(), MaxOp(),
-                                           (int64_t)nl, t.stream));
-    size_t temp2 = 0;
-    SF_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, temp2, flag.as<uint32_t>(), excl.as<uint32_t>(),
-                                          (int64_t)nl, t.stream));
-    DevBuf tmp(std::max(temp, temp2) + 16);
-    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, ts.as<uint32_t>(), ts.as<uint32_t>(), MaxOp(),
-                                           (int64_t)nl, t.stream));
-    chunk_flag_kernel<<<grid_for(nl), 256, 0, t.stream>>>(ts.as<uint32_t>(), nl, C, flag.as<uint32_t>());
-    SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, temp2, flag.as<uint32_t>(), excl.as<uint32_t>(),
-                                          (int64_t)nl, t.stream));
-    count_launch(5);
-    uint32_t last_excl, last_flag;
-    unsigned long long ntiles;
-    SF_CUDA(cudaMemcpyAsync(&last_excl, excl.as<uint32_t>() + nl - 1, 4, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaMemcpyAsync(&last_flag, flag.as<uint32_t>() + nl - 1, 4, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaMemcpyAsync(&ntiles, cnt.p, 8, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaStreamSynchronize(t.stream));
-    p.num_chunks = (uint64_t)last_excl + last_flag;
-    p.num_tiles = ntiles;
-    p.chunk_begin.alloc((p.num_chunks + 1) * 4 + 16);
-    p.chunk_tile.alloc(p.num_chunks * 8 + 16);
-    chunk_scatter_kernel<<<grid_for(nl), 256, 0, t.stream>>>(flag.as<uint32_t>(), excl.as<uint32_t>(), tk, nl,
-                                                            p.chunk_begin.as<uint32_t>(),
-                                                            p.chunk_tile.as<uint64_t>());
-    set_u32_kernel<<<1, 1, 0, t.stream>>>(p.chunk_begin.as<uint32_t>() + p.num_chunks, (uint32_t)nl);
-    count_launch(2);
+    if (!staged) {
+      p.num_tiles = 1;
+      p.num_chunks = (nl + C - 1) / C;
+      p.chunk_begin.alloc((p.num_chunks + 1) * 4 + 16);
+      p.chunk_tile.alloc(p.num_chunks * 8 + 16);
+      chunk_fill_kernel<<<grid_for(p.num_chunks + 1), 256, 0, t.stream>>>(
+          nullptr, nullptr, nullptr, nullptr, 1, C, nl, p.num_chunks, p.chunk_begin.as<uint32_t>(),
+          p.chunk_tile.as<uint64_t>());
+      count_launch();
+    } else {
+      uint64_t tiles_bound = 1;
+      for (int m = 0; m < N; ++m)
+        if (launch.staged_mask & (1u << m))
+          tiles_bound = std::min<uint64_t>(nl, tiles_bound * ((t.dims[m] + launch.block_rows[m] - 1) / launch.block_rows[m]));
+      tiles_bound = std::min<uint64_t>(tiles_bound, nl);
+      DevBuf uniq(tiles_bound * 8 + 16), cnts(tiles_bound * 4 + 16), nruns(16), nch(tiles_bound * 4 + 16),
+          tstart(tiles_bound * 4 + 16), coff(tiles_bound * 4 + 16);
+      SF_CUDA(cudaMemsetAsync(cnts.p, 0, tiles_bound * 4 + 16, t.stream));
+      size_t t1 = 0, t2 = 0;
+      SF_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, t1, tkeys.as<uint64_t>(), uniq.as<uint64_t>(),
+                                                 cnts.as<uint32_t>(), nruns.as<uint32_t>(), (int64_t)nl, t.stream));
+      SF_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, t2, cnts.as<uint32_t>(), tstart.as<uint32_t>(),
+                                            (int64_t)tiles_bound, t.stream));
+      DevBuf tmp(std::max(t1, t2) + 16);
+      SF_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, t1, tkeys.as<uint64_t>(), uniq.as<uint64_t>(),
+                                                 cnts.as<uint32_t>(), nruns.as<uint32_t>(), (int64_t)nl, t.stream));
+      chunk_count_kernel<<<grid_for(tiles_bound), 256, 0, t.stream>>>(cnts.as<uint32_t>(), tiles_bound, C,
+                                                                      nch.as<uint32_t>());
+      SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, t2, cnts.as<uint32_t>(), tstart.as<uint32_t>(),
+                                            (int64_t)tiles_bound, t.stream));
+      SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, t2, nch.as<uint32_t>(), coff.as<uint32_t>(),
+                                            (int64_t)tiles_bound, t.stream));
+      count_launch(5);
+      uint32_t nr = 0, last_off = 0, last_n = 0;
+      SF_CUDA(cudaMemcpyAsync(&nr, nruns.p, 4, cudaMemcpyDeviceToHost, t.stream));
+      SF_CUDA(cudaMemcpyAsync(&last_off, coff.as<uint32_t>() + tiles_bound - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+      SF_CUDA(cudaMemcpyAsync(&last_n, nch.as<uint32_t>() + tiles_bound - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+      SF_CUDA(cudaStreamSynchronize(t.stream));
+      trace_mark("build: chunk count sync");
+      p.num_tiles = nr;
+      p.num_chunks = (uint64_t)last_off + last_n;
+      p.chunk_begin.alloc((p.num_chunks + 1) * 4 + 16);
+      p.chunk_tile.alloc(p.num_chunks * 8 + 16);
+      chunk_fill_kernel<<<grid_for(p.num_chunks + 1), 256, 0, t.stream>>>(
+          uniq.as<uint64_t>(), tstart.as<uint32_t>(), coff.as<uint32_t>(), nullptr, nr, C, nl, p.num_chunks,
+          p.chunk_begin.as<uint32_t>(), p.chunk_tile.as<uint64_t>());
+      count_launch();
+    }
     SF_CUDA(cudaGetLastError());
   } else {
     p.chunk_begin.alloc(16);
