@@ -173,6 +173,14 @@ static void upload(Tensor& t, const uint32_t* const* inds, const float* vals, in
   // pinned staging ring for pageable input: one slot per stream
   std::vector<void*> stage(nstreams, nullptr);
   std::vector<cudaEvent_t> done(nstreams, nullptr);
+  // A8: each segment's matricized keys are sorted on its stream behind its copy (presort)
+  const bool presort = presort_begin(t, seg_len);
+  std::vector<DevBuf> ptemp(presort ? nstreams : 0);
+  size_t ptemp_bytes = 0;
+  if (presort) {
+    ptemp_bytes = presort_temp_bytes(t, seg_len);
+    for (auto& b : ptemp) b.alloc(ptemp_bytes + 16);
+  }
   try {
     if (pageable) {
       for (int s = 0; s < nstreams; ++s) {
@@ -205,8 +213,10 @@ static void upload(Tensor& t, const uint32_t* const* inds, const float* vals, in
         SF_CUDA(cudaMemcpyAsync(t.val.as<float>() + a, vals + a, len * 4, cudaMemcpyHostToDevice, st[s]));
       }
       validate_indices(N, t.dims, len, dseg, d_flag, st[s]);
+      if (presort) presort_segment(t, a, len, st[s], ptemp[s].p, ptemp_bytes);
     }
     for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
+    t.pre_alt.release();
   } catch (...) {
     for (auto& s : st) cudaStreamSynchronize(s);
     for (auto& s : st) cudaStreamDestroy(s);

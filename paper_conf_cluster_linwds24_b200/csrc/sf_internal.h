@@ -102,6 +102,15 @@ struct Tensor {
   bool have_features[SF_MAX_MODES] = {};
   sf_features_t features[SF_MAX_MODES] = {};
   std::map<std::pair<int, int>, Plan*> plans;  // (mode, rank) -> plan
+  // A8 upload || presort (sf_plan.cu presort_*): for each mode, the matricized key of every
+  // uploaded segment composed with its input position, (key << pre_pb) | pos, sorted on the
+  // segment's upload stream while later segments are still in flight; the first sf_plan of
+  // the mode merges the sorted runs instead of sorting all nonzeros.
+  DevBuf pre[SF_MAX_MODES];
+  bool have_pre[SF_MAX_MODES] = {};
+  DevBuf pre_alt;              // composed keys of a segment before its sort (upload only)
+  uint64_t pre_seg_len = 0;
+  int pre_pb = 0;              // position bits
   cudaStream_t stream = nullptr;               // internal stream for planning
   ~Tensor();
 };
@@ -171,6 +180,12 @@ inline int frag_groups_per_warp(int R) {
 }
 
 // ---- planning (sf_plan.cu) ----
+// upload || presort: decide and allocate (returns false: no mode qualifies / disabled by
+// SF_PRESORT=0 / not enough memory), per-segment work on the upload stream, CUB temp bytes
+// one segment's sort needs.
+bool presort_begin(Tensor& t, uint64_t seg_len);
+void presort_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t s, void* temp, size_t temp_bytes);
+size_t presort_temp_bytes(const Tensor& t, uint64_t seg_len);
 // keys/pos (optional): receive the matricized order (sorted keys, input positions) when
 // this call had to sort, so build_plan can reuse it instead of sorting again.
 void compute_features(Tensor& t, int mode, sf_features_t* out, DevBuf* keys, DevBuf* pos);

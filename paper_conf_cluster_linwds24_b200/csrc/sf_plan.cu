@@ -16,7 +16,10 @@
 // All of it is integer work; tests compare it == against oracle/plan.py.
 #include <cub/cub.cuh>
 
+#include <cub/device/device_merge.cuh>
+
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "sf_internal.h"
@@ -128,8 +131,128 @@ struct MaxOp {
   __device__ __forceinline__ uint32_t operator()(uint32_t a, uint32_t b) const { return a > b ? a : b; }
 };
 
+// ---------------------------------------------------------------------------
+// A8 upload || presort.  Composite key c = (i_n * I_s + i_s) << pb | e (e = input position,
+// pb = bits(nnz - 1)) is unique, so sorting / merging c is the stable matricized sort.
+static inline int key_bits(const Tensor& t, int mode) {
+  const int s = secondary_mode(t, mode);
+  return std::max(1, bitlen(t.dims[mode] * t.dims[s] - 1));
+}
+
+__global__ void compose_key_kernel(const uint32_t* __restrict__ in, const uint32_t* __restrict__ is, uint64_t Is,
+                                   uint64_t a, uint64_t len, int pb, uint64_t* __restrict__ out) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < len; e += stride)
+    out[e] = (((uint64_t)in[e] * Is + (uint64_t)is[e]) << pb) | (a + e);
+}
+
+__global__ void split_key_kernel(const uint64_t* __restrict__ c, uint64_t n, int pb, uint64_t* __restrict__ key,
+                                 uint32_t* __restrict__ pos) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t mask = (1ull << pb) - 1ull;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    const uint64_t x = c[e];
+    key[e] = x >> pb;
+    pos[e] = (uint32_t)(x & mask);
+  }
+}
+
+static void aos_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t st);  // below
+
+bool presort_begin(Tensor& t, uint64_t seg_len) {
+  const char* env = std::getenv("SF_PRESORT");
+  if (env && env[0] == '0') return false;
+  const uint64_t n = t.nnz;
+  if (n < 2 || seg_len >= n || n >= (1ull << 30)) return false;
+  const int pb = std::max(1, bitlen(n - 1));
+  int modes = 0;
+  for (int m = 0; m < t.nmodes; ++m) modes += (key_bits(t, m) + pb <= 64);
+  if (!modes) return false;
+  size_t free_b = 0, total_b = 0;
+  SF_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  // pre keys + the segment staging buffer now, and a merge buffer + split keys/positions later
+  if ((double)n * 8.0 * (modes + 4) > 0.6 * (double)free_b) return false;
+  t.pre_pb = pb;
+  t.pre_seg_len = seg_len;
+  for (int m = 0; m < t.nmodes; ++m) {
+    t.have_pre[m] = key_bits(t, m) + pb <= 64;
+    if (t.have_pre[m]) t.pre[m].alloc(n * 8 + 16);
+  }
+  t.pre_alt.alloc(n * 8 + 16);
+  const int WR = (t.nmodes + 1 <= 4) ? 4 : (t.nmodes + 1 <= 8 ? 8 : 16);
+  t.aos.alloc((size_t)n * WR * 4 + 64);  // the AoS copy is built per segment too
+  t.aos_words = WR;
+  return true;
+}
+
+size_t presort_temp_bytes(const Tensor& t, uint64_t seg_len) {
+  size_t b = 0;
+  SF_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, b, (const uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)seg_len,
+                                         0, 64, (cudaStream_t)0));
+  (void)t;
+  return b;
+}
+
+void presort_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t st, void* temp, size_t temp_bytes) {
+  aos_segment(t, a, len, st);
+  for (int m = 0; m < t.nmodes; ++m) {
+    if (!t.have_pre[m]) continue;
+    const int s = secondary_mode(t, m);
+    uint64_t* alt = t.pre_alt.as<uint64_t>() + a;
+    compose_key_kernel<<<grid_for(len), 256, 0, st>>>(t.ind[m].as<uint32_t>() + a, t.ind[s].as<uint32_t>() + a,
+                                                      t.dims[s], a, len, t.pre_pb, alt);
+    // the position bits are already ascending inside the segment and LSD radix sorting is
+    // stable: sorting only the key bits [pb, pb + kb) orders the composites completely
+    size_t tb = temp_bytes;
+    SF_CUDA(cub::DeviceRadixSort::SortKeys(temp, tb, alt, t.pre[m].as<uint64_t>() + a, (int64_t)len, t.pre_pb,
+                                           t.pre_pb + key_bits(t, m), st));
+    count_launch(1 + (uint64_t)((key_bits(t, m) + 7) / 8) * 3);
+  }
+  SF_CUDA(cudaGetLastError());
+}
+
+// Merge the sorted segment runs of mode `mode` (pairwise, log2(#runs) rounds) and split the
+// composite keys into the matricized keys + input positions.
+static void presort_finish(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_out) {
+  const uint64_t n = t.nnz;
+  DevBuf cur = std::move(t.pre[mode]);
+  t.have_pre[mode] = false;
+  DevBuf nxt(n * 8 + 16), tmp;
+  size_t tmp_bytes = 0;
+  for (uint64_t L = t.pre_seg_len; L < n; L *= 2) {
+    for (uint64_t a = 0; a < n; a += 2 * L) {
+      const uint64_t b = std::min(n, a + L), c = std::min(n, a + 2 * L);
+      if (b >= c) {  // odd run out: carried over
+        SF_CUDA(cudaMemcpyAsync(nxt.as<uint64_t>() + a, cur.as<uint64_t>() + a, (b - a) * 8,
+                                cudaMemcpyDeviceToDevice, t.stream));
+        continue;
+      }
+      size_t need = 0;
+      SF_CUDA(cub::DeviceMerge::MergeKeys(nullptr, need, cur.as<uint64_t>() + a, (int)(b - a),
+                                          cur.as<uint64_t>() + b, (int)(c - b), nxt.as<uint64_t>() + a,
+                                          cuda::std::less<uint64_t>{}, t.stream));
+      if (need > tmp_bytes) {
+        tmp.alloc(need + 16);
+        tmp_bytes = need;
+      }
+      SF_CUDA(cub::DeviceMerge::MergeKeys(tmp.p, need, cur.as<uint64_t>() + a, (int)(b - a),
+                                          cur.as<uint64_t>() + b, (int)(c - b), nxt.as<uint64_t>() + a,
+                                          cuda::std::less<uint64_t>{}, t.stream));
+      count_launch(2);
+    }
+    std::swap(cur, nxt);
+  }
+  keys_out = std::move(nxt);  // n * 8 bytes, reused for the split keys
+  pos_out.alloc(n * 4 + 16);
+  split_key_kernel<<<grid_for(n), 256, 0, t.stream>>>(cur.as<uint64_t>(), n, t.pre_pb, keys_out.as<uint64_t>(),
+                                                      pos_out.as<uint32_t>());
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
 // Matricized sort of the whole tensor for `mode`. Returns sorted keys + positions.
 static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_out) {
+  if (t.have_pre[mode]) return presort_finish(t, mode, keys_out, pos_out);
   const uint64_t n = t.nnz;
   const int s = secondary_mode(t, mode);
   const uint64_t Is = t.dims[s];
@@ -269,6 +392,17 @@ __global__ void build_aos_kernel(AosParams a, uint64_t n) {
     for (int m = 0; m < a.nmodes; ++m) r[m] = a.ind[m][e];
     r[a.nmodes] = __float_as_uint(a.val[e]);
   }
+}
+
+static void aos_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t st) {
+  AosParams p{};
+  for (int m = 0; m < t.nmodes; ++m) p.ind[m] = t.ind[m].as<uint32_t>() + a;
+  p.val = t.val.as<float>() + a;
+  p.aos = t.aos.as<uint32_t>() + a * (uint64_t)t.aos_words;
+  p.nmodes = t.nmodes;
+  p.W = t.aos_words;
+  build_aos_kernel<<<grid_for(len), 256, 0, st>>>(p, len);
+  count_launch();
 }
 
 template <int W>

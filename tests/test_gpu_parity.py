@@ -241,3 +241,33 @@ def test_generic_paths_and_degenerate_dims(cuda_device, dims, R):
         Yo, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
         assert np.max(S) < 2 ** 24
         assert np.array_equal(Y[n].astype(np.float64), Yo), n
+
+
+@pytest.mark.parametrize("segments,streams", [(2, 2), (7, 3), (16, 4)])
+def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
+    """A8 upload || presort: per-segment sorted runs merged at the first plan give the same
+    matricized order, features, chunks and Y as the full sort (oracle/plan.py ==)."""
+    dims = (300, 41, 530)
+    inds, vals = synth.gen_coo(dims, 25013, 12, zipf=(1.0, 0.5, 0.8))  # ragged segments
+    facs = synth.gen_factors(dims, 16, 13, "signed")
+    ti = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    tv = torch.from_numpy(vals).pin_memory()
+    tf = [G.dev_f(f) for f in facs]
+    for flag in ("1", "0"):
+        monkeypatch.setenv("SF_PRESORT", flag)
+        with sf.Tensor(dims, ti, tv, segments=segments, streams=streams) as t:
+            for n in range(3):
+                others = [m for m in range(3) if m != n]
+                L = sf.Launch.make(kernel=FRAG, chunk_nnz=100, staged={others[0]: 13})
+                t.set_launch(n, 16, L)  # first plan of the mode: consumes the merged runs
+                f = t.features(n)
+                of = oplan.features(dims, inds, n)
+                for k in ("num_slices", "num_fibers", "max_nnz_per_slice", "max_nnz_per_fiber"):
+                    assert f[k] == of[k], (flag, k)
+                perm, chunks = t.plan_export(n, 16)
+                ref = oplan.plan_order(dims, inds, n, (others[0],), {others[0]: 13})
+                assert np.array_equal(perm.astype(np.int64), ref), (flag, n)
+                y = torch.empty((dims[n], 16), device="cuda:0")
+                t.mttkrp(n, tf, y)
+                torch.cuda.synchronize()
+                G.assert_parity(y.cpu().numpy(), dims, inds, vals, facs, 16, n)
