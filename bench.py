@@ -249,7 +249,8 @@ def main():
         plan_ms[n] = T.plan_info(n, R)["plan_ms"]
     infos = {n: T.plan_info(n, R) for n in range(N)}
     outs = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
-    exch = sfdist.BoundaryExchange(world, rank, R, dev, host_staging=same_gpu) if world > 1 else None
+    # one boundary exchange per step for all modes (a single all_gather, dist.StepExchange)
+    exch = sfdist.StepExchange(world, rank, R, dev, host_staging=same_gpu) if world > 1 else None
 
     def max_over_ranks(x):
         t = torch.tensor([x], dtype=torch.float64, device="cpu" if same_gpu else dev)
@@ -263,8 +264,8 @@ def main():
             T.mttkrp(n, d_facs, outs[n], stream=stream)
             if ev is not None:
                 ev[n][1].record(stream)
-            if exch is not None:
-                exch.combine(outs[n], infos[n]["row_begin"], infos[n]["row_end"], stream)
+        if exch is not None:
+            exch.combine([(outs[n], infos[n]["row_begin"], infos[n]["row_end"]) for n in range(N)], stream)
 
     for _ in range(args.warmup):
         step()
@@ -349,13 +350,14 @@ def main():
                     else:
                         T2.plan(n, R)
                 inf = {n: T2.plan_info(n, R) for n in range(N)}
+                os_ = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
                 for n in range(N):
-                    o = torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev)
-                    T2.mttkrp(n, df, o, stream=stream)
-                    if exch is not None:
-                        exch.combine(o, inf[n]["row_begin"], inf[n]["row_end"], stream)
-                    with torch.cuda.stream(stream):
-                        h_out[n].copy_(o, non_blocking=True)
+                    T2.mttkrp(n, df, os_[n], stream=stream)
+                if exch is not None:
+                    exch.combine([(os_[n], inf[n]["row_begin"], inf[n]["row_end"]) for n in range(N)], stream)
+                with torch.cuda.stream(stream):
+                    for n in range(N):
+                        h_out[n].copy_(os_[n], non_blocking=True)
                 torch.cuda.synchronize(dev)
 
         e2e_step()  # warm-up

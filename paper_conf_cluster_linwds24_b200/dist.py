@@ -113,6 +113,57 @@ class BoundaryExchange:
         return Y
 
 
+class StepExchange:
+    """Steps 1-4 for several outputs at once (e.g. every mode of a CP-ALS sweep / bench step)
+    with ONE all_gather: item i's packets sit at [src][i][slot] of the gathered buffer, so a
+    step pays one collective latency instead of one per mode.  Items share the rank R."""
+
+    def __init__(self, world, rank, R, device, rows_op=None, group=None, host_staging=False):
+        self.ex = BoundaryExchange(world, rank, R, device, rows_op=rows_op, group=group,
+                                   host_staging=host_staging)
+        self._cache = {}
+
+    def _layout(self, keys):
+        if keys not in self._cache:
+            ex, W, K = self.ex, self.ex.world, len(keys)
+            per = []
+            for i, (rb, re_) in enumerate(keys):
+                pack, _, zero, ranges = ex._maps(rb, re_)
+                _, add_src = owner_maps(ranges)
+                tgt = [-1] * (2 * W * K)
+                for row, src, slot in add_src[ex.rank]:
+                    tgt[(src * K + i) * 2 + slot] = row
+                per.append((pack, zero, torch.tensor(tgt, dtype=torch.int64, device=ex.device)))
+            send = torch.empty((K * 2, ex.R), dtype=torch.float32, device=ex.device)
+            recv = torch.empty((W * K * 2, ex.R), dtype=torch.float32, device=ex.device)
+            self._cache[keys] = (per, send, recv, list(recv.view(W, K * 2, ex.R).unbind(0)))
+        return self._cache[keys]
+
+    def combine(self, items, stream=None):
+        """items: [(Y, row_begin, row_end), ...]; every Y ends row-sharded (see module doc)."""
+        ex = self.ex
+        keys = tuple((int(rb), int(re_)) for _, rb, re_ in items)
+        per, send, recv, recv_list = self._layout(keys)
+        cuda = any(Y.is_cuda for Y, _, _ in items)
+        ctx = torch.cuda.stream(stream) if (stream is not None and cuda) else _null()
+        with ctx:
+            for i, (Y, _, _) in enumerate(items):
+                ex.rows_op(Y, per[i][0], send[2 * i:2 * i + 2], 0, stream)
+            if ex.host_staging:
+                if cuda:
+                    torch.cuda.current_stream().synchronize()
+                hs = send.cpu()
+                hr = [torch.empty_like(hs) for _ in range(ex.world)]
+                dist.all_gather(hr, hs, group=ex.group)
+                recv.copy_(torch.cat(hr, 0))
+            else:
+                dist.all_gather(recv_list, send, group=ex.group)
+            for i, (Y, _, _) in enumerate(items):
+                ex.rows_op(Y, per[i][1], None, 2, stream)
+                ex.rows_op(Y, per[i][2], recv, 1, stream)
+        return [Y for Y, _, _ in items]
+
+
 class _null:
     def __enter__(self):
         return self

@@ -14,7 +14,7 @@ import torch.multiprocessing as mp
 import oracle
 import synth
 from oracle import plan as oplan
-from paper_conf_cluster_linwds24_b200.dist import BoundaryExchange, owner_maps
+from paper_conf_cluster_linwds24_b200.dist import BoundaryExchange, StepExchange, owner_maps
 
 
 def _cpu_rows_op(Y, rows, buf, op, stream=None):
@@ -56,6 +56,19 @@ def _worker(rank, world, port, dims, nnz, R, seed, q):
         ex.combine(Yt, rb, re_)
         ex.combine  # cached maps reused on a second call
         res[n] = (Yt.numpy(), rb, re_)
+    # the same exchange for all modes at once (one all_gather per step) must agree exactly
+    items = []
+    for n in range(len(dims)):
+        perm0 = oplan.matricized_order(dims, inds, n)
+        lo, hi = oplan.shard_range(nnz, world, rank)
+        sel = perm0[lo:hi]
+        Y, _ = oracle.mttkrp(dims, [a[sel] for a in inds], vals[sel], facs, R, n, with_scale=False)
+        items.append((torch.from_numpy(Y.astype(np.float32)), res[n][1], res[n][2]))
+    sx = StepExchange(world, rank, R, torch.device("cpu"), rows_op=_cpu_rows_op)
+    for _ in range(2):  # second call: cached layout; inputs re-made so the sums stay exact
+        outs = sx.combine([(Y.clone(), rb, re_) for Y, rb, re_ in items])
+    for n in range(len(dims)):
+        assert np.array_equal(outs[n].numpy(), res[n][0]), n
     q.put((rank, res))
     dist.destroy_process_group()
 
