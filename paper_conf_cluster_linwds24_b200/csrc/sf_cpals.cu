@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <vector>
 
 #include "sf_internal.h"
@@ -53,6 +54,221 @@ __global__ void gram_kernel(const float* __restrict__ A, uint64_t I, int R, doub
     if (e >= RR) break;
     atomicAdd(&G[e], acc[q]);
   }
+}
+
+// Register-tiled Gram for R in {16, 32, 64}: the R x R output is cut into 4 x 4 blocks, one
+// per thread of a "row group" of (R/4)^2 threads; the 256 / (R/4)^2 row groups of a CTA split
+// each staged tile of TR rows.  Per row a thread does two LDS.128 and 16 FMAs (compute-bound,
+// unlike the scalar kernel above); fp32 inside a tile, folded into fp64 per tile, row groups
+// reduced in shared memory, one fp64 atomic per entry per CTA.
+template <int R>
+__global__ void __launch_bounds__(256) gram_rt_kernel(const float* __restrict__ A, uint64_t I,
+                                                      double* __restrict__ G) {
+  constexpr int TR = 128, NB = R / 4, TPG = NB * NB, NG = 256 / TPG;
+  __shared__ __align__(16) float tile[TR * R];
+  __shared__ double red[NG > 1 ? NG * 16 * TPG : 1];  // row-group partials (48 KB static at R = 32)
+  const int tid = threadIdx.x, g = tid / TPG, l = tid % TPG, bi = l / NB, bj = l % NB;
+  double acc[16];
+#pragma unroll
+  for (int q = 0; q < 16; ++q) acc[q] = 0.0;
+  const uint64_t ntiles = (I + TR - 1) / TR;
+  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+    const uint64_t r0 = tb * TR;
+    const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
+    const float4* src = reinterpret_cast<const float4*>(A + r0 * R);
+    float4* dst = reinterpret_cast<float4*>(tile);
+    for (int e = tid; e < TR * R / 4; e += 256) dst[e] = (e < rows * R / 4) ? __ldg(src + e) : make_float4(0, 0, 0, 0);
+    __syncthreads();
+    float s[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q) s[q] = 0.f;
+    for (int rr = g; rr < TR; rr += NG) {
+      const float4 a = *reinterpret_cast<const float4*>(tile + rr * R + 4 * bi);
+      const float4 b = *reinterpret_cast<const float4*>(tile + rr * R + 4 * bj);
+      const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 4; ++y) s[x * 4 + y] = fmaf(av[x], bv[y], s[x * 4 + y]);
+    }
+#pragma unroll
+    for (int q = 0; q < 16; ++q) acc[q] += (double)s[q];
+    __syncthreads();
+  }
+  if constexpr (NG > 1) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) red[(g * 16 + q) * TPG + l] = acc[q];
+    __syncthreads();
+  }
+  if (g == 0) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      double v = acc[q];
+      if constexpr (NG > 1)
+        for (int h = 1; h < NG; ++h) v += red[(h * 16 + q) * TPG + l];
+      const int x = q / 4, y = q % 4;
+      atomicAdd(&G[(4 * bi + x) * R + 4 * bj + y], v);
+    }
+  }
+}
+
+// A = M x Vinv for R in {16, 32, 64}: one thread per row, its R outputs in registers, Vinv
+// broadcast from shared memory (R / 4 LDS.128 per k for R FMAs).
+template <int R>
+__global__ void __launch_bounds__(256) rowmat_rt_kernel(const float* __restrict__ M, uint64_t I,
+                                                        const float* __restrict__ Vinv, float* __restrict__ A) {
+  __shared__ __align__(16) float V[R * R];
+  for (int e = threadIdx.x; e < R * R; e += blockDim.x) V[e] = Vinv[e];
+  __syncthreads();
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < I; i += stride) {
+    const float4* m4 = reinterpret_cast<const float4*>(M + i * R);
+    float acc[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) acc[r] = 0.f;
+#pragma unroll 2
+    for (int k4 = 0; k4 < R / 4; ++k4) {
+      const float4 mv = __ldg(m4 + k4);
+      const float mk[4] = {mv.x, mv.y, mv.z, mv.w};
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) {
+        const float4* v4 = reinterpret_cast<const float4*>(V + (4 * k4 + kk) * R);
+#pragma unroll
+        for (int c = 0; c < R / 4; ++c) {
+          const float4 v = v4[c];
+          acc[4 * c] = fmaf(mk[kk], v.x, acc[4 * c]);
+          acc[4 * c + 1] = fmaf(mk[kk], v.y, acc[4 * c + 1]);
+          acc[4 * c + 2] = fmaf(mk[kk], v.z, acc[4 * c + 2]);
+          acc[4 * c + 3] = fmaf(mk[kk], v.w, acc[4 * c + 3]);
+        }
+      }
+    }
+    float4* a4 = reinterpret_cast<float4*>(A + i * R);
+#pragma unroll
+    for (int c = 0; c < R / 4; ++c) a4[c] = make_float4(acc[4 * c], acc[4 * c + 1], acc[4 * c + 2], acc[4 * c + 3]);
+  }
+}
+
+// Alg. 1 line 5 and the Gram refresh fused (R in {16, 32, 64}): per tile of TR = 4096 / R
+// rows, M is read once into shared memory, A = M Vinv is formed in registers (4 rows x 4
+// columns per thread, rows strided by NRB so a quarter-warp's LDS.128 hit distinct banks),
+// written back through shared memory with coalesced stores, and G_n += A^T A (fp32 per
+// tile, fp64 across tiles) plus, for the fit, <M, A> are taken from the same tile: M is
+// read once and A written once (the separate kernels read A again for the Gram and M and A
+// again for the fit).
+template <int R>
+__global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restrict__ M, uint64_t I,
+                                                           const float* __restrict__ Vinv, float* __restrict__ A,
+                                                           double* __restrict__ G, double* __restrict__ dot) {
+  constexpr int NCB = R / 4, NRB = 256 / NCB, TR = 4 * NRB, LD = R + 4;  // padded row stride
+  constexpr int TPG = NCB * NCB, NG = 256 / TPG;
+  extern __shared__ __align__(16) float sm[];
+  float* Ms = sm;                 // TR x LD
+  float* As = Ms + TR * LD;       // TR x LD
+  float* Vs = As + TR * LD;       // R x R
+  const int tid = threadIdx.x;
+  for (int e = tid; e < R * R; e += 256) Vs[e] = Vinv[e];
+  const int rs = tid % NRB, cb = tid / NRB;            // A-block: rows rs + NRB*x, cols 4cb..4cb+3
+  const int g = tid / TPG, l = tid % TPG, bi = l / NCB, bj = l % NCB;  // Gram block
+  double gacc[16];
+#pragma unroll
+  for (int q = 0; q < 16; ++q) gacc[q] = 0.0;
+  double dacc = 0.0;
+  const uint64_t ntiles = (I + TR - 1) / TR;
+  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+    const uint64_t r0 = tb * TR;
+    const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
+    __syncthreads();  // previous tile's Gram reads of As are done
+    const float4* src = reinterpret_cast<const float4*>(M + r0 * R);
+    for (int e = tid; e < TR * NCB; e += 256) {
+      const int r = e / NCB, c = e % NCB;
+      const float4 v = (r < rows) ? __ldg(src + e) : make_float4(0.f, 0.f, 0.f, 0.f);
+      *reinterpret_cast<float4*>(Ms + r * LD + 4 * c) = v;
+    }
+    __syncthreads();
+    float a[4][4];
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+      for (int y = 0; y < 4; ++y) a[x][y] = 0.f;
+#pragma unroll 2
+    for (int k4 = 0; k4 < NCB; ++k4) {
+      float4 m[4], v[4];
+#pragma unroll
+      for (int x = 0; x < 4; ++x) m[x] = *reinterpret_cast<const float4*>(Ms + (rs + NRB * x) * LD + 4 * k4);
+#pragma unroll
+      for (int kk = 0; kk < 4; ++kk) v[kk] = *reinterpret_cast<const float4*>(Vs + (4 * k4 + kk) * R + 4 * cb);
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        const float mk[4] = {m[x].x, m[x].y, m[x].z, m[x].w};
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk) {
+          a[x][0] = fmaf(mk[kk], v[kk].x, a[x][0]);
+          a[x][1] = fmaf(mk[kk], v[kk].y, a[x][1]);
+          a[x][2] = fmaf(mk[kk], v[kk].z, a[x][2]);
+          a[x][3] = fmaf(mk[kk], v[kk].w, a[x][3]);
+        }
+      }
+    }
+    float dpart = 0.f;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const int r = rs + NRB * x;
+      *reinterpret_cast<float4*>(As + r * LD + 4 * cb) = make_float4(a[x][0], a[x][1], a[x][2], a[x][3]);
+      if (dot) {
+        const float4 mm = *reinterpret_cast<const float4*>(Ms + r * LD + 4 * cb);
+        dpart = fmaf(mm.x, a[x][0], fmaf(mm.y, a[x][1], fmaf(mm.z, a[x][2], fmaf(mm.w, a[x][3], dpart))));
+      }
+    }
+    dacc += (double)dpart;
+    __syncthreads();
+    float4* dst = reinterpret_cast<float4*>(A + r0 * R);
+    for (int e = tid; e < rows * NCB; e += 256) {
+      const int r = e / NCB, c = e % NCB;
+      dst[e] = *reinterpret_cast<const float4*>(As + r * LD + 4 * c);
+    }
+    float s4[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q) s4[q] = 0.f;
+    for (int rr = g; rr < rows; rr += NG) {
+      const float4 x4 = *reinterpret_cast<const float4*>(As + rr * LD + 4 * bi);
+      const float4 y4 = *reinterpret_cast<const float4*>(As + rr * LD + 4 * bj);
+      const float av[4] = {x4.x, x4.y, x4.z, x4.w}, bv[4] = {y4.x, y4.y, y4.z, y4.w};
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 4; ++y) s4[x * 4 + y] = fmaf(av[x], bv[y], s4[x * 4 + y]);
+    }
+#pragma unroll
+    for (int q = 0; q < 16; ++q) gacc[q] += (double)s4[q];
+  }
+  // reduce the NG row groups' Gram partials (shared memory reused) and the fit dot
+  __syncthreads();
+  double* red = reinterpret_cast<double*>(sm);
+  if constexpr (NG > 1) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) red[(g * 16 + q) * TPG + l] = gacc[q];
+  }
+  __syncthreads();
+  if (g == 0) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      double v = gacc[q];
+      if constexpr (NG > 1)
+        for (int h = 1; h < NG; ++h) v += red[(h * 16 + q) * TPG + l];
+      atomicAdd(&G[(4 * bi + q / 4) * R + 4 * bj + q % 4], v);
+    }
+  }
+  if (dot) {
+    for (int o = 16; o > 0; o >>= 1) dacc += __shfl_xor_sync(0xffffffffu, dacc, o);
+    if ((tid & 31) == 0) atomicAdd(dot, dacc);
+  }
+}
+
+template <int R>
+static size_t update_rt_smem() {
+  constexpr int NCB = R / 4, NRB = 256 / NCB, TR = 4 * NRB, LD = R + 4;
+  return (size_t)(2 * TR * LD + R * R) * sizeof(float);
 }
 
 // Vinv = (Hadamard_{m != n} G_m)^†, one CTA, fp64 Gauss-Jordan on [V | I].
@@ -186,8 +402,56 @@ static int grid_of(uint64_t n, int threads) {
 
 static void gram(const float* A, uint64_t I, int R, double* G, cudaStream_t s) {
   SF_CUDA(cudaMemsetAsync(G, 0, sizeof(double) * R * R, s));
-  const uint64_t tiles = (I + 63) / 64;
-  gram_kernel<<<grid_of(tiles, 1), 256, 64 * R * sizeof(float), s>>>(A, I, R, G);
+  const int rt_grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((I + 127) / 128, 148ull * 4));
+  switch (R) {  // register-tiled kernels; the scalar one for other ranks
+    case 16: gram_rt_kernel<16><<<rt_grid, 256, 0, s>>>(A, I, G); break;
+    case 32: gram_rt_kernel<32><<<rt_grid, 256, 0, s>>>(A, I, G); break;
+    case 64: gram_rt_kernel<64><<<rt_grid, 256, 0, s>>>(A, I, G); break;
+    default: {
+      const uint64_t tiles = (I + 63) / 64;
+      gram_kernel<<<grid_of(tiles, 1), 256, 64 * R * sizeof(float), s>>>(A, I, R, G);
+    }
+  }
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+// A = M Vinv, G = A^T A, and (dot != nullptr) *dot += <M, A>; false: rank not specialised.
+template <int R>
+static void update_one(const float* M, uint64_t I, const float* Vinv, float* A, double* G, double* dot,
+                       cudaStream_t s) {
+  const size_t smem = update_rt_smem<R>();
+  SF_CUDA(cudaFuncSetAttribute(update_rt_kernel<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  constexpr uint64_t TR = 4096 / R;
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((I + TR - 1) / TR, 148ull * 2));
+  update_rt_kernel<R><<<grid, 256, smem, s>>>(M, I, Vinv, A, G, dot);
+}
+
+static bool update_fused(const float* M, uint64_t I, int R, const float* Vinv, float* A, double* G, double* dot,
+                         cudaStream_t s) {
+  const char* env = std::getenv("SF_CPALS_FUSED");  // "0": separate kernels (A/B)
+  if (env && env[0] == '0') return false;
+  SF_CUDA(cudaMemsetAsync(G, 0, sizeof(double) * R * R, s));
+  switch (R) {
+    case 16: update_one<16>(M, I, Vinv, A, G, dot, s); break;
+    case 32: update_one<32>(M, I, Vinv, A, G, dot, s); break;
+    case 64: update_one<64>(M, I, Vinv, A, G, dot, s); break;
+    default: return false;
+  }
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+  return true;
+}
+
+static void rowmat(const float* M, uint64_t I, int R, const float* Vinv, float* A, cudaStream_t s) {
+  const int g = (int)std::max<uint64_t>(1, std::min<uint64_t>((I + 255) / 256, 148ull * 8));
+  switch (R) {
+    case 16: rowmat_rt_kernel<16><<<g, 256, 0, s>>>(M, I, Vinv, A); break;
+    case 32: rowmat_rt_kernel<32><<<g, 256, 0, s>>>(M, I, Vinv, A); break;
+    case 64: rowmat_rt_kernel<64><<<g, 256, 0, s>>>(M, I, Vinv, A); break;
+    default:
+      rowmat_kernel<<<grid_of(I * (uint64_t)R, 256), 256, (size_t)R * R * sizeof(float), s>>>(M, I, R, Vinv, A);
+  }
   count_launch();
   SF_CUDA(cudaGetLastError());
 }
@@ -210,26 +474,34 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
   SF_CUDA(cudaMemcpyAsync(&normX2, scal.p, sizeof(double), cudaMemcpyDeviceToHost, s));
   SF_CUDA(cudaStreamSynchronize(s));
   const float* const* cf = const_cast<const float* const*>(factors);
+  // [V | I] in fp64: 64 KB at R = 64, above the 48 KB default dynamic shared-memory limit
+  const size_t pinv_smem = (size_t)R * 2 * R * sizeof(double);
+  SF_CUDA(cudaFuncSetAttribute(pinv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pinv_smem));
   double prev = -1.0;
   int k = 0;
   for (; k < iters; ++k) {
     for (int n = 0; n < N; ++n) {
-      pinv_kernel<<<1, 256, (size_t)R * 2 * R * sizeof(double), s>>>(dG, N, n, R, Vinv64.as<double>(),
-                                                                    Vinv32.as<float>());
+      pinv_kernel<<<1, 256, pinv_smem, s>>>(dG, N, n, R, Vinv64.as<double>(), Vinv32.as<float>());
       count_launch();
+      SF_CUDA(cudaGetLastError());
       launch_mttkrp(t, *plans[n], cf, M.as<float>(), s);
-      rowmat_kernel<<<grid_of(t.dims[n] * (uint64_t)R, 256), 256, (size_t)R * R * sizeof(float), s>>>(
-          M.as<float>(), t.dims[n], R, Vinv32.as<float>(), factors[n]);
-      count_launch();
-      gram(factors[n], t.dims[n], R, dG + (size_t)n * R * R, s);
+      // fit after the sweep needs <M_N, A_N> of the last mode
+      double* dot = (n == N - 1) ? scal.as<double>() + 1 : nullptr;
+      if (n == N - 1) SF_CUDA(cudaMemsetAsync(scal.as<double>() + 1, 0, 2 * sizeof(double), s));
+      if (!update_fused(M.as<float>(), t.dims[n], R, Vinv32.as<float>(), factors[n], dG + (size_t)n * R * R, dot,
+                        s)) {
+        rowmat(M.as<float>(), t.dims[n], R, Vinv32.as<float>(), factors[n], s);
+        gram(factors[n], t.dims[n], R, dG + (size_t)n * R * R, s);
+        if (dot) {
+          const uint64_t nl = t.dims[n] * (uint64_t)R;
+          dot_kernel<<<grid_of(nl, 256), 256, 0, s>>>(M.as<float>(), factors[n], nl, dot);
+          count_launch();
+        }
+      }
       SF_CUDA(cudaGetLastError());
     }
-    // fit after the sweep: M holds the last mode's MTTKRP, factors[N-1] its update
-    SF_CUDA(cudaMemsetAsync(scal.as<double>() + 1, 0, 2 * sizeof(double), s));
-    const uint64_t nl = t.dims[N - 1] * (uint64_t)R;
-    dot_kernel<<<grid_of(nl, 256), 256, 0, s>>>(M.as<float>(), factors[N - 1], nl, scal.as<double>() + 1);
     model_norm_kernel<<<1, 256, 0, s>>>(dG, N, R, scal.as<double>() + 2);
-    count_launch(2);
+    count_launch();
     double h[3];
     SF_CUDA(cudaMemcpyAsync(h, scal.p, 3 * sizeof(double), cudaMemcpyDeviceToHost, s));
     SF_CUDA(cudaStreamSynchronize(s));

@@ -20,7 +20,7 @@ def _lowrank_coo(rng, dims, R, density, noise=0.01):
     return [i.astype(np.uint32) for i in idx], X.astype(np.float32)
 
 
-@pytest.mark.parametrize("R", [8, 16, 32])
+@pytest.mark.parametrize("R", [8, 16, 32, 64])
 def test_cpals_matches_oracle(cuda_device, R):
     rng = np.random.default_rng(R)
     dims = (60, 50, 40)
