@@ -20,15 +20,37 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 
+def random_configs(count, seed):
+    """Held-out check of the selection rule: random tensors (never a BASELINE/Table III shape)
+    large enough that gathered factors exceed L2."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    out = []
+    for k in range(count):
+        N = int(rng.choice([3, 3, 4]))
+        R = int(rng.choice([16, 32]))
+        nnz = int(10 ** rng.uniform(7.5, 8.2))
+        dims = [int(10 ** rng.uniform(4.0, 7.3)) for _ in range(N)]
+        zipf = [float(rng.choice([0.0, 0.5, 0.8, 1.0, 1.2])) for _ in range(N)]
+        out.append(synth.Config(f"rand{k}", tuple(dims), nnz, R, tuple(zipf), 40000000 + k, 40001000 + k,
+                                "random held-out tensor (tools/l2tile_study.py)"))
+    return out
+
+
 def main():
     import torch
 
     import paper_conf_cluster_linwds24_b200 as sf
     names = sys.argv[1].split(",") if len(sys.argv) > 1 else ["nell1"]
+    if names[0].startswith("random"):  # random:COUNT:SEED
+        _, cnt, sd = (names[0].split(":") + ["8", "1"])[:3]
+        cfgs = random_configs(int(cnt), int(sd))
+    else:
+        cfgs = [synth.CONFIGS[nm] for nm in names]
     min_mb = float(os.environ.get("MIN_MB", "24"))
     block_mb = [float(x) for x in os.environ.get("BLOCK_MB", "16,32,64").split(",")]
-    for name in names:
-        cfg = synth.CONFIGS[name]
+    for cfg in cfgs:
+        name = cfg.name
         d_inds, d_vals = synth.config_tensor_device(cfg)
         facs = synth.config_factors_device(cfg)
         R = cfg.rank
@@ -50,12 +72,20 @@ def main():
 
         for n in range(cfg.nmodes):
             out = torch.empty((cfg.dims[n], R), dtype=torch.float32, device="cuda")
+            # the selector without the L2-tile rule is the reference ("auto"); with it: "rule"
+            os.environ["SF_L2_TILES"] = "0"
             T.plan(n, R)
             auto = timed(n, out)
             ref = out.clone()
             info = T.plan_info(n, R)
-            print(json.dumps({"config": name, "mode": n, "launch": "auto", "ms": auto,
-                              "picked": info["launch"]}), flush=True)
+            print(json.dumps({"config": name, "dims": list(cfg.dims), "nnz": cfg.nnz, "rank": R, "mode": n,
+                              "launch": "auto", "ms": auto, "picked": info["launch"]}), flush=True)
+            T.plan_release(n, R)
+            os.environ["SF_L2_TILES"] = "1"
+            T.plan(n, R)
+            ms = timed(n, out)
+            print(json.dumps({"config": name, "mode": n, "launch": "rule", "ms": ms, "speedup_vs_auto": auto / ms,
+                              "picked": T.plan_info(n, R)["launch"]}), flush=True)
             T.plan_release(n, R)
             for m in range(cfg.nmodes):
                 fac_mb = cfg.dims[m] * R * 4 / 2**20

@@ -67,6 +67,29 @@ __global__ void __launch_bounds__(512) k(const float4* __restrict__ gtab, float*
         acc.x += u.x; acc.y += u.y; acc.z += u.z; acc.w += u.w;
         acc2.x += w.x; acc2.y += w.y; acc2.z += w.z; acc2.w += w.w;
       }
+    } else if (MODE >= 10) {  // L2 row, load variants (p applies)
+      if (take) {
+        const uint32_t grow = (h >> 9) & 32767u;
+        const float4* p = gtab + (size_t)grow * 8 + 2 * lig;
+        float4 u, w;
+        if (MODE == 10)
+          asm volatile("ld.global.cg.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                       : "=f"(u.x), "=f"(u.y), "=f"(u.z), "=f"(u.w), "=f"(w.x), "=f"(w.y), "=f"(w.z), "=f"(w.w) : "l"(p));
+        else if (MODE == 11)
+          asm volatile("ld.global.nc.L1::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                       : "=f"(u.x), "=f"(u.y), "=f"(u.z), "=f"(u.w), "=f"(w.x), "=f"(w.y), "=f"(w.z), "=f"(w.w) : "l"(p));
+        else if (MODE == 12)
+          asm volatile("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                       : "=f"(u.x), "=f"(u.y), "=f"(u.z), "=f"(u.w), "=f"(w.x), "=f"(w.y), "=f"(w.z), "=f"(w.w) : "l"(p));
+        else {  // 13: two 128-bit no_allocate loads
+          asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                       : "=f"(u.x), "=f"(u.y), "=f"(u.z), "=f"(u.w) : "l"(p));
+          asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                       : "=f"(w.x), "=f"(w.y), "=f"(w.z), "=f"(w.w) : "l"(p + 1));
+        }
+        acc.x += u.x; acc.y += u.y; acc.z += u.z; acc.w += u.w;
+        acc2.x += w.x; acc2.y += w.y; acc2.z += w.z; acc2.w += w.w;
+      }
     } else if (MODE == 2) {
       const uint32_t r = (it * 8 + group) & 2047u;
       const float4 u = s[r];
@@ -110,6 +133,11 @@ int main() {
   for (double p : {1.0, 0.75, 0.58, 0.5, 0.25, 0.0}) run(k<0, 8>, "smem row G=8 (1xLDS.128)", p, 4);
   for (double p : {1.0, 0.75, 0.58, 0.5, 0.25, 0.0}) run(k<1, 4>, "L2 row G=4 (LDG.256)", p, 8);
   run(k<4, 4>, "L1 row G=4 (LDG.256 L1 hit)", 1.0, 8);
+  run(k<1, 4>, "L2 row .nc.L1::no_allocate", 1.0, 8);
+  run(k<10, 4>, "L2 row .cg v8", 1.0, 8);
+  run(k<11, 4>, "L2 row .nc.L1::evict_first", 1.0, 8);
+  run(k<12, 4>, "L2 row .nc (default)", 1.0, 8);
+  run(k<13, 4>, "L2 row 2x v4 no_allocate", 1.0, 8);
   ctas = 37 * 4;
   run(k<1, 4>, "L2 row G=4, 37 SMs", 1.0, 8);
   ctas = 74 * 4;
