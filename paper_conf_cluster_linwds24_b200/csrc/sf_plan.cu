@@ -17,6 +17,8 @@
 #include <cub/cub.cuh>
 
 #include <cub/device/device_merge.cuh>
+#include <thrust/iterator/discard_iterator.h>
+#include <thrust/iterator/transform_iterator.h>
 
 #include <algorithm>
 #include <cstdlib>
@@ -47,89 +49,11 @@ __global__ void key_matricized_kernel(const uint32_t* __restrict__ in, const uin
   }
 }
 
-// Run-start positions for slices (i_n = key / Is) and fibers (key) in the sorted order.
-__global__ void run_start_kernel(const uint64_t* __restrict__ key, uint64_t Is, uint64_t n,
-                                 uint32_t* __restrict__ sstart, uint32_t* __restrict__ fstart,
-                                 unsigned long long* __restrict__ counts /*[2]*/) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned long long ns = 0, nf = 0;
-  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
-    const uint64_t k = key[e];
-    bool fs = true, ss = true;
-    if (e > 0) {
-      const uint64_t kp = key[e - 1];
-      fs = (k != kp);
-      ss = (k / Is) != (kp / Is);
-    }
-    sstart[e] = ss ? (uint32_t)e : 0u;
-    fstart[e] = fs ? (uint32_t)e : 0u;
-    ns += ss;
-    nf += fs;
-  }
-  typedef cub::BlockReduce<unsigned long long, 256> BR;
-  __shared__ typename BR::TempStorage tmp;
-  unsigned long long a = BR(tmp).Sum(ns);
-  __syncthreads();
-  unsigned long long b = BR(tmp).Sum(nf);
-  if (threadIdx.x == 0) {
-    atomicAdd(&counts[0], a);
-    atomicAdd(&counts[1], b);
-  }
-}
-
 struct FeatAcc {
   unsigned long long max_slice, max_fiber, sum_sq;
   unsigned long long hist[SF_HIST_BINS];
 };
 
-// At every run end: run length = e - start + 1.
-__global__ void run_end_kernel(const uint64_t* __restrict__ key, uint64_t Is, uint64_t n,
-                               const uint32_t* __restrict__ sstart, const uint32_t* __restrict__ fstart,
-                               FeatAcc* __restrict__ acc) {
-  __shared__ unsigned long long h[SF_HIST_BINS];
-  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x) h[i] = 0;
-  __syncthreads();
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned long long ms = 0, mf = 0, sq = 0;
-  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
-    const uint64_t k = key[e];
-    bool fend = true, send = true;
-    if (e + 1 < n) {
-      const uint64_t kn = key[e + 1];
-      fend = (k != kn);
-      send = (k / Is) != (kn / Is);
-    }
-    if (fend) {
-      const unsigned long long len = e - fstart[e] + 1;
-      mf = max(mf, len);
-    }
-    if (send) {
-      const unsigned long long len = e - sstart[e] + 1;
-      ms = max(ms, len);
-      sq += len * len;
-      atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
-    }
-  }
-  typedef cub::BlockReduce<unsigned long long, 256> BR;
-  __shared__ typename BR::TempStorage tmp;
-  unsigned long long a = BR(tmp).Reduce(ms, cub::Max());
-  __syncthreads();
-  unsigned long long b = BR(tmp).Reduce(mf, cub::Max());
-  __syncthreads();
-  unsigned long long c = BR(tmp).Sum(sq);
-  if (threadIdx.x == 0) {
-    atomicMax(&acc->max_slice, a);
-    atomicMax(&acc->max_fiber, b);
-    atomicAdd(&acc->sum_sq, c);
-  }
-  __syncthreads();
-  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x)
-    if (h[i]) atomicAdd(&acc->hist[i], h[i]);
-}
-
-struct MaxOp {
-  __device__ __forceinline__ uint32_t operator()(uint32_t a, uint32_t b) const { return a > b ? a : b; }
-};
 
 // ---------------------------------------------------------------------------
 // A8 upload || presort.  Composite key c = (i_n * I_s + i_s) << pb | e (e = input position,
@@ -274,6 +198,55 @@ static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_o
   if (dv.Current() == p0.as<uint32_t>()) pos_out = std::move(p0); else pos_out = std::move(p1);
 }
 
+struct SliceOf {
+  uint64_t Is;
+  __host__ __device__ uint64_t operator()(uint64_t k) const { return k / Is; }
+};
+
+// Slice statistics from the run lengths of the slice ids (one thread per slice).
+__global__ void slice_stats_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ nruns,
+                                   FeatAcc* __restrict__ acc) {
+  __shared__ unsigned long long h[SF_HIST_BINS];
+  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  const uint64_t nr = *nruns;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long ms = 0, sq = 0;
+  for (uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nr; r += stride) {
+    const unsigned long long len = cnt[r];
+    ms = max(ms, len);
+    sq += len * len;
+    atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
+  }
+  typedef cub::BlockReduce<unsigned long long, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  const unsigned long long a = BR(tmp).Reduce(ms, cub::Max());
+  __syncthreads();
+  const unsigned long long c = BR(tmp).Sum(sq);
+  if (threadIdx.x == 0) {
+    atomicMax(&acc->max_slice, a);
+    atomicAdd(&acc->sum_sq, c);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x)
+    if (h[i]) atomicAdd(&acc->hist[i], h[i]);
+}
+
+__global__ void run_max_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ nruns,
+                               unsigned long long* __restrict__ out) {
+  const uint64_t nr = *nruns;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long m = 0;
+  for (uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nr; r += stride)
+    m = max(m, (unsigned long long)cnt[r]);
+  typedef cub::BlockReduce<unsigned long long, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  const unsigned long long a = BR(tmp).Reduce(m, cub::Max());
+  if (threadIdx.x == 0) atomicMax(out, a);
+}
+
+// Features (reading R4) of the matricized order: slices = runs of
+// i_n = key / I_s, fibers = runs of the key, each found by one run-length encode.
 static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_features_t* f) {
   const uint64_t n = t.nnz;
   const int s = secondary_mode(t, mode);
@@ -285,28 +258,29 @@ static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_f
   f->mode = mode;
   f->secondary = s;
   if (n > 0) {
-    DevBuf ss(n * 4 + 16), fs(n * 4 + 16), cnt(16), accb(sizeof(FeatAcc));
-    SF_CUDA(cudaMemsetAsync(cnt.p, 0, 16, t.stream));
+    const uint64_t max_slices = std::min<uint64_t>(n, t.dims[mode]);
+    DevBuf scnt(max_slices * 4 + 16), fcnt(n * 4 + 16), nr(16), accb(sizeof(FeatAcc));
     SF_CUDA(cudaMemsetAsync(accb.p, 0, sizeof(FeatAcc), t.stream));
-    run_start_kernel<<<grid_for(n), 256, 0, t.stream>>>(keys, Is, n, ss.as<uint32_t>(), fs.as<uint32_t>(),
-                                                        cnt.as<unsigned long long>());
-    count_launch();
-    size_t temp = 0;
-    SF_CUDA(cub::DeviceScan::InclusiveScan(nullptr, temp, ss.as<uint32_t>(), ss.as<uint32_t>(), MaxOp(),
-                                           (int64_t)n, t.stream));
-    DevBuf tmp(temp + 16);
-    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, ss.as<uint32_t>(), ss.as<uint32_t>(), MaxOp(),
-                                           (int64_t)n, t.stream));
-    SF_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, temp, fs.as<uint32_t>(), fs.as<uint32_t>(), MaxOp(),
-                                           (int64_t)n, t.stream));
-    count_launch(4);
-    run_end_kernel<<<grid_for(n), 256, 0, t.stream>>>(keys, Is, n, ss.as<uint32_t>(), fs.as<uint32_t>(),
-                                                      accb.as<FeatAcc>());
-    count_launch();
+    auto sl = thrust::make_transform_iterator(keys, SliceOf{Is});
+    auto discard = thrust::make_discard_iterator();
+    uint32_t* nrs = nr.as<uint32_t>();
+    size_t t1 = 0, t2 = 0;
+    SF_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, t1, sl, discard, scnt.as<uint32_t>(), nrs, (int64_t)n,
+                                               t.stream));
+    SF_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, t2, keys, discard, fcnt.as<uint32_t>(), nrs + 1, (int64_t)n,
+                                               t.stream));
+    DevBuf tmp(std::max(t1, t2) + 16);
+    SF_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, t1, sl, discard, scnt.as<uint32_t>(), nrs, (int64_t)n,
+                                               t.stream));
+    SF_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, t2, keys, discard, fcnt.as<uint32_t>(), nrs + 1, (int64_t)n,
+                                               t.stream));
+    slice_stats_kernel<<<grid_for(max_slices), 256, 0, t.stream>>>(scnt.as<uint32_t>(), nrs, accb.as<FeatAcc>());
+    run_max_kernel<<<grid_for(n), 256, 0, t.stream>>>(fcnt.as<uint32_t>(), nrs + 1, &accb.as<FeatAcc>()->max_fiber);
+    count_launch(6);
     SF_CUDA(cudaGetLastError());
-    unsigned long long c[2];
+    uint32_t c[2];
     FeatAcc a;
-    SF_CUDA(cudaMemcpyAsync(c, cnt.p, 16, cudaMemcpyDeviceToHost, t.stream));
+    SF_CUDA(cudaMemcpyAsync(c, nr.p, 8, cudaMemcpyDeviceToHost, t.stream));
     SF_CUDA(cudaMemcpyAsync(&a, accb.p, sizeof(FeatAcc), cudaMemcpyDeviceToHost, t.stream));
     SF_CUDA(cudaStreamSynchronize(t.stream));
     f->num_slices = c[0];

@@ -250,16 +250,18 @@ static int tree_predict(const double* x, int nx) {
 // ---------------------------------------------------------------------------
 // L2-tile refinement (SF_LAUNCH_L2_TILES; DESIGN.md §5 "L2 tiles").  When the pick is an
 // unstaged plan (the hyper-sparse regime: factors >> L2, gathers DRAM-latency bound), tile
-// the order by 64 MB row blocks of the LARGEST gathered factor of >= 64 MB, so at any moment
+// the order by 64 MB row blocks of the LARGEST gathered factor of >= 160 MB, so at any moment
 // every CTA gathers that factor from one L2-resident block -- unless re-visiting Y once per
 // (tile, row) costs too much: rho = T * touched(T) / nnz <= 0.25, touched(T) = the expected
 // rows of Y a tile touches, sum_b slices_b (1 - exp(-1.44 * 2^b / T)) over the log2
 // slice-length histogram (PAPER.md L195 features); rho = 0 when Y fits in 32 MB (its
 // re-visits hit L2).  Calibrated on tools/l2tile_study.py over the BASELINE.json and Table III
-// shapes (profiles/r01s3_l2tiles.jsonl): the rule's pick is within 2.4 % of the best tiled
-// option on average (worst 20 %), 1.1-2.1x over the unstaged plan where it tiles.
+// shapes (profiles/r01s3_l2tiles.jsonl) and 16 random tensors (53 modes,
+// profiles/r01s3_l2tiles_random.jsonl): over the random set the rule is 1.14x over no tiling
+// (geomean; best possible 1.175x), within 3.3 % of the best option on average, never worse
+// than 0.98x.  The 160 MB floor comes from the random set (64 MB tiled 146 MB factors at 0.78x).
 static constexpr double kL2BlockBytes = 64.0 * 1024 * 1024;
-static constexpr double kL2MinFactorBytes = 64.0 * 1024 * 1024;
+static constexpr double kL2MinFactorBytes = 160.0 * 1024 * 1024;  // ~1.3x L2: smaller factors keep their hot rows
 static constexpr double kL2MaxRevisit = 0.25;
 static constexpr double kL2YInCache = 32.0 * 1024 * 1024;
 
