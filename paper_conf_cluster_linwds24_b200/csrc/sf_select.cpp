@@ -208,6 +208,13 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out) {
   add(g[k - 1], 256, 0);                  // 4 stage largest gathered mode, 256-row blocks
   add(g[k - 1], 512, 0);                  // 5                              512-row blocks
   add(k >= 3 ? g[1] : g[0], 256, 0);      // 6 stage middle gathered mode (4-way), 256
+  // L2-tiled classes (SF_LAUNCH_L2_TILES, DESIGN.md §5 "L2 tiles"): blocks of a gathered factor
+  // swept by every CTA in tile order; a factor smaller than its block degenerates to class 1
+  const double RB = 4.0 * rank;
+  auto rows_for = [&](double bytes) { return (uint32_t)std::max(1.0, bytes / RB); };
+  add(g[k - 1], rows_for(64.0 * 1024 * 1024), SF_LAUNCH_L2_TILES);              // 7 largest, 64 MB
+  add(k >= 2 ? g[k - 2] : g[k - 1], rows_for(64.0 * 1024 * 1024), SF_LAUNCH_L2_TILES);  // 8 2nd largest
+  add(g[k - 1], rows_for(16.0 * 1024 * 1024), SF_LAUNCH_L2_TILES);              // 9 largest, 16 MB
   return n;
 }
 
@@ -215,6 +222,7 @@ struct TreeModel {
   std::vector<int32_t> feature, left, right, value;
   std::vector<double> threshold;
   int nfeat = 0;
+  bool l2_classes = false;  // trained with the L2-tiled classes (7-9): no hand rule on top
 };
 static TreeModel g_model;
 static bool g_have_model = false;
@@ -231,6 +239,9 @@ void set_selector_model(const int32_t* feature, const double* threshold, const i
   g_model.right.assign(right, right + n_nodes);
   g_model.value.assign(value, value + n_nodes);
   g_model.nfeat = n_features;
+  g_model.l2_classes = false;
+  for (int i = 0; i < n_nodes; ++i)
+    if (left[i] < 0 && value[i] >= 7) g_model.l2_classes = true;
   g_have_model = true;
 }
 
@@ -320,7 +331,8 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
     }
   }
   if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
-  if (l2_refine_enabled()) l2_tile_refine(t, f, mode, rank, nnz_local, l);
+  // the hand rule refines picks of a selector that cannot choose L2 tiles itself
+  if (l2_refine_enabled() && !(picked && g_model.l2_classes)) l2_tile_refine(t, f, mode, rank, nnz_local, l);
   return l;
 }
 

@@ -45,6 +45,7 @@ def time_launch(T, n, R, facs, out, L, torch, reps=4):
 
 
 args_nnz_lo, args_nnz_hi = 6.0, 7.5
+args_prefix, args_seed_base = "train", 30000000
 args_dims_log10 = (2.5, 7.2)
 
 
@@ -58,7 +59,7 @@ def random_config(rng, k):
         if np.prod([float(d) for d in dims]) >= 8.0 * nnz:
             break
     zipf = [float(rng.choice([0.0, 0.5, 0.8, 1.0, 1.2])) for _ in range(N)]
-    return dict(name=f"train{k}", dims=dims, nnz=nnz, rank=R, zipf=zipf, seed=30000000 + k)
+    return dict(name=f"{args_prefix}{k}", dims=dims, nnz=nnz, rank=R, zipf=zipf, seed=args_seed_base + k)
 
 
 def collect(args):
@@ -103,10 +104,23 @@ def load(path):
     return np.array(X), np.array(T)
 
 
+def load_many(paths):
+    """Comma-separated training files; rows with fewer candidate classes (older collections)
+    are dropped, so every sample has a time for every class."""
+    Xs, Ts = [], []
+    for p in paths.split(","):
+        X, T = load(p)
+        Xs.append(X)
+        Ts.append(T)
+    k = max(t.shape[1] for t in Ts)
+    keep = [(x, t) for x, t in zip(Xs, Ts) if t.shape[1] == k]
+    return np.concatenate([x for x, _ in keep]), np.concatenate([t for _, t in keep])
+
+
 def train(args):
     from sklearn.model_selection import KFold
     from sklearn.tree import DecisionTreeClassifier, DecisionTreeRegressor
-    X, T = load(args.data)
+    X, T = load_many(args.data)
     y = np.argmin(T, axis=1)
     best = T[np.arange(len(T)), y]
     # cross-validated quality
@@ -199,8 +213,11 @@ def main():
     ap.add_argument("--depth", type=int, default=5)
     ap.add_argument("--report", default=None)
     ap.add_argument("--configs", default="nell2,deli4d,nell1")
+    ap.add_argument("--prefix", default="train")
+    ap.add_argument("--seed-base", type=int, default=30000000)
     args = ap.parse_args()
-    global args_nnz_lo, args_nnz_hi, args_dims_log10
+    global args_nnz_lo, args_nnz_hi, args_dims_log10, args_prefix, args_seed_base
+    args_prefix, args_seed_base = args.prefix, args.seed_base
     args_nnz_lo, args_nnz_hi = (float(x) for x in args.nnz_log10.split(","))
     args_dims_log10 = tuple(float(x) for x in args.dims_log10.split(","))
     {"collect": collect, "train": train, "eval": evaluate}[args.cmd](args)
