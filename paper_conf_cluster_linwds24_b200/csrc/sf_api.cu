@@ -106,7 +106,7 @@ void DevBuf::release() {
 }
 
 size_t Plan::device_bytes() const {
-  size_t b = val.bytes + rec.bytes + rowid.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes;
+  size_t b = val.bytes + rec.bytes + rowid.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes + tile_chunk.bytes;
   for (int m = 0; m < SF_MAX_MODES; ++m) b += ind[m].bytes;
   return b;
 }

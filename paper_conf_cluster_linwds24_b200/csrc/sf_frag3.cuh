@@ -51,6 +51,9 @@ struct Frag3Params {
   float* out;
   const uint32_t* chunk_begin;        // num_chunks + 1
   const uint64_t* chunk_tile;         // num_chunks
+  const uint32_t* tile_chunk;         // num_tiles + 1: first chunk of every tile, then num_chunks
+  const uint32_t* cta_chunk;          // grid + 1: first chunk of every CTA (frag3_cta_range_kernel)
+  uint32_t num_tiles;
   uint32_t num_chunks;
   uint32_t nnz;
   int slot_mode[SF_MAX_MODES];        // gathered slot -> mode (staged slots first)
@@ -141,10 +144,19 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   // CTA range: nnz-balanced chunks [j0, j1) of the plan order, or (L2 tiles) every chunk,
   // of which each tile segment contributes its blockIdx.x-th 1/grid share.
   const bool l2t = (S == 0) && p.l2tiles;
-  const uint32_t j0 = l2t ? 0u : frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)blockIdx.x * p.nnz) / grid);
-  const uint32_t j1 = l2t ? p.num_chunks
-                          : frag3_lower_chunk(p.chunk_begin, p.num_chunks, ((uint64_t)(blockIdx.x + 1) * p.nnz) / grid);
+  const uint32_t j0 = l2t ? 0u : __ldg(p.cta_chunk + blockIdx.x);
+  const uint32_t j1 = l2t ? p.num_chunks : __ldg(p.cta_chunk + blockIdx.x + 1);
   if (j0 >= j1) return;
+  // tile of chunk j0 (tiles are walked by index from there: no per-segment search)
+  uint32_t ti = 0;
+  if (S > 0 || l2t) {
+    uint32_t lo = 0, hi = p.num_tiles;  // last tile with tile_chunk <= j0
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (__ldg(p.tile_chunk + mid) <= j0) lo = mid; else hi = mid;
+    }
+    ti = lo;
+  }
 
   if (lane == 0) {
     mbar_init(&wbar[0], 1);
@@ -169,23 +181,12 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   uint32_t seg = j0;
   while (seg < j1) {
     uint32_t seg_end = j1;
-    if (S == 0 && l2t) {  // this tile's chunks [seg, seg_end)
-      const uint64_t tile = __ldg(p.chunk_tile + seg);
-      uint32_t lo = seg + 1, hi = j1;
-      while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(p.chunk_tile + mid) == tile) lo = mid + 1; else hi = mid;
-      }
-      seg_end = lo;
+    if (S > 0 || l2t) {  // this tile's chunks inside [seg, j1)
+      seg_end = min(j1, __ldg(p.tile_chunk + ti + 1));
+      ++ti;
     }
     if constexpr (S > 0) {
       const uint64_t tile = __ldg(p.chunk_tile + seg);
-      uint32_t lo = seg + 1, hi = j1;  // first chunk with a different (larger) tile
-      while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(p.chunk_tile + mid) == tile) lo = mid + 1; else hi = mid;
-      }
-      seg_end = lo;
       uint64_t t = tile;
       uint32_t row0[S];
 #pragma unroll
@@ -448,17 +449,25 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
 
 // A5 pre-pass for owner mode: zero the rows whose run crosses a group sub-range start
 // (they receive atomic partial sums).  One thread per (CTA, group) of the frag3 launch.
+// CTA c's chunk range [cta_chunk[c], cta_chunk[c+1]): chunks whose first nonzero lies in
+// [c*nnz/G, (c+1)*nnz/G), computed once per (plan, grid) instead of by every CTA.
+static __global__ void frag3_cta_range_kernel(const uint32_t* __restrict__ cb, uint32_t num_chunks, uint32_t nnz,
+                                              uint32_t ctas, uint32_t* __restrict__ cta_chunk) {
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c <= ctas; c += gridDim.x * blockDim.x)
+    cta_chunk[c] = frag3_lower_chunk(cb, num_chunks, ((uint64_t)c * nnz) / ctas);
+}
+
 template <int R>
-__global__ void boundary_zero3_kernel(const uint32_t* __restrict__ chunk_begin, uint32_t num_chunks,
-                                      uint32_t nnz, uint32_t ctas, uint32_t groups_per_cta,
+__global__ void boundary_zero3_kernel(const uint32_t* __restrict__ chunk_begin, const uint32_t* __restrict__ cta_chunk,
+                                      uint32_t ctas, uint32_t groups_per_cta,
                                       const uint32_t* __restrict__ rec, uint32_t W, uint32_t om,
                                       float* __restrict__ out) {
   const uint64_t total = (uint64_t)ctas * groups_per_cta;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += stride) {
     const uint32_t c = (uint32_t)(t / groups_per_cta), gam = (uint32_t)(t % groups_per_cta);
-    const uint32_t j0 = frag3_lower_chunk(chunk_begin, num_chunks, ((uint64_t)c * nnz) / ctas);
-    const uint32_t j1 = frag3_lower_chunk(chunk_begin, num_chunks, ((uint64_t)(c + 1) * nnz) / ctas);
+    const uint32_t j0 = cta_chunk[c];
+    const uint32_t j1 = cta_chunk[c + 1];
     if (j0 >= j1) continue;
     const uint32_t a = chunk_begin[j0], b = chunk_begin[j1];
     const uint32_t pos = frag3_group_begin(a, b - a, gam, groups_per_cta);
@@ -547,7 +556,7 @@ int frag3_occ_one(int threads, size_t smem) {
                            cudaStream_t s) {                                                             \
     const uint64_t total = (uint64_t)ctas * groups;                                                      \
     const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((total + 255) / 256, 148 * 16));     \
-    boundary_zero3_kernel<R><<<grid, 256, 0, s>>>(fp.chunk_begin, fp.num_chunks, fp.nnz, ctas, groups,  \
+    boundary_zero3_kernel<R><<<grid, 256, 0, s>>>(fp.chunk_begin, fp.cta_chunk, ctas, groups,           \
                                                   fp.rec, fp.W, fp.out_mask, out);      \
   }
 

@@ -77,6 +77,9 @@ struct Plan {
   DevBuf perm;          // uint32 input position per sorted slot
   DevBuf chunk_begin;   // uint32[num_chunks + 1]
   DevBuf chunk_tile;    // uint64[num_chunks]
+  DevBuf tile_chunk;    // uint32[num_tiles + 1]: first chunk of every tile, then num_chunks
+  mutable DevBuf cta_chunk;  // uint32[grid + 1]: first chunk of every CTA of the last launch grid
+  mutable int cta_grid = 0;
   mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
   bool rec_packed = false;               // frag3 PK records (N >= 4, indices bit-packed)
   bool rec_compact = false;              // frag3 CR records: 8 bytes [gathered fields | run-start

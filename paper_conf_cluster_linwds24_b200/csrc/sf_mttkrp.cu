@@ -258,6 +258,8 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   fp.out = out;
   fp.chunk_begin = p.chunk_begin.as<uint32_t>();
   fp.chunk_tile = p.chunk_tile.as<uint64_t>();
+  fp.tile_chunk = p.tile_chunk.as<uint32_t>();
+  fp.num_tiles = (uint32_t)p.num_tiles;
   fp.num_chunks = (uint32_t)p.num_chunks;
   fp.nnz = (uint32_t)p.nnz_local;
   const uint32_t gpw = (uint32_t)frag_groups_per_warp(R);
@@ -290,6 +292,15 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
   grid = std::max(grid, 1);
   const uint32_t groups = (uint32_t)(threads / 32) * gpw;
+  if (p.cta_grid != grid) {  // per-CTA chunk ranges, once per (plan, grid)
+    p.cta_chunk.alloc(((size_t)grid + 1) * 4 + 16);
+    frag3_cta_range_kernel<<<(grid + 256) / 256, 256, 0, s>>>(fp.chunk_begin, fp.num_chunks, fp.nnz, (uint32_t)grid,
+                                                             p.cta_chunk.as<uint32_t>());
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+    p.cta_grid = grid;
+  }
+  fp.cta_chunk = p.cta_chunk.as<uint32_t>();
   const bool det = owner && (l.flags & SF_LAUNCH_DETERMINISTIC);
   const uint64_t nslots = 2ull * (uint64_t)grid * groups;
   if (det) {  // A7 deterministic option: carry slots instead of atomics (no pre-zero needed)

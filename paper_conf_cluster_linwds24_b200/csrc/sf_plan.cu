@@ -521,6 +521,14 @@ __global__ void chunk_count_kernel(const uint32_t* __restrict__ cnt, uint64_t nt
     nch[t] = (cnt[t] + C - 1) / C;
 }
 
+// tile_chunk[t] = first chunk of tile t (coff, or 0 for the single tile of an unstaged plan),
+// tile_chunk[nr] = nchunks: the kernel walks tiles by index instead of searching chunk_tile.
+__global__ void tile_chunk_kernel(const uint32_t* __restrict__ coff, uint32_t nr, uint64_t nchunks,
+                                  uint32_t* __restrict__ tile_chunk) {
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t <= nr; t += gridDim.x * blockDim.x)
+    tile_chunk[t] = (t == nr) ? (uint32_t)nchunks : (coff ? coff[t] : 0u);
+}
+
 // chunk j (< nchunks) of tile t (coff[t] <= j < coff[t+1], binary search over the nr tiles):
 // begins at tstart[t] + (j - coff[t]) * C, tile id uniq[t]; cbegin[nchunks] = n.  Without
 // tiles (uniq == nullptr) every chunk is j * C of tile 0.
@@ -795,7 +803,9 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       chunk_fill_kernel<<<grid_for(p.num_chunks + 1), 256, 0, t.stream>>>(
           nullptr, nullptr, nullptr, nullptr, 1, C, nl, p.num_chunks, p.chunk_begin.as<uint32_t>(),
           p.chunk_tile.as<uint64_t>());
-      count_launch();
+      p.tile_chunk.alloc(2 * 4 + 16);
+      tile_chunk_kernel<<<1, 32, 0, t.stream>>>(nullptr, 1, p.num_chunks, p.tile_chunk.as<uint32_t>());
+      count_launch(2);
     } else {
       uint64_t tiles_bound = 1;
       for (int m = 0; m < N; ++m)
@@ -833,12 +843,17 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       chunk_fill_kernel<<<grid_for(p.num_chunks + 1), 256, 0, t.stream>>>(
           uniq.as<uint64_t>(), tstart.as<uint32_t>(), coff.as<uint32_t>(), nullptr, nr, C, nl, p.num_chunks,
           p.chunk_begin.as<uint32_t>(), p.chunk_tile.as<uint64_t>());
-      count_launch();
+      p.tile_chunk.alloc(((uint64_t)nr + 1) * 4 + 16);
+      tile_chunk_kernel<<<grid_for((uint64_t)nr + 1), 256, 0, t.stream>>>(coff.as<uint32_t>(), nr, p.num_chunks,
+                                                                         p.tile_chunk.as<uint32_t>());
+      count_launch(2);
     }
     SF_CUDA(cudaGetLastError());
   } else {
     p.chunk_begin.alloc(16);
     SF_CUDA(cudaMemsetAsync(p.chunk_begin.p, 0, 16, t.stream));
+    p.tile_chunk.alloc(16);
+    SF_CUDA(cudaMemsetAsync(p.tile_chunk.p, 0, 16, t.stream));
   }
   SF_CUDA(cudaEventRecord(ev1, t.stream));
   SF_CUDA(cudaEventSynchronize(ev1));
