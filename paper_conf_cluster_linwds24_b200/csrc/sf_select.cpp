@@ -282,6 +282,8 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
       f.nnz == 0)
     return;
   const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
+  const char* env = std::getenv("SF_L2_MAX_REVISIT");  // calibration override of kL2MaxRevisit
+  const double max_revisit = env ? std::atof(env) : kL2MaxRevisit;
   int best = -1;
   double bestF = 0;
   for (int m = 0; m < t.nmodes; ++m) {
@@ -296,7 +298,7 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
         touched += (double)f.slice_hist[b] * (1.0 - std::exp(-1.44 * std::ldexp(1.0, b) / T));
       rho = T * touched / (double)f.nnz;
     }
-    if (rho > kL2MaxRevisit) continue;
+    if (rho > max_revisit) continue;
     best = m;
     bestF = F;
   }
