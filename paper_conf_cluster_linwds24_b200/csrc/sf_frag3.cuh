@@ -529,7 +529,15 @@ void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem,
   if constexpr (N == 3) {
     if (fp.W == 2) k = frag3_kernel<N, R, S, kRecCompact>;
   }
-  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // opt-in shared memory once per (device, instantiation, size): host overhead of small launches
+  static size_t smem_set[16][3] = {};
+  int dev = 0;
+  SF_CUDA(cudaGetDevice(&dev));
+  const int v = fp.W == 2 ? 2 : (fp.W == 4 && N >= 4 ? 1 : 0);
+  if (dev >= 16 || smem > smem_set[dev][v]) {
+    SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (dev < 16) smem_set[dev][v] = smem;
+  }
   k<<<grid, threads, smem, s>>>(fp);
 }
 

@@ -80,6 +80,8 @@ struct Plan {
   DevBuf tile_chunk;    // uint32[num_tiles + 1]: first chunk of every tile, then num_chunks
   mutable DevBuf cta_chunk;  // uint32[grid + 1]: first chunk of every CTA of the last launch grid
   mutable int cta_grid = 0;
+  mutable int occ = 0, occ_threads = 0;  // cached CTAs/SM of the kernel for (threads, smem)
+  mutable size_t occ_smem = 0;
   mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
   bool rec_packed = false;               // frag3 PK records (N >= 4, indices bit-packed)
   bool rec_compact = false;              // frag3 CR records: 8 bytes [gathered fields | run-start

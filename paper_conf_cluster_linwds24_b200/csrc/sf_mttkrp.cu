@@ -286,7 +286,12 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   const size_t smem = frag_smem_bytes(t, n, R, l);
   const int threads = l.block_threads;
   int per_sm = l.ctas_per_sm;
-  const int occ = frag3_occ(N, R, S, threads, smem);
+  if (p.occ_threads != threads || p.occ_smem != smem) {  // occupancy query once per plan launch shape
+    p.occ = frag3_occ(N, R, S, threads, smem);
+    p.occ_threads = threads;
+    p.occ_smem = smem;
+  }
+  const int occ = p.occ;
   if (occ <= 0) throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: launch does not fit an SM"};
   if (per_sm <= 0 || per_sm > occ) per_sm = occ;
   int grid = (int)std::min<uint64_t>((uint64_t)per_sm * t.num_sms, p.num_chunks);
