@@ -271,3 +271,25 @@ def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
                 t.mttkrp(n, tf, y)
                 torch.cuda.synchronize()
                 G.assert_parity(y.cpu().numpy(), dims, inds, vals, facs, 16, n)
+
+
+@pytest.mark.parametrize("kind", ["l2tiles", "staged", "compact"])
+def test_shards_with_tiled_plans(cuda_device, kind):
+    """§8(e) with tiled plans: each shard's L2-tiled / shared-memory-tiled / compact-record
+    plan covers only its slice of the matricized order; the P partial outputs sum to the
+    full result exactly (integer data) and to the oracle; host input (upload || presort)."""
+    dims, R = (150, 110, 90), 32
+    inds, vals = synth.gen_coo(dims, 24007, 31, zipf=(1.0, 0.6, 0.8), val_kind="int")
+    facs = synth.gen_factors(dims, R, 32, "int")
+    for n in range(3):
+        others = [m for m in range(3) if m != n]
+        flags = {"l2tiles": sf.LAUNCH_L2_TILES, "staged": 0, "compact": sf.LAUNCH_COMPACT}[kind]
+        L = sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={others[-1]: max(1, dims[others[-1]] // 3)},
+                           flags=flags)
+        Yfull, _ = oracle.mttkrp(dims, inds, vals, facs, R, n)
+        for P in (2, 5):
+            acc = np.zeros_like(Yfull)
+            for p in range(P):
+                Y, info = G.run(dims, inds, vals, facs, R, modes=[n], launch=L, shard=(P, p), device_input=False)
+                acc += Y[n]
+            assert np.array_equal(acc, Yfull), (kind, n, P)
