@@ -56,6 +56,17 @@ def grid(dims, n, R, quick):
             for C, th, fl in itertools.product(chunks, threads, (2,) if not st else (10,)):
                 yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl,
                        "staged": {m: min(r, dims[m]) for m, r in zip(st, rows)}}
+    # L2-tiled plans (SF_LAUNCH_L2_TILES = 64): one gathered factor >= 16 MB in 16/32/64 MB blocks
+    for m in others:
+        fac = dims[m] * R * 4
+        if fac < 16 * 2**20:
+            continue
+        for mb in ((64,) if quick else (16, 32, 64)):
+            rows = int(mb * 2**20 / (R * 4))
+            if rows >= dims[m]:
+                continue
+            for C, th in itertools.product(chunks, threads):
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": 2 | 64, "staged": {m: rows}}
     yield {"kernel": 1}
 
 
