@@ -2,22 +2,28 @@
 """ScalFrag-on-B200 benchmark: mode-n sparse MTTKRP (Eq. (4)).
 
 Contract (one JSON line on rank 0):
-  python bench.py [--gpus N --steps K --warmup W] [--config nell2] [--impl ours|reference]
+  python bench.py [--gpus N --steps K --warmup W] [--config nell1] [--impl ours|reference]
 
-* workload: BASELINE.json configs[1] (nell-2-shaped 12092x9184x28818, nnz=76,879,419,
-  R=32), synthetic, seeded (synth/), the largest config whose metric is quoted at 1 GPU.
+* workload: BASELINE.json configs[3] (nell-1-shaped 2902330 x 2143368 x 25495389,
+  nnz = 143,599,552, R = 32): the config BASELINE.json's metric is quoted on "at 1/2/4/8
+  GPUs" and the largest 1-GPU config whose plans all stay resident; synthetic, seeded
+  (synth/).  Other configs: --config nell2 | deli4d | amazon | tiny | <Table III shape>.
 * step: one sf_mttkrp per mode over all N modes (a CP-ALS sweep's MTTKRPs) on the
-  planned, HBM-resident tensor; for N>1 each rank owns a contiguous shard of every
-  mode's matricized order (§8(e)) and the step includes the boundary-row exchange
-  (NCCL all_gather + sf_rows_add).  Planning (sort/tile/features/select) is a
-  one-time cost per (mode, rank), reported as plan_ms, and is inside `e2e`.
-* value: GFLOP/s = sum_modes N*nnz*R / step time (flop convention N*nnz*R,
-  DESIGN.md reading R14), max over ranks, CUDA events on the launching stream.
+  planned, HBM-resident tensor; at N>1 each rank owns a contiguous shard of every mode's
+  matricized order (§8(e)), writes only its local row block, and every sf_mttkrp ends with
+  the boundary-row exchange (one NCCL allgather of R floats per rank, csrc/sf_comm.cu).  Planning (sort/tile/features/select) is a one-time cost per
+  (mode, rank), reported as plan_ms, and is inside `e2e`.
+  When every mode's plan does not fit HBM at once (amazon: 1.74 B nonzeros), each mode is
+  planned, timed (W warm-up + K event-timed launches) and released in turn, and the step
+  time is the sum of the per-mode means ("plans": "one mode at a time" in `config`).
+* value: GFLOP/s = sum_modes N*nnz*R / step time (flop convention N*nnz*R, DESIGN.md
+  reading R14), max over ranks, CUDA events on the launching stream.
 * e2e: the same metric through the public C ABI from PINNED HOST buffers:
   sf_tensor_create (segmented H2D + validate) + factor H2D + sf_plan (all modes)
   + sf_mttkrp (all modes) + D2H of every Y, every step.
 * roofline: dominant kernel = frag3_kernel; algorithmic bytes per launch =
-  4(N+1)*nnz + 4R*sum_m I_m, over its event-timed duration.
+  4(N+1)*nnz + 4R*sum_m I_m (SURVEY §8(d) D-3), over its event-timed duration;
+  traffic = ncu dram bytes per launch of that config (profiles/ncu_traffic.json).
 * cpu_baseline: the oracle (oracle/oracle.c, fp64, 1 thread) on a bounded sample.
 """
 from __future__ import annotations
@@ -25,6 +31,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -39,14 +46,30 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "src": "fallback (B200_PROFILING.md)"}
+METRIC = "MTTKRP GFLOP/s (all modes, N*nnz*R convention)"
 
 
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json)"}
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured (MEASURED_PEAKS.json hbm_gbs)"}
     return PEAKS_FALLBACK
+
+
+def load_traffic(cfg_name):
+    """ncu dram bytes (read + write) per frag3 launch of this config, averaged over its modes
+    (profiles/ncu_traffic.json, written from `ncu --set full` captures)."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None, None
+    try:
+        d = json.load(open(p)).get("configs", {}).get(cfg_name)
+    except Exception:
+        return None, None
+    if not d:
+        return None, None
+    return d.get("dram_bytes_per_launch"), d.get("source")
 
 
 # ---------------------------------------------------------------------------
@@ -113,6 +136,13 @@ def flops_per_mode(cfg, nnz=None):
     return cfg.nmodes * (cfg.nnz if nnz is None else nnz) * cfg.rank
 
 
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
 def cpu_oracle_sample(cfg, inds, vals, facs, sample_nnz):
     """Time the oracle (as it stands, 1 thread) on the first `sample_nnz` nonzeros, all modes."""
     import oracle
@@ -125,6 +155,17 @@ def cpu_oracle_sample(cfg, inds, vals, facs, sample_nnz):
         oracle.mttkrp(cfg.dims, si, sv, facs, cfg.rank, m, with_scale=False)
     dt = time.perf_counter() - t0
     return n, dt
+
+
+def workload_config(cfg, world, one_plan=False):
+    d = {"workload": f"{cfg.name}: {cfg.note}", "dims": list(cfg.dims), "nnz": cfg.nnz,
+         "rank": cfg.rank, "zipf": list(cfg.zipf), "modes": cfg.nmodes,
+         "parallelism": f"nnz-shard{world}" if world > 1 else "single",
+         "l2": "inputs larger than L2: each mode streams its own >=1 GB sorted record copy per launch; "
+               "factors are gathered through L2 as the method intends",
+         "step": "one sf_mttkrp per mode over all modes (+ boundary exchange at N>1)",
+         "plans": "one mode at a time (plan, time, release)" if one_plan else "all modes resident"}
+    return d
 
 
 def run_reference(args, cfg, rank, world):
@@ -146,13 +187,15 @@ def run_reference(args, cfg, rank, world):
     dt = time.perf_counter() - t0
     flops = flops_per_mode(cfg, per_step) * cfg.nmodes * args.steps
     v = flops / dt / 1e9
-    line = {"metric": "MTTKRP GFLOP/s (all modes, N*nnz*R convention)", "value": v, "unit": "GFLOP/s",
+    line = {"metric": METRIC, "value": v, "unit": "GFLOP/s",
             "impl": "reference", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": workload_config(cfg, world),
-            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
-                             "sample": f"first {per_step} nonzeros of the workload per step, all {cfg.nmodes} modes"},
+            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": 1, "host_cores": host_cores(),
+                             "kind": "oracle",
+                             "sample": f"first {per_step} nonzeros of the workload per step, all {cfg.nmodes} "
+                                       f"modes, fp64 single thread (1 of {host_cores()} host cores)"},
             "e2e": {"value": v, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -164,13 +207,23 @@ def launch_from_json(sf, d):
     return sf.Launch.make(**d)
 
 
-def workload_config(cfg, world):
-    return {"workload": f"{cfg.name}: {cfg.note}", "dims": list(cfg.dims), "nnz": cfg.nnz,
-            "rank": cfg.rank, "zipf": list(cfg.zipf), "modes": cfg.nmodes,
-            "parallelism": f"nnz-shard{world}" if world > 1 else "single",
-            "l2": "inputs larger than L2: each mode streams its own 4(N+1)*nnz-byte sorted copy "
-                  "(>1 GB) per launch; factors are gathered through L2 as the method intends",
-            "step": "one sf_mttkrp per mode over all modes (+ boundary exchange at N>1)"}
+def plans_fit(cfg, free_bytes):
+    """Can every mode's plan stay resident next to the raw COO?  Per nonzero: raw SoA
+    4(N+1) B, the AoS copy 16/32 B, one 16/32-B record per mode, ~24 B of sort scratch."""
+    N, nnz = cfg.nmodes, cfg.nnz
+    rec = 16 if N <= 3 else 32
+    need = nnz * (4 * (N + 1) + rec + N * rec + 24) + 4 * cfg.rank * sum(cfg.dims) * 2
+    return need < 0.85 * free_bytes
+
+
+def self_launch(args):
+    """--gpus N without torchrun: re-run this command under torch.distributed.run."""
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
 
 
 def main():
@@ -178,19 +231,25 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="nell2")
+    ap.add_argument("--config", default="nell1")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-sample", type=int, default=30_000_000)
     ap.add_argument("--ref-sample", type=int, default=1_000_000)
+    ap.add_argument("--one-plan", action="store_true", help="plan/time/release one mode at a time")
     ap.add_argument("--launch-json", default=None, help="override launches: {mode: launch dict}")
     args = ap.parse_args()
 
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        self_launch(args)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        sys.exit(2)
     cfg = synth.CONFIGS[args.config]
 
     if args.impl == "reference":
@@ -221,84 +280,127 @@ def main():
     t_gen = time.perf_counter()
     d_inds, d_vals = synth.config_tensor_device(cfg, device=dev)
     d_facs = synth.config_factors_device(cfg, device=dev)
-    h_inds = [a.cpu().pin_memory() for a in d_inds]
-    h_vals = d_vals.cpu().pin_memory()
-    h_facs = [f.cpu().pin_memory() for f in d_facs]
-    inds = [a.numpy().view(np.uint32) for a in h_inds]
-    vals = h_vals.numpy()
-    facs = [f.numpy() for f in h_facs]
+    raw_bytes = sum(a.numel() * 4 for a in d_inds) + d_vals.numel() * 4
+    import psutil
+    want_host = not (args.no_e2e and (args.no_cpu or rank != 0 or world > 1))
+    host_ok = psutil.virtual_memory().available > 2.5 * raw_bytes
+    e2e_skip = None if host_ok else f"host RAM: {psutil.virtual_memory().available / 2**30:.0f} GiB available"
+    h_inds = h_vals = h_facs = inds = vals = facs = None
+    if want_host and host_ok:
+        h_inds = [a.cpu().pin_memory() for a in d_inds]
+        h_vals = d_vals.cpu().pin_memory()
+        h_facs = [f.cpu().pin_memory() for f in d_facs]
+        inds = [a.numpy().view(np.uint32) for a in h_inds]
+        vals = h_vals.numpy()
+        facs = [f.numpy() for f in h_facs]
     t_gen = time.perf_counter() - t_gen
     stream = torch.cuda.Stream(device=dev)
 
-    # ---- resident tensor + plans ----
+    # ---- resident tensor ----
     T = sf.Tensor(cfg.dims, d_inds, d_vals)
     del d_inds, d_vals
     torch.cuda.empty_cache()
-    if world > 1:
-        T.set_shard(world, rank)
+    if world > 1:  # shard + the boundary exchange inside sf_mttkrp (NCCL; gloo transport on one GPU)
+        sfdist.attach(T, world, rank)
+    free, _ = torch.cuda.mem_get_info(dev)
+    one_plan = args.one_plan or not plans_fit(cfg, free)
     overrides = {}
     if args.launch_json:
         src = args.launch_json
         overrides = json.load(open(src[1:])) if src.startswith("@") else json.loads(src)
-    plan_ms = {}
-    for n in range(N):
+
+    def plan_mode(TT, n):
         if str(n) in overrides:
-            T.set_launch(n, R, launch_from_json(sf, overrides[str(n)]))
+            TT.set_launch(n, R, launch_from_json(sf, overrides[str(n)]))
         else:
-            T.plan(n, R)
-        plan_ms[n] = T.plan_info(n, R)["plan_ms"]
-    infos = {n: T.plan_info(n, R) for n in range(N)}
-    outs = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
-    # one boundary exchange per step for all modes (a single all_gather, dist.StepExchange)
-    exch = sfdist.StepExchange(world, rank, R, dev, host_staging=same_gpu) if world > 1 else None
+            TT.plan(n, R)
 
     def max_over_ranks(x):
         t = torch.tensor([x], dtype=torch.float64, device="cpu" if same_gpu else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    def step(ev=None):
-        for n in range(N):
-            if ev is not None:
-                ev[n][0].record(stream)
-            T.mttkrp(n, d_facs, outs[n], stream=stream)
-            if ev is not None:
-                ev[n][1].record(stream)
-        if exch is not None:
-            exch.combine([(outs[n], infos[n]["row_begin"], infos[n]["row_end"]) for n in range(N)], stream)
+    def barrier_sync():
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
 
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize(dev)
-
-    evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in range(N)]
-           for _ in range(args.steps)]
-    t0 = torch.cuda.Event(enable_timing=True)
-    t1 = torch.cuda.Event(enable_timing=True)
     clk = ClockSampler(local_dev)
-    clk.start()
-    time.sleep(0.3)
-    launches0 = sf.kernel_launches()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize(dev)
-    t0.record(stream)
-    for k in range(args.steps):
-        step(evs[k])
-    t1.record(stream)
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
-    launches = sf.kernel_launches() - launches0
-    clocks = clk.stop()
-    ms_total = t0.elapsed_time(t1)
+    plan_ms, infos, per_mode_ms = {}, {}, {}
+    launches = 0
+    if not one_plan:
+        for n in range(N):
+            plan_mode(T, n)
+            plan_ms[n] = T.plan_info(n, R)["plan_ms"]
+        infos = {n: T.plan_info(n, R) for n in range(N)}
+        outs = [torch.empty((infos[n]["out_rows"], R), dtype=torch.float32, device=dev) for n in range(N)]
+
+        def step(ev=None):
+            for n in range(N):
+                if ev is not None:
+                    ev[n][0].record(stream)
+                T.mttkrp(n, d_facs, outs[n], stream=stream)
+                if ev is not None:
+                    ev[n][1].record(stream)
+
+        for _ in range(args.warmup):
+            step()
+        evs = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in range(N)]
+               for _ in range(args.steps)]
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        clk.start()
+        time.sleep(0.3)
+        launches0 = sf.kernel_launches()
+        barrier_sync()
+        t0.record(stream)
+        for k in range(args.steps):
+            step(evs[k])
+        t1.record(stream)
+        barrier_sync()
+        launches = sf.kernel_launches() - launches0
+        clocks = clk.stop()
+        ms_total = t0.elapsed_time(t1)
+        per_mode_ms = {n: statistics.mean(evs[k][n][0].elapsed_time(evs[k][n][1]) for k in range(args.steps))
+                       for n in range(N)}
+    else:
+        # one plan resident at a time: per mode plan -> W warm-up -> K timed launches -> release
+        ms_total = 0.0
+        clk.start()
+        time.sleep(0.3)
+        for n in range(N):
+            plan_mode(T, n)
+            info = T.plan_info(n, R)
+            plan_ms[n], infos[n] = info["plan_ms"], info
+            out = torch.empty((info["out_rows"], R), dtype=torch.float32, device=dev)
+            for _ in range(args.warmup):
+                T.mttkrp(n, d_facs, out, stream=stream)
+            ev = [[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
+                  for _ in range(args.steps)]
+            l0 = sf.kernel_launches()
+            barrier_sync()
+            t0 = torch.cuda.Event(enable_timing=True)
+            t1 = torch.cuda.Event(enable_timing=True)
+            t0.record(stream)
+            for k in range(args.steps):
+                ev[k][0].record(stream)
+                T.mttkrp(n, d_facs, out, stream=stream)
+                ev[k][1].record(stream)
+            t1.record(stream)
+            barrier_sync()
+            launches += sf.kernel_launches() - l0
+            ms_total += t0.elapsed_time(t1)
+            per_mode_ms[n] = statistics.mean(e[0].elapsed_time(e[1]) for e in ev)
+            del out
+            T.plan_release(n, R)
+            torch.cuda.empty_cache()
+        clocks = clk.stop()
     if world > 1:
         ms_total = max_over_ranks(ms_total)
     ms_step = ms_total / args.steps
     flops_step = flops_per_mode(cfg) * N
     value = flops_step / (ms_step * 1e-3) / 1e9
-    per_mode_ms = {n: statistics.mean(evs[k][n][0].elapsed_time(evs[k][n][1]) for k in range(args.steps))
-                   for n in range(N)}
     bm = bytes_model(cfg)
     peaks = load_peaks()
     mean_launch_ms = statistics.mean(per_mode_ms.values())
@@ -306,64 +408,52 @@ def main():
     nnz_local = statistics.mean(infos[n]["nnz_local"] for n in range(N))
     bytes_launch = 4 * (N + 1) * nnz_local + 4 * R * sum(cfg.dims)
     achieved = bytes_launch / (mean_launch_ms * 1e-3) / 1e9
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(prof):
-        try:
-            d = json.load(open(prof))
-            if d.get("config") == cfg.name and world == 1:
-                traffic = d.get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    traffic, traffic_src = load_traffic(cfg.name) if world == 1 else (None, None)
 
     # ---- the same step with re-planning (A2-A4 on the device-resident raw COO) ----
-    # Planning is a one-time cost per (mode, rank) in CP-ALS; reported beside `value` so the
-    # whole §8(a) path (sort + tiles + features + selection + kernel) is measured too.
-    auto = sf.Launch()
-    auto.kernel = 0
-    torch.cuda.synchronize(dev)
-    p0 = time.perf_counter()
-    for n in range(N):
-        T.set_launch(n, R, auto)  # SF_KERNEL_AUTO: re-plan with the selector
-        T.mttkrp(n, d_facs, outs[n], stream=stream)
-    torch.cuda.synchronize(dev)
-    plan_step_ms = (time.perf_counter() - p0) * 1e3
-    if world > 1:
-        plan_step_ms = max_over_ranks(plan_step_ms)
-    infos = {n: T.plan_info(n, R) for n in range(N)}
+    plan_step_ms = None
+    if not one_plan:
+        auto = sf.Launch()
+        auto.kernel = 0
+        torch.cuda.synchronize(dev)
+        p0 = time.perf_counter()
+        for n in range(N):
+            T.set_launch(n, R, auto)  # SF_KERNEL_AUTO: re-plan with the selector
+            T.mttkrp(n, d_facs, outs[n], stream=stream)
+        torch.cuda.synchronize(dev)
+        plan_step_ms = (time.perf_counter() - p0) * 1e3
+        if world > 1:
+            plan_step_ms = max_over_ranks(plan_step_ms)
+        del outs
+    T.close()
+    torch.cuda.empty_cache()
 
     # ---- e2e through the public API from pinned host buffers ----
     e2e = None
-    if not args.no_e2e:
-        h_out = [torch.empty((cfg.dims[n], R), dtype=torch.float32).pin_memory() for n in range(N)]
+    if not args.no_e2e and h_inds is not None:
+        h_out = [torch.empty((infos[n]["out_rows"], R), dtype=torch.float32).pin_memory() for n in range(N)]
         h2d = sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4 + sum(f.numel() * 4 for f in h_facs)
         d2h = sum(o.numel() * 4 for o in h_out)
 
         def e2e_step():
             with sf.Tensor(cfg.dims, h_inds, h_vals) as T2:
                 if world > 1:
-                    T2.set_shard(world, rank)
+                    sfdist.attach(T2, world, rank)
                 df = [f.to(dev, non_blocking=True) for f in h_facs]
                 for n in range(N):
-                    if str(n) in overrides:
-                        T2.set_launch(n, R, launch_from_json(sf, overrides[str(n)]))
-                    else:
-                        T2.plan(n, R)
-                inf = {n: T2.plan_info(n, R) for n in range(N)}
-                os_ = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
-                for n in range(N):
-                    T2.mttkrp(n, df, os_[n], stream=stream)
-                if exch is not None:
-                    exch.combine([(os_[n], inf[n]["row_begin"], inf[n]["row_end"]) for n in range(N)], stream)
-                with torch.cuda.stream(stream):
-                    for n in range(N):
-                        h_out[n].copy_(os_[n], non_blocking=True)
+                    plan_mode(T2, n)
+                    inf = T2.plan_info(n, R)
+                    o = torch.empty((inf["out_rows"], R), dtype=torch.float32, device=dev)
+                    T2.mttkrp(n, df, o, stream=stream)
+                    with torch.cuda.stream(stream):
+                        h_out[n][:o.shape[0]].copy_(o, non_blocking=True)
+                    if one_plan:
+                        stream.synchronize()
+                        T2.plan_release(n, R)
                 torch.cuda.synchronize(dev)
 
         e2e_step()  # warm-up
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize(dev)
+        barrier_sync()
         s0 = time.perf_counter()
         for _ in range(args.e2e_steps):
             e2e_step()
@@ -376,24 +466,27 @@ def main():
                "steps": args.e2e_steps,
                "includes": "sf_tensor_create(pinned host COO, segmented H2D+validate) + factor H2D + "
                            "sf_plan x N + sf_mttkrp x N + D2H of every Y (host wall clock)"}
+    elif not args.no_e2e and e2e_skip:
+        e2e = {"value": None, "skipped": e2e_skip}
 
     # ---- CPU oracle baseline (rank 0, N=1 only) ----
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and world == 1 and not args.no_cpu and inds is not None:
         n_s, dt = cpu_oracle_sample(cfg, inds, vals, facs, args.cpu_sample)
-        cpu = {"value": flops_per_mode(cfg, n_s) * N / dt / 1e9, "unit": "GFLOP/s", "cores": 1,
+        hc = host_cores()
+        cpu = {"value": flops_per_mode(cfg, n_s) * N / dt / 1e9, "unit": "GFLOP/s", "cores": 1, "host_cores": hc,
                "kind": "oracle", "sample": f"first {n_s} of {cfg.nnz} nonzeros, all {N} modes, "
-                                            f"fp64 single thread, {dt:.1f} s"}
+                                            f"fp64 single thread (1 of {hc} host cores), {dt:.1f} s"}
 
     if rank == 0:
         line = {
-            "metric": "MTTKRP GFLOP/s (all modes, N*nnz*R convention)",
+            "metric": METRIC,
             "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": workload_config(cfg, world),
+            "config": workload_config(cfg, world, one_plan),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                         "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                         "frac": achieved / peaks["hbm_gbs"], "traffic": traffic, "traffic_src": traffic_src,
                          "kernel": "frag3_kernel", "peak_src": peaks["src"],
                          "bytes_per_launch": bytes_launch, "launch_ms": mean_launch_ms},
             "cpu_baseline": cpu,
@@ -405,14 +498,13 @@ def main():
                                   "launch": infos[n]["launch"], "num_tiles": infos[n]["num_tiles"],
                                   "num_chunks": infos[n]["num_chunks"]}
                          for n in range(N)},
-            "plan_step": {"ms": plan_step_ms, "value": flops_step / (plan_step_ms * 1e-3) / 1e9,
-                          "unit": "GFLOP/s",
-                          "includes": "per mode: sf_plan (matricized sort, features, selection, tiles, "
-                                      "chunks) + sf_mttkrp, device-resident raw COO, host wall clock"},
+            "plan_step": None if plan_step_ms is None else {
+                "ms": plan_step_ms, "value": flops_step / (plan_step_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
+                "includes": "per mode: sf_plan (matricized sort, features, selection, tiles, chunks) + "
+                            "sf_mttkrp, device-resident raw COO, host wall clock"},
             "gen_s": t_gen,
         }
         print(json.dumps(line), flush=True)
-    T.close()
     if world > 1:
         dist.destroy_process_group()
 

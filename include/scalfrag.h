@@ -19,7 +19,8 @@
  *     returns a thread-local detail string.
  *   - 2 <= nmodes <= SF_MAX_MODES; 1 <= dims[m] <= 2^32-1; indices are 0-based
  *     uint32; values fp32; factors fp32 row-major I_m x rank (ld = rank).
- *   - Per-device nnz (per shard) must be < 2^32.  nnz = 0 is valid (Y = 0).
+ *   - nnz must be < 2^32 (plans store input positions as uint32; SF_ERR_UNSUPPORTED
+ *     otherwise).  nnz = 0 is valid (Y = 0).
  *   - A handle is bound to the CUDA device current at create time; it owns all
  *     device arrays, plans and scratch.  Handles are not thread-safe; calls on
  *     different handles are independent.
@@ -48,8 +49,9 @@ typedef enum {
   SF_ERR_INDEX_OUT_OF_RANGE = 2, /* some inds[m][e] >= dims[m] */
   SF_ERR_OUT_OF_MEMORY = 3,      /* cudaMalloc / pinned allocation failed */
   SF_ERR_NOT_PLANNED = 4,        /* sf_mttkrp before sf_plan(mode, rank) */
-  SF_ERR_UNSUPPORTED = 5,        /* e.g. shard nnz >= 2^32 */
-  SF_ERR_CUDA = 6                /* a CUDA runtime call failed (detail in sf_last_error) */
+  SF_ERR_UNSUPPORTED = 5,        /* e.g. nnz >= 2^32, rank/nmodes without a kernel */
+  SF_ERR_CUDA = 6,               /* a CUDA runtime call failed (detail in sf_last_error) */
+  SF_ERR_NCCL = 7                /* a collective failed (NCCL, or the caller's transport returned != 0) */
 } sf_status;
 
 /* Kernel families. */
@@ -71,9 +73,14 @@ typedef struct {
                             blocks of block_rows[m] rows (a "tensor block") */
   uint32_t block_rows[SF_MAX_MODES];
   uint32_t flags;        /* FRAG: SF_LAUNCH_* bits below */
+  uint32_t hot_kb;       /* FRAG: hot-row cache budget in KiB (0 = off).  The most frequent rows
+                            of the gathered factors that are neither staged nor L2-tiled (by
+                            nonzero count in this plan, one global threshold) are copied per
+                            call into one dense block and gathered from there (DESIGN.md §5
+                            "hot-row cache"); plain records need I_m < 2^31, packed records one
+                            spare bit per such field (else the slot is skipped). */
 } sf_launch_t;
 #define SF_LAUNCH_NO_OWNER_STORES 4u /* FRAG, unstaged: memset Y + atomics only (disable A5) */
-#define SF_LAUNCH_NO_CARRY 8u /* legacy (round-1 stretch kernel); ignored: frag3 flushes once per run */
 #define SF_LAUNCH_DETERMINISTIC 32u /* FRAG: A7 two-pass carry combine instead of atomics; forces an
                                        unstaged owner-store plan; Y is bitwise reproducible run to run */
 #define SF_LAUNCH_L2_TILES 64u /* FRAG: the staged_mask modes are NOT copied into shared memory; they
@@ -82,12 +89,6 @@ typedef struct {
                                  taking 1/grid of each, so the factor rows gathered at any moment
                                  are one block that stays L2-resident (for factors >> L2).  Forces
                                  memset + atomics (no owner stores); ignored with DETERMINISTIC. */
-#define SF_LAUNCH_COMPACT 128u /* FRAG, N = 3, non-owner plans: 8-byte records (gathered indices + run
-                                  delta, value; i_n per slot in a side array) where the fields fit
-                                  30 bits.  Halves the record stream, but measured 9 % slower on
-                                  nell-2 (+19 % issued instructions for the decode): opt-in. */
-#define SF_LAUNCH_L1_NO_ALLOCATE 2u /* informational: global gathers always bypass L1 allocation
-                                       (ld.global.nc.L1::no_allocate.v8.f32; measured faster) */
 
 /* Tensor feature vector (reading R4). Integers are exact. */
 typedef struct {
@@ -113,6 +114,8 @@ typedef struct {
   uint64_t num_chunks;
   uint64_t row_begin;   /* this shard touches rows [row_begin, row_end) of Y */
   uint64_t row_end;
+  uint64_t out_row0;    /* sf_mttkrp's `out` holds rows [out_row0, out_row0 + out_rows) of Y: */
+  uint64_t out_rows;    /*   all of Y at nranks == 1, the local block [row_begin, row_end) else */
   uint64_t device_bytes;
   double plan_ms;       /* device time of the last sf_plan for this (mode, rank) */
 } sf_plan_info_t;
@@ -135,8 +138,41 @@ sf_status sf_tensor_destroy(sf_tensor_t t);
 
 /* Multi-GPU (§8(e)): restrict this handle to shard `rank` of `nranks`: for every mode
  * it owns matricized positions [floor(rank*nnz/nranks), floor((rank+1)*nnz/nranks)).
- * Drops existing plans.  Default 1/0. */
+ * With nranks > 1, sf_mttkrp writes only this shard's LOCAL ROW BLOCK (sf_shard_rows).
+ * Drops existing plans (synchronizes the device first).  Default 1/0. */
 sf_status sf_set_shard(sf_tensor_t t, int nranks, int rank);
+
+/* Rows [*row_begin, *row_end) of Y that sf_mttkrp(mode, rank) writes into `out` (out row 0 =
+ * Y row *row_begin): all of Y for an unsharded handle, this shard's local row block else
+ * (the rows its nonzeros touch; adjacent shards share at most one boundary row, which the
+ * exchange below assigns to the lowest rank touching it).  Needs sf_plan(mode, rank). */
+sf_status sf_shard_rows(sf_tensor_t t, int mode, int rank, uint64_t* row_begin, uint64_t* row_end);
+
+/* Collective transport for sharded handles.  With a comm attached,
+ * sf_mttkrp ends with the boundary-row exchange on its stream: the partial of a shard's
+ * first row, if a lower rank also touches it, is sent to that owner (and zeroed locally);
+ * the owner adds the partials in rank order.  Afterwards the local blocks hold a
+ * ROW-SHARDED Y: each row's value lives on its owner, the other copies are 0, rows no
+ * shard touches are 0 everywhere.  One allgather of rank*4 bytes per rank per call.
+ *   sf_comm_unique_id: rank 0 creates a 128-byte NCCL id (broadcast it, e.g. by torch).
+ *   sf_comm_attach:    ncclCommInitRank on this handle's device + sf_set_shard(nranks, rank).
+ *   sf_comm_attach_transport: the same exchange over the caller's allgatherv (tests, or a
+ *                      non-NCCL fabric); fn returns 0 on success.
+ * NCCL is loaded at run time (dlopen libnccl.so.2); SF_ERR_NCCL on any collective error. */
+typedef int (*sf_allgatherv_fn)(void* ctx, const void* send, void* recv, const uint64_t* bytes,
+                                const uint64_t* displs, int nranks, void* stream);
+sf_status sf_comm_unique_id(void* id128);
+sf_status sf_comm_attach(sf_tensor_t t, int nranks, int rank, const void* id128);
+sf_status sf_comm_attach_transport(sf_tensor_t t, int nranks, int rank, sf_allgatherv_fn fn, void* ctx);
+sf_status sf_comm_detach(sf_tensor_t t);
+/* Replicated Y from the row-sharded local blocks after sf_mttkrp (optional):
+ * full (device, I_mode x rank) receives every rank's owned rows, zeros elsewhere. */
+sf_status sf_allgather_rows(sf_tensor_t t, int mode, int rank, const float* local, float* full, void* stream);
+/* Host-only (no GPU needed): the exchange rule for given touched row ranges
+ * (ranges[2k], ranges[2k+1] = [begin, end) of rank k; begin == end: empty shard).
+ * send_first[k] = 1 iff rank k's first row is owned by a lower rank; owner[k] = the owner
+ * of rank k's first row (the lowest rank touching it; k itself if it owns it; -1 if empty). */
+sf_status sf_exchange_map(int nranks, const uint64_t* ranges, int32_t* send_first, int32_t* owner);
 
 /* ---- planning (§8(a) A2-A4) -------------------------------------------- */
 
@@ -177,8 +213,9 @@ sf_status sf_set_selector_model(const int32_t* feature, const double* threshold,
 /* ---- the hot path (§8(a) A5-A7) ---------------------------------------- */
 
 /* Y = mode-`mode` MTTKRP.  factors: host array of nmodes DEVICE pointers (factors[mode]
- * is ignored and may be NULL); out: device I_mode x rank fp32, overwritten (with a
- * shard set, only rows [row_begin,row_end) are written; the rest are zeroed).
+ * is ignored and may be NULL); out: device fp32, out_rows x rank (sf_shard_rows /
+ * sf_plan_info: I_mode x rank unsharded, the local row block of a shard), overwritten.
+ * With a comm attached the boundary-row exchange follows on the same stream.
  * Stream-ordered, returns after enqueue.  out must not alias a factor. */
 sf_status sf_mttkrp(sf_tensor_t t, int mode, const float* const* factors, int rank, float* out,
                     void* stream);
@@ -207,7 +244,10 @@ sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int co
  * hot path for line 4 of Alg. 1 (plans are built on demand with the selector).  factors:
  * nmodes DEVICE pointers, fp32 I_m x rank row-major, in/out (initial guess -> result).
  * fits: host array of >= iters doubles (may be NULL), fit after each sweep; stops early
- * when tol > 0 and |fit_k - fit_{k-1}| < tol.  rank <= 64; no shard (nranks must be 1).
+ * when tol > 0 and |fit_k - fit_{k-1}| < tol.  rank <= 64.  Sharded handles need a comm
+ * (sf_comm_attach*) and the SAME initial factors on every rank: each rank computes
+ * A_n = M V^+ for its owned rows, the row blocks are allgathered (every rank ends with the
+ * full, identical factors) and the Grams / fit terms are summed in rank order.
  * Stream-ordered work, synchronizes once per sweep (to read the fit). */
 sf_status sf_cpals(sf_tensor_t t, int rank, float* const* factors, int iters, double tol, double* fits,
                    int* iters_done, void* stream);

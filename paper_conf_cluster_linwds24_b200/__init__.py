@@ -23,14 +23,13 @@ _lib = None
 SF_MAX_MODES = 8
 SF_HIST_BINS = 40
 KERNEL_AUTO, KERNEL_COO, KERNEL_FRAG = 0, 1, 2
-LAUNCH_L1_NO_ALLOCATE, LAUNCH_NO_OWNER_STORES, LAUNCH_NO_CARRY = 2, 4, 8
+LAUNCH_NO_OWNER_STORES = 4
 LAUNCH_DETERMINISTIC = 32
 LAUNCH_L2_TILES = 64
-LAUNCH_COMPACT = 128
 
 STATUS = {0: "SF_OK", 1: "SF_ERR_INVALID_ARG", 2: "SF_ERR_INDEX_OUT_OF_RANGE",
           3: "SF_ERR_OUT_OF_MEMORY", 4: "SF_ERR_NOT_PLANNED", 5: "SF_ERR_UNSUPPORTED",
-          6: "SF_ERR_CUDA"}
+          6: "SF_ERR_CUDA", 7: "SF_ERR_NCCL"}
 
 
 class SfError(RuntimeError):
@@ -43,20 +42,22 @@ class Launch(ctypes.Structure):
     _fields_ = [("kernel", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("chunk_nnz", ctypes.c_int32),
                 ("staged_mask", ctypes.c_uint32), ("block_rows", ctypes.c_uint32 * SF_MAX_MODES),
-                ("flags", ctypes.c_uint32)]
+                ("flags", ctypes.c_uint32), ("hot_kb", ctypes.c_uint32)]
 
     def as_dict(self):
         return {"kernel": {0: "auto", 1: "coo", 2: "frag"}.get(self.kernel, self.kernel),
                 "block_threads": self.block_threads, "ctas_per_sm": self.ctas_per_sm,
                 "chunk_nnz": self.chunk_nnz, "staged_mask": self.staged_mask,
-                "block_rows": list(self.block_rows), "flags": self.flags}
+                "block_rows": list(self.block_rows), "flags": self.flags, "hot_kb": self.hot_kb}
 
     @classmethod
     def make(cls, kernel=KERNEL_FRAG, block_threads=512, ctas_per_sm=0, chunk_nnz=128,
-             staged=None, flags=0):
-        """staged: {mode: block_rows}; flags: LAUNCH_* bits (include/scalfrag.h)"""
+             staged=None, flags=0, hot_kb=0):
+        """staged: {mode: block_rows}; flags: LAUNCH_* bits (include/scalfrag.h);
+        hot_kb: hot-row cache budget in KiB (0 = off)"""
         l = cls()
         l.flags = flags
+        l.hot_kb = hot_kb
         l.kernel, l.block_threads, l.ctas_per_sm, l.chunk_nnz = kernel, block_threads, ctas_per_sm, chunk_nnz
         mask = 0
         for m, r in (staged or {}).items():
@@ -86,14 +87,15 @@ class PlanInfo(ctypes.Structure):
     _fields_ = [("feat", Features), ("launch", Launch), ("nnz_local", ctypes.c_uint64),
                 ("num_tiles", ctypes.c_uint64), ("num_chunks", ctypes.c_uint64),
                 ("row_begin", ctypes.c_uint64), ("row_end", ctypes.c_uint64),
+                ("out_row0", ctypes.c_uint64), ("out_rows", ctypes.c_uint64),
                 ("device_bytes", ctypes.c_uint64), ("plan_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {"features": self.feat.as_dict(), "launch": self.launch.as_dict(),
                 "nnz_local": self.nnz_local, "num_tiles": self.num_tiles,
                 "num_chunks": self.num_chunks, "row_begin": self.row_begin,
-                "row_end": self.row_end, "device_bytes": self.device_bytes,
-                "plan_ms": self.plan_ms}
+                "row_end": self.row_end, "out_row0": self.out_row0, "out_rows": self.out_rows,
+                "device_bytes": self.device_bytes, "plan_ms": self.plan_ms}
 
 
 EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
@@ -101,7 +103,14 @@ EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_
             "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
             "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
-            "sf_trim_cache"]
+            "sf_trim_cache", "sf_shard_rows", "sf_comm_unique_id", "sf_comm_attach",
+            "sf_comm_attach_transport", "sf_comm_detach", "sf_allgather_rows", "sf_exchange_map"]
+
+# int fn(void* ctx, const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs,
+#        int nranks, void* stream)
+ALLGATHERV_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                 ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64), ctypes.c_int,
+                                 ctypes.c_void_p)
 
 
 def lib(build_if_missing: bool = True):
@@ -134,12 +143,16 @@ def lib(build_if_missing: bool = True):
             L.sf_cpals.argtypes = [P, I, P, I, ctypes.c_double, P, ctypes.POINTER(I), P]
             L.sf_plan_release.argtypes = [P, I, I]
             L.sf_trim_cache.argtypes = []
-            for fn in ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
-                       "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
-                       "sf_mttkrp", "sf_mttkrp_streamed", "sf_rows_op", "sf_selector_features",
-                       "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
-            "sf_trim_cache"]:
-                getattr(L, fn).restype = ctypes.c_int
+            L.sf_shard_rows.argtypes = [P, I, I, ctypes.POINTER(U64), ctypes.POINTER(U64)]
+            L.sf_comm_unique_id.argtypes = [P]
+            L.sf_comm_attach.argtypes = [P, I, I, P]
+            L.sf_comm_attach_transport.argtypes = [P, I, I, ALLGATHERV_FN, P]
+            L.sf_comm_detach.argtypes = [P]
+            L.sf_allgather_rows.argtypes = [P, I, I, P, P, P]
+            L.sf_exchange_map.argtypes = [I, P, P, P]
+            for fn in EXPORTED:
+                if fn not in ("sf_status_string", "sf_last_error", "sf_kernel_launches", "sf_version"):
+                    getattr(L, fn).restype = ctypes.c_int
             L.sf_status_string.argtypes = [I]
             L.sf_status_string.restype = ctypes.c_char_p
             L.sf_last_error.argtypes = []
@@ -149,17 +162,12 @@ def lib(build_if_missing: bool = True):
             L.sf_version.argtypes = []
             L.sf_version.restype = ctypes.c_char_p
             _lib = L
-        if _lib is not None and not getattr(lib, "_model_loaded", False):
-            lib._model_loaded = True
-            if os.environ.get("SF_SELECTOR", DEFAULT_SELECTOR) == "model" and os.path.exists(MODEL_PATH):
-                _install_model(_lib, MODEL_PATH)
     return _lib
 
 
+# The deployed learned selector (tools/train_selector.py) is compiled into libscalfrag.so
+# and installed when it loads (_build.write_model_inc); set_selector_model replaces it.
 MODEL_PATH = os.path.join(_HERE, "selector_model.json")
-# "rules" (sf_select.cpp, calibrated on sweeps) or "model" (the learned DecisionTree,
-# tools/train_selector.py).  See DESIGN.md §5 for the held-out comparison that sets this.
-DEFAULT_SELECTOR = "model"
 
 
 def _install_model(L, path):
@@ -178,7 +186,10 @@ def _install_model(L, path):
 
 def set_selector_model(model):
     """model: dict with 'tree' (feature/threshold/left/right/value lists) and 'n_features',
-    or None to fall back to the rule-based selector."""
+    None to fall back to the rule-based selector, or "default" for the compiled-in model."""
+    if isinstance(model, str) and model == "default":
+        _install_model(lib(), MODEL_PATH)
+        return
     L = lib()
     if model is None:
         _check(L.sf_set_selector_model(None, None, None, None, None, 0, 0))
@@ -269,6 +280,32 @@ class Tensor:
     def set_shard(self, nranks, rank):
         _check(lib().sf_set_shard(self._h, int(nranks), int(rank)))
 
+    def shard_rows(self, mode, rank):
+        """Rows [begin, end) of Y that mttkrp(mode) writes into `out` (the local row block
+        of a shard; all of Y unsharded)."""
+        b, e = ctypes.c_uint64(0), ctypes.c_uint64(0)
+        _check(lib().sf_shard_rows(self._h, int(mode), int(rank), ctypes.byref(b), ctypes.byref(e)))
+        return b.value, e.value
+
+    def comm_attach(self, nranks, rank, unique_id: bytes):
+        """NCCL communicator for the boundary exchange (+ sf_set_shard(nranks, rank))."""
+        buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+        _check(lib().sf_comm_attach(self._h, int(nranks), int(rank), buf))
+
+    def comm_attach_transport(self, nranks, rank, fn):
+        """Boundary exchange over a Python allgatherv (ALLGATHERV_FN; kept alive here)."""
+        self._transport = fn if isinstance(fn, ALLGATHERV_FN) else ALLGATHERV_FN(fn)
+        _check(lib().sf_comm_attach_transport(self._h, int(nranks), int(rank), self._transport, None))
+
+    def comm_detach(self):
+        _check(lib().sf_comm_detach(self._h))
+
+    def allgather_rows(self, mode, local, full, stream=None):
+        """Replicated Y (full, I_mode x R on every rank) from the row-sharded local blocks."""
+        _check(lib().sf_allgather_rows(self._h, int(mode), int(full.shape[1]), _ptr(local), _ptr(full),
+                                       _stream_handle(stream)))
+        return full
+
     def plan(self, mode, rank, deterministic=False):
         """sf_plan (selector's launch); deterministic=True plans the A7 two-pass carry
         combine instead (unstaged owner-store fragment plan, bitwise reproducible Y)."""
@@ -349,6 +386,25 @@ def mttkrp_streamed(dims, inds, vals, factors, mode, out, segments=8, streams=4)
     _check(lib().sf_mttkrp_streamed(N, d, int(len(vals)), ip, _ptr(vals), fp, int(out.shape[1]), int(mode),
                                     _ptr(out), int(segments), int(streams)))
     return out
+
+
+def comm_unique_id() -> bytes:
+    """A new 128-byte NCCL unique id (rank 0; broadcast it to the other ranks)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().sf_comm_unique_id(buf))
+    return buf.raw
+
+
+def exchange_map(ranges):
+    """Host-only exchange rule (sf_exchange_map): ranges = [(row_begin, row_end)] per rank.
+    Returns (send_first[k], owner[k])."""
+    import numpy as np
+    P = len(ranges)
+    r = np.ascontiguousarray(np.array(ranges, dtype=np.uint64).reshape(P, 2))
+    sendf = np.zeros(P, np.int32)
+    owner = np.zeros(P, np.int32)
+    _check(lib(build_if_missing=True).sf_exchange_map(P, r.ctypes.data, sendf.ctypes.data, owner.ctypes.data))
+    return sendf.tolist(), owner.tolist()
 
 
 ROWS_PACK, ROWS_ADD, ROWS_ZERO = 0, 1, 2

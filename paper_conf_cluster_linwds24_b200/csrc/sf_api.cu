@@ -41,22 +41,26 @@ void trace_mark(const char* phase) {
 }
 
 // Caching device allocator.  cudaMalloc/cudaFree of GB-sized plan arrays cost tens of ms
-// each and cudaFree synchronizes the device; blocks are instead kept in a size-keyed free
-// list and reused (best fit within 2x).  Reuse is stream-safe because every library buffer
-// is produced and consumed on the handle's planning stream, or the device is synchronized
-// first (plan replacement and handle destruction call cudaDeviceSynchronize).
+// each and cudaFree synchronizes the device; blocks are instead kept in a free list keyed by
+// (device, size) and reused (best fit within 2x) -- a block is only ever handed back to a
+// buffer on the device it was allocated on.  Reuse is stream-safe because every library
+// buffer is produced and consumed on the handle's planning stream, or the device is
+// synchronized first (plan replacement, sf_set_shard and handle destruction call
+// cudaDeviceSynchronize).
 struct BlockCache {
   std::mutex mu;
-  std::multimap<size_t, void*> free_blocks;
+  std::multimap<std::pair<int, size_t>, void*> free_blocks;  // (device, bytes) -> block
   size_t cached = 0;
   void* get(size_t b, size_t* got) {
+    int dev = 0;
+    SF_CUDA(cudaGetDevice(&dev));
     {
       std::lock_guard<std::mutex> g(mu);
-      auto it = free_blocks.lower_bound(b);
-      if (it != free_blocks.end() && it->first <= 2 * b + (1u << 20)) {
+      auto it = free_blocks.lower_bound({dev, b});
+      if (it != free_blocks.end() && it->first.first == dev && it->first.second <= 2 * b + (1u << 20)) {
         void* q = it->second;
-        *got = it->first;
-        cached -= it->first;
+        *got = it->first.second;
+        cached -= it->first.second;
         free_blocks.erase(it);
         return q;
       }
@@ -76,14 +80,28 @@ struct BlockCache {
     return q;
   }
   void put(void* q, size_t b) {
+    int dev = 0;
+    cudaPointerAttributes a{};
+    if (cudaPointerGetAttributes(&a, q) == cudaSuccess) dev = a.device;
+    else cudaGetLastError();
     std::lock_guard<std::mutex> g(mu);
-    free_blocks.emplace(b, q);
+    free_blocks.emplace(std::make_pair(dev, b), q);
     cached += b;
   }
-  void trim() {
+  void trim() {  // every block is freed on its own device, after that device is idle
     std::lock_guard<std::mutex> g(mu);
-    cudaDeviceSynchronize();
-    for (auto& kv : free_blocks) cudaFree(kv.second);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    int synced = -1;
+    for (auto& kv : free_blocks) {
+      if (kv.first.first != synced) {
+        cudaSetDevice(kv.first.first);
+        cudaDeviceSynchronize();
+        synced = kv.first.first;
+      }
+      cudaFree(kv.second);
+    }
+    cudaSetDevice(cur);
     free_blocks.clear();
     cached = 0;
   }
@@ -106,14 +124,17 @@ void DevBuf::release() {
 }
 
 size_t Plan::device_bytes() const {
-  size_t b = val.bytes + rec.bytes + rowid.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes + tile_chunk.bytes;
-  for (int m = 0; m < SF_MAX_MODES; ++m) b += ind[m].bytes;
+  size_t b = val.bytes + rec.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes + tile_chunk.bytes +
+             hot_cache.bytes;
+  for (int m = 0; m < SF_MAX_MODES; ++m) b += ind[m].bytes + hot_rows[m].bytes;
   return b;
 }
 
 Tensor::~Tensor() {
   for (auto& kv : plans) delete kv.second;
   plans.clear();
+  delete comm;
+  comm = nullptr;
   if (stream) cudaStreamDestroy(stream);
 }
 
@@ -294,6 +315,8 @@ sf_status sf_tensor_create_ex(int nmodes, const uint64_t* dims, uint64_t nnz,
       if (dims[m] < 1 || dims[m] > 0xFFFFFFFFull)
         throw StatusError{SF_ERR_INVALID_ARG, "dims[m] must be in [1, 2^32-1]"};
     if (nnz > 0 && (!inds || !vals)) throw StatusError{SF_ERR_INVALID_ARG, "inds/vals NULL"};
+    if (nnz > 0xFFFFFFFFull)  // plans store input positions and slots as uint32
+      throw StatusError{SF_ERR_UNSUPPORTED, "nnz must be < 2^32 (input positions are uint32)"};
     if (nnz > 0)
       for (int m = 0; m < nmodes; ++m)
         if (!inds[m]) throw StatusError{SF_ERR_INVALID_ARG, "inds[m] is NULL"};
@@ -363,6 +386,10 @@ sf_status sf_set_shard(sf_tensor_t h, int nranks, int rank) {
     if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
     if (nranks < 1 || rank < 0 || rank >= nranks) throw StatusError{SF_ERR_INVALID_ARG, "bad shard"};
     Tensor* t = as_tensor(h);
+    if (!t->plans.empty()) {  // an in-flight sf_mttkrp may still read the plans' buffers
+      SF_CUDA(cudaSetDevice(t->device));
+      SF_CUDA(cudaDeviceSynchronize());
+    }
     for (auto& kv : t->plans) delete kv.second;
     t->plans.clear();
     t->nranks = nranks;
@@ -441,6 +468,8 @@ sf_status sf_plan_info(sf_tensor_t h, int mode, int rank, sf_plan_info_t* out) {
     out->num_chunks = p->num_chunks;
     out->row_begin = p->row_begin;
     out->row_end = p->row_end;
+    out->out_row0 = p->out_row0;
+    out->out_rows = p->out_rows;
     out->device_bytes = p->device_bytes();
     out->plan_ms = p->plan_ms;
     return SF_OK;
@@ -486,6 +515,49 @@ sf_status sf_mttkrp(sf_tensor_t h, int mode, const float* const* factors, int ra
     for (int m = 0; m < t->nmodes; ++m)
       if (m != mode && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
     launch_mttkrp(*t, *p, factors, out, static_cast<cudaStream_t>(stream));
+    exchange_rows(*t, *p, out, static_cast<cudaStream_t>(stream));
+    return SF_OK;
+  });
+}
+
+sf_status sf_shard_rows(sf_tensor_t h, int mode, int rank, uint64_t* row_begin, uint64_t* row_end) {
+  return guard([&]() -> sf_status {
+    if (!h || !row_begin || !row_end) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    Plan* p = get_plan(*t, mode, rank);
+    if (!p) throw StatusError{SF_ERR_NOT_PLANNED, "sf_plan(mode, rank) has not been called"};
+    *row_begin = p->out_row0;
+    *row_end = p->out_row0 + p->out_rows;
+    return SF_OK;
+  });
+}
+
+sf_status sf_allgather_rows(sf_tensor_t h, int mode, int rank, const float* local, float* full, void* stream) {
+  return guard([&]() -> sf_status {
+    if (!h || !full || !local) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
+    Tensor* t = as_tensor(h);
+    check_mode_rank(*t, mode, rank);
+    Plan* p = get_plan(*t, mode, rank);
+    if (!p) throw StatusError{SF_ERR_NOT_PLANNED, "sf_plan(mode, rank) has not been called"};
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    SF_CUDA(cudaMemsetAsync(full, 0, sizeof(float) * (size_t)rank * t->dims[mode], s));
+    if (t->nranks == 1 || !t->comm) {
+      if (t->nranks > 1) throw StatusError{SF_ERR_INVALID_ARG, "sharded handle without a comm"};
+      SF_CUDA(cudaMemcpyAsync(full, local, sizeof(float) * (size_t)rank * t->dims[mode], cudaMemcpyDeviceToDevice, s));
+      return SF_OK;
+    }
+    ensure_ranges(*t, *p, s);
+    const int P = t->nranks;
+    std::vector<int32_t> sendf(P), owner(P);
+    sf_exchange_map(P, p->ranges.data(), sendf.data(), owner.data());
+    std::vector<uint64_t> blk(2 * P);  // owned rows of every rank
+    for (int k = 0; k < P; ++k) {
+      const uint64_t b = p->ranges[2 * k], e = p->ranges[2 * k + 1];
+      blk[2 * k] = e > b ? b + (uint64_t)sendf[k] : b;
+      blk[2 * k + 1] = std::max(blk[2 * k], e);
+    }
+    allgather_blocks(*t, blk, local + (size_t)sendf[t->rank] * rank, full, rank, s);
     return SF_OK;
   });
 }
@@ -567,7 +639,8 @@ sf_status sf_cpals(sf_tensor_t h, int rank, float* const* factors, int iters, do
     if (!h || !factors || iters < 0) throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
     Tensor* t = as_tensor(h);
     check_mode_rank(*t, 0, rank);
-    if (t->nranks != 1) throw StatusError{SF_ERR_UNSUPPORTED, "sf_cpals: sharded handles not supported"};
+    if (t->nranks != 1 && !t->comm)
+      throw StatusError{SF_ERR_INVALID_ARG, "sf_cpals: a sharded handle needs sf_comm_attach*"};
     for (int m = 0; m < t->nmodes; ++m)
       if (!factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
     SF_CUDA(cudaSetDevice(t->device));
@@ -628,6 +701,7 @@ const char* sf_status_string(sf_status s) {
     case SF_ERR_NOT_PLANNED: return "SF_ERR_NOT_PLANNED";
     case SF_ERR_UNSUPPORTED: return "SF_ERR_UNSUPPORTED";
     case SF_ERR_CUDA: return "SF_ERR_CUDA";
+    case SF_ERR_NCCL: return "SF_ERR_NCCL";
     default: return "SF_ERR_UNKNOWN";
   }
 }

@@ -456,17 +456,53 @@ static void rowmat(const float* M, uint64_t I, int R, const float* Vinv, float* 
   SF_CUDA(cudaGetLastError());
 }
 
+// out[e] = sum_k parts[k][e] in rank order (identical on every rank)
+__global__ void sum_parts_kernel(const double* __restrict__ parts, int P, int n, double* __restrict__ out) {
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
+    double acc = 0.0;
+    for (int k = 0; k < P; ++k) acc += parts[(size_t)k * n + e];
+    out[e] = acc;
+  }
+}
+
+// Rows of Y assigned to each rank of a sharded plan for the row-local update A_n = M V^+:
+// rank k owns [row_begin_k + send_first_k, row_end_k) (sf_comm.cu exchange rule); the
+// assignment extends each owned block over the empty rows up to the next owned block, so
+// the blocks partition [0, I_n) (blk[2k], blk[2k+1]).
+static std::vector<uint64_t> assigned_blocks(const Plan& p, int P, uint64_t I) {
+  std::vector<int32_t> sendf(P), owner(P);
+  sf_exchange_map(P, p.ranges.data(), sendf.data(), owner.data());
+  std::vector<uint64_t> ob(P), nonempty(P);
+  for (int k = 0; k < P; ++k) {
+    const uint64_t b = p.ranges[2 * k], e = p.ranges[2 * k + 1];
+    ob[k] = b + (uint64_t)sendf[k];
+    nonempty[k] = e > ob[k];
+  }
+  std::vector<uint64_t> blk(2 * P);
+  uint64_t next = I;  // begin of the next non-empty owned block, scanning from the right
+  for (int k = P - 1; k >= 0; --k) {
+    if (nonempty[k]) next = ob[k];
+    blk[2 * k] = (k == 0) ? 0 : next;
+  }
+  for (int k = 0; k < P; ++k) blk[2 * k + 1] = (k + 1 < P) ? blk[2 * (k + 1)] : I;
+  return blk;
+}
+
 void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, double* fits, int* done,
            cudaStream_t s, Plan* const* plans) {
   const int N = t.nmodes;
   if (R > 64) throw StatusError{SF_ERR_UNSUPPORTED, "sf_cpals: rank must be <= 64"};
+  const bool sharded = t.nranks > 1;
+  if (sharded && !t.comm) throw StatusError{SF_ERR_INVALID_ARG, "sf_cpals: a sharded handle needs a comm"};
+  const int P = t.nranks;
   uint64_t maxI = 0;
   for (int m = 0; m < N; ++m) maxI = std::max<uint64_t>(maxI, t.dims[m]);
   DevBuf M(maxI * R * sizeof(float)), G((size_t)N * R * R * sizeof(double)), Vinv64(R * R * sizeof(double)),
-      Vinv32(R * R * sizeof(float)), scal(4 * sizeof(double));
+      Vinv32(R * R * sizeof(float)), scal(4 * sizeof(double)),
+      parts(sharded ? (size_t)P * R * R * sizeof(double) + 64 : 16);
   double* dG = G.as<double>();
   for (int m = 0; m < N; ++m) gram(factors[m], t.dims[m], R, dG + (size_t)m * R * R, s);
-  // ||X||^2 (whole tensor; this handle holds the full COO)
+  // ||X||^2 (whole tensor: every rank holds the full raw COO)
   SF_CUDA(cudaMemsetAsync(scal.p, 0, 4 * sizeof(double), s));
   dot_kernel<<<grid_of(t.nnz, 256), 256, 0, s>>>(t.val.as<float>(), nullptr, t.nnz, scal.as<double>());
   count_launch();
@@ -477,6 +513,21 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
   // [V | I] in fp64: 64 KB at R = 64, above the 48 KB default dynamic shared-memory limit
   const size_t pinv_smem = (size_t)R * 2 * R * sizeof(double);
   SF_CUDA(cudaFuncSetAttribute(pinv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pinv_smem));
+  // sharded: per mode, the rows this rank updates (Alg. 1 line 5 is row-local)
+  std::vector<std::vector<uint64_t>> blk(N);
+  if (sharded)
+    for (int n = 0; n < N; ++n) {
+      ensure_ranges(t, *plans[n], s);
+      blk[n] = assigned_blocks(*plans[n], P, t.dims[n]);
+    }
+  // sum a per-rank partial (count doubles at dst) over the ranks, in rank order
+  auto allreduce_parts = [&](double* dst, int count) {
+    std::vector<uint64_t> bytes(P, (uint64_t)count * 8), displs(P);
+    for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * count * 8;
+    t.comm->allgatherv(dst, parts.p, bytes.data(), displs.data(), s);
+    sum_parts_kernel<<<grid_of((uint64_t)count, 256), 256, 0, s>>>(parts.as<double>(), P, count, dst);
+    count_launch();
+  };
   double prev = -1.0;
   int k = 0;
   for (; k < iters; ++k) {
@@ -484,21 +535,41 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
       pinv_kernel<<<1, 256, pinv_smem, s>>>(dG, N, n, R, Vinv64.as<double>(), Vinv32.as<float>());
       count_launch();
       SF_CUDA(cudaGetLastError());
-      launch_mttkrp(t, *plans[n], cf, M.as<float>(), s);
+      const Plan& p = *plans[n];
+      // M holds Y rows [a0, a1) for the update (all of Y unsharded); the plan's out block
+      // [out_row0, out_row0 + out_rows) lies inside [a0 - 1, a1) (a shared first row is sent
+      // to its owner and zeroed by the exchange)
+      uint64_t a0 = 0, a1 = t.dims[n];
+      if (sharded) {
+        a0 = blk[n][2 * t.rank];
+        a1 = blk[n][2 * t.rank + 1];
+        SF_CUDA(cudaMemsetAsync(M.as<float>() + a0 * R, 0, (a1 - a0) * R * sizeof(float), s));
+      }
+      float* Mblk = M.as<float>() + p.out_row0 * R;
+      launch_mttkrp(t, p, cf, Mblk, s);
+      exchange_rows(t, *plans[n], Mblk, s);
+      const uint64_t I = a1 - a0;
+      const float* Mown = M.as<float>() + a0 * R;
+      float* Aown = factors[n] + a0 * R;
       // fit after the sweep needs <M_N, A_N> of the last mode
       double* dot = (n == N - 1) ? scal.as<double>() + 1 : nullptr;
       if (n == N - 1) SF_CUDA(cudaMemsetAsync(scal.as<double>() + 1, 0, 2 * sizeof(double), s));
-      if (!update_fused(M.as<float>(), t.dims[n], R, Vinv32.as<float>(), factors[n], dG + (size_t)n * R * R, dot,
-                        s)) {
-        rowmat(M.as<float>(), t.dims[n], R, Vinv32.as<float>(), factors[n], s);
-        gram(factors[n], t.dims[n], R, dG + (size_t)n * R * R, s);
+      double* Gn = dG + (size_t)n * R * R;
+      if (!update_fused(Mown, I, R, Vinv32.as<float>(), Aown, Gn, dot, s)) {
+        rowmat(Mown, I, R, Vinv32.as<float>(), Aown, s);
+        gram(Aown, I, R, Gn, s);
         if (dot) {
-          const uint64_t nl = t.dims[n] * (uint64_t)R;
-          dot_kernel<<<grid_of(nl, 256), 256, 0, s>>>(M.as<float>(), factors[n], nl, dot);
+          const uint64_t nl = I * (uint64_t)R;
+          dot_kernel<<<grid_of(nl, 256), 256, 0, s>>>(Mown, Aown, nl, dot);
           count_launch();
         }
       }
       SF_CUDA(cudaGetLastError());
+      if (sharded) {  // every rank ends with the full A_n, G_n and <M_N, A_N>
+        allgather_blocks(t, blk[n], Aown, factors[n], R, s);
+        allreduce_parts(Gn, R * R);
+        if (dot) allreduce_parts(dot, 1);
+      }
     }
     model_norm_kernel<<<1, 256, 0, s>>>(dG, N, R, scal.as<double>() + 2);
     count_launch();

@@ -22,6 +22,10 @@
 // groups; the first lane of every group issues its own bulk copy
 // (cp.async.bulk ... mbarrier::complete_tx) after declaring its bytes with
 // mbarrier.expect_tx, and lane 0 arrives once all leaders have declared.
+// Hot-row cache (SF launch hot_kb): a gathered slot's most frequent rows are
+// copied per call into one dense block (hot_fill_kernel); their records carry the row's
+// slot in that block with the slot's hot bit set, so the gathers of the hot rows touch a
+// compact, TLB- and L2-friendly region instead of rows scattered over the whole factor.
 #pragma once
 
 #include "sf_frag.cuh"
@@ -46,8 +50,9 @@ __device__ __forceinline__ uint32_t frag3_lower_chunk(const uint32_t* cb, uint32
 
 struct Frag3Params {
   const uint32_t* rec;                // kernel-order records (slot order), W words each
-  const uint32_t* rowid;              // CR records: i_n per kernel-order slot
   const float* fac[SF_MAX_MODES];     // by mode
+  int64_t hot_delta[SF_MAX_MODES];    // per gathered slot: hot block - factor, in float4 units
+  uint32_t hot_bit[SF_MAX_MODES];     // per gathered slot: the record's hot flag bit (0 = none)
   float* out;
   const uint32_t* chunk_begin;        // num_chunks + 1
   const uint64_t* chunk_tile;         // num_chunks
@@ -97,12 +102,9 @@ __device__ __forceinline__ uint32_t pk_field(uint32_t w0, uint32_t w1, uint32_t 
 }
 
 // Record formats (RF): kRecPlain [i_n, g_0 .. g_{N-2}, v, 0..] (W = 4 or 8); kRecPacked
-// (N >= 4: N bit fields in words 0..2, v in word 3); kRecCompact (non-owner N = 3 plans
-// whose gathered fields leave >= 2 of 32 bits: word 0 = fields (staged slots: the row inside
-// the tile's block) | the run delta d in the top bits (boff[0], mask bmask[0] = E):
-// d = 0 inside a run, i_n - i_n(prev) in [1, E) at a run start, E = "read p.rowid" (tile
-// starts, big jumps); word 1 = v.  A group reads p.rowid once per sub-range start.
-constexpr int kRecPlain = 0, kRecPacked = 1, kRecCompact = 2;
+// (N >= 4: N bit fields in words 0..2, v in word 3).  (8-byte compact records with run
+// deltas were measured 9 % slower on nell-2 and removed.)
+constexpr int kRecPlain = 0, kRecPacked = 1;
 
 template <int N, int R, int S, int RF>
 __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
@@ -113,8 +115,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   constexpr int GPW = 32 / LPN; // lane groups per warp
   constexpr int G = N - 1;      // gathered slots
   constexpr bool PK = RF == kRecPacked;
-  constexpr bool CR = RF == kRecCompact;
-  constexpr int W = CR ? 2 : (PK ? 4 : RecWords<N>::W);
+  constexpr int W = PK ? 4 : RecWords<N>::W;
   static_assert(!PK || N >= 4, "packed records are for N >= 4");
   constexpr int RB = R * 4;     // bytes per factor row
   constexpr int R4 = R / 4;     // float4 per factor row
@@ -132,7 +133,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   const bool leader = lane_in_group == 0;
 
   const uint32_t K = p.K;
-  const uint32_t RS = CR ? frag3_cr_region_words(K) : frag3_region_words(K, W);
+  const uint32_t RS = frag3_region_words(K, W);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw);
   const uint32_t bar_bytes = ((2u * nwarps + 1u) * 8u + 127u) & ~127u;
   uint32_t* ring = reinterpret_cast<uint32_t*>(smem_raw + bar_bytes) + (size_t)warp * kFragStages * GPW * RS;
@@ -208,8 +209,8 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
         }
       }
 #pragma unroll
-      for (int q = 0; q < S; ++q)  // CR records carry the row inside the block
-        sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (CR ? (ptrdiff_t)0 : (ptrdiff_t)row0[q] * R4);
+      for (int q = 0; q < S; ++q)
+        sbase[q] = reinterpret_cast<const float4*>(fac_smem + p.fac_off[q]) - (ptrdiff_t)row0[q] * R4;
     }
     // this group's sub-range [gs, ge) of the tile segment [a, b)
     uint32_t a = __ldg(p.chunk_begin + seg), b = __ldg(p.chunk_begin + seg_end);
@@ -222,20 +223,13 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     const uint32_t ge = frag3_group_begin(a, b - a, gam + 1, Gam);
     const uint32_t T = (__reduce_max_sync(0xFFFFFFFFu, ge - gs) + K - 1) / K;  // stages of this warp
     uint32_t* const my_region0 = ring + (size_t)group * RS;
-    // CR: stages are copied from the 16-byte-aligned record at or before s0; every stage
-    // start s0 = gs + t*K has the parity of gs (K is even), so record k sits at k + o
-    const uint32_t o = CR ? (gs & 1u) : 0u;
 
     // stage t of this warp into ring slot st: every group leader copies its own records
     auto issue = [&](uint32_t t, int st) {
       if (leader) {
         const uint32_t s0 = gs + t * K;
         if (s0 < ge) {
-          uint32_t first = s0, cnt = min(K, ge - s0);
-          if constexpr (CR) {
-            first = s0 & ~1u;
-            cnt = ((s0 + cnt + 1u) & ~1u) - first;
-          }
+          const uint32_t first = s0, cnt = min(K, ge - s0);
           const uint32_t bytes = cnt * (uint32_t)(W * 4);
           mbar_expect_tx_only(&wbar[st], bytes);
           bulk_g2s(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
@@ -270,7 +264,11 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     float4 acc0 = make_float4(0.f, 0.f, 0.f, 0.f), acc1 = acc0;
     auto gather = [&](int q, uint32_t row_idx) -> F8 {
       const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
-      const size_t row = (size_t)row_idx * R4;
+      size_t row = (size_t)row_idx * R4;
+      if (q >= S) {  // hot-row cache: the slot inside the dense hot block
+        const uint32_t hb = p.hot_bit[q];
+        if (row_idx & hb) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
+      }
       F8 r;
       if constexpr (VEC == 8) {
         if (q < S) {
@@ -327,35 +325,17 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
       const int st = (int)(it % kFragStages);
       mbar_wait(&wbar[st], (it / kFragStages) & 1u);
       const uint32_t* reg = my_region0 + (size_t)st * GPW * RS;
-      const uint32_t* reg_o = reg + 2 * o;  // CR: record 0 of this stage
       const uint32_t s0 = gs + t * K;
       const uint32_t n = (s0 < ge) ? min(K, ge - s0) : 0u;
       if (n > 0) {
         if (t == 0) {  // open the sub-range's first run
-          if constexpr (CR) {
-            // start one run early so the first record's delta d0 lands on rowid[gs]: its
-            // flush of the still-empty accumulator is harmless (adds zeros to a valid row)
-            const uint32_t d0 = reg[2 * o] >> p.boff[0];
-            cur = __ldg(p.rowid + gs);
-            if (d0 != 0u && d0 != p.bmask[0]) cur -= d0;
-          } else {
-            cur = reg[0] & p.out_mask;
-          }
+          cur = reg[0] & p.out_mask;
           if constexpr (S == 0) {
             if (p.owner && !first_shared && gs > 0) zero_rows(before, cur);  // gap rows are ours
           }
         }
         // record k of this group: [i_n, g_0 .. g_{G-1}, v]
-        // CR: i = the run delta d (0: same run)
         auto load_rec = [&](uint32_t k, uint32_t& i, uint32_t (&g)[G], float& v) {
-          if constexpr (CR) {
-            const uint2 w = *reinterpret_cast<const uint2*>(reg_o + (size_t)k * 2);
-            i = w.x >> p.boff[0];
-#pragma unroll
-            for (int q = 0; q < G; ++q) g[q] = (w.x >> p.boff[1 + q]) & p.bmask[1 + q];
-            v = __uint_as_float(w.y);
-            return;
-          }
           const uint32_t* rp = reg + (size_t)k * W;
           const uint4 w0 = lds128(rp);
           uint32_t w[W];
@@ -398,16 +378,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if constexpr (CR) {
-              if (ii[u]) {
-                flush_run(shared);
-                advanced = true;
-                if (ii[u] == p.bmask[0]) cur = __ldg(p.rowid + s0 + k + u);
-                else cur += ii[u];
-              }
-            } else if (ii[u] != cur) {
-              advance(ii[u]);
-            }
+            if (ii[u] != cur) advance(ii[u]);
             const float4 vb = make_float4(vv[u], vv[u], vv[u], vv[u]);
             f4fma_(acc0, vb, pr[u].a);
             if constexpr (VEC == 8) f4fma_(acc1, vb, pr[u].b);
@@ -424,16 +395,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
             f4mul_(pr.a, x.a);
             if constexpr (VEC == 8) f4mul_(pr.b, x.b);
           }
-          if constexpr (CR) {
-            if (i) {
-              flush_run(shared);
-              advanced = true;
-              if (i == p.bmask[0]) cur = __ldg(p.rowid + s0 + k);
-              else cur += i;
-            }
-          } else if (i != cur) {
-            advance(i);
-          }
+          if (i != cur) advance(i);
           const float4 vb = make_float4(v, v, v, v);
           f4fma_(acc0, vb, pr.a);
           if constexpr (VEC == 8) f4fma_(acc1, vb, pr.b);
@@ -526,14 +488,11 @@ void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem,
   if constexpr (N >= 4) {
     if (fp.W == 4) k = frag3_kernel<N, R, S, kRecPacked>;
   }
-  if constexpr (N == 3) {
-    if (fp.W == 2) k = frag3_kernel<N, R, S, kRecCompact>;
-  }
   // opt-in shared memory once per (device, instantiation, size): host overhead of small launches
-  static size_t smem_set[16][3] = {};
+  static size_t smem_set[16][2] = {};
   int dev = 0;
   SF_CUDA(cudaGetDevice(&dev));
-  const int v = fp.W == 2 ? 2 : (fp.W == 4 && N >= 4 ? 1 : 0);
+  const int v = (fp.W == 4 && N >= 4) ? 1 : 0;
   if (dev >= 16 || smem > smem_set[dev][v]) {
     SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (dev < 16) smem_set[dev][v] = smem;

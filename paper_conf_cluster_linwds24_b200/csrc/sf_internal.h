@@ -84,12 +84,39 @@ struct Plan {
   mutable size_t occ_smem = 0;
   mutable DevBuf carry; // A7 deterministic option: per-group carry slots (rows + partials)
   bool rec_packed = false;               // frag3 PK records (N >= 4, indices bit-packed)
-  bool rec_compact = false;              // frag3 CR records: 8 bytes [gathered fields | run-start
-                                         // bit 31, v]; i_n per slot in `rowid` (non-owner plans)
-  DevBuf rowid;                          // CR: uint32 i_n per kernel-order slot
+  // Hot-row cache (launch.hot_kb > 0): per gathered slot q with hot rows, the original row of
+  // every hot slot (hot_rows[q], hot_count[q] entries), the record flag bit (hot_bit[q]) and the
+  // slot's first row in the dense per-call copy `hot_cache` (hot_off[q]).
+  uint32_t hot_bit[SF_MAX_MODES] = {};
+  uint64_t hot_count[SF_MAX_MODES] = {};
+  uint64_t hot_off[SF_MAX_MODES] = {};
+  DevBuf hot_rows[SF_MAX_MODES];
+  mutable DevBuf hot_cache;
+  uint64_t hot_total = 0;                // rows in hot_cache
   uint32_t rec_boff[SF_MAX_MODES] = {};  // PK: bit offset of field f (slot order)
   uint32_t rec_bmask[SF_MAX_MODES] = {}; // PK: width mask of field f
+  // Multi-GPU exchange map (sf_comm.cu), built at the first exchange of this plan from every
+  // rank's touched row range: ranges[2k], ranges[2k+1] = rows [begin, end) of rank k.
+  std::vector<uint64_t> ranges;
+  bool send_first = false;    // this rank's first row is owned by a lower rank
+  std::vector<int> add_srcs;  // ranks whose first row is this rank's last row (ascending)
+  mutable DevBuf xbuf;        // exchange buffers: send (R floats) + recv (nranks * R floats)
+  // The caller's `out` block: rows [out_row0, out_row0 + out_rows) of Y (the whole Y at
+  // nranks == 1, the touched row range [row_begin, row_end) of a shard otherwise).
+  uint64_t out_row0 = 0, out_rows = 0;
   size_t device_bytes() const;
+};
+
+// Collective transport of a sharded handle (sf_comm.cu): NCCL (sf_comm_attach) or a caller
+// callback (sf_comm_attach_transport).  allgatherv: rank k contributes bytes[k] bytes from
+// `send`; every rank receives them at recv + displs[k] (device memory, stream-ordered).
+struct Comm {
+  int nranks = 1, rank = 0;
+  void* nccl = nullptr;  // ncclComm_t
+  sf_allgatherv_fn fn = nullptr;
+  void* ctx = nullptr;
+  void allgatherv(const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs, cudaStream_t s);
+  ~Comm();
 };
 
 struct Tensor {
@@ -117,6 +144,7 @@ struct Tensor {
   uint64_t pre_seg_len = 0;
   int pre_pb = 0;              // position bits
   cudaStream_t stream = nullptr;               // internal stream for planning
+  Comm* comm = nullptr;                        // sharded handles: collective transport
   ~Tensor();
 };
 
@@ -163,13 +191,6 @@ __host__ __device__ inline int rec_words_for(int N) { return (N + 1 <= 4) ? 4 : 
 __host__ __device__ __forceinline__ uint32_t frag3_region_words(uint32_t K, uint32_t W) {
   const uint32_t base = K * W;
   return ((base / 4u) % 2u == 0u) ? base + 4u : base + 8u;
-}
-
-// CR (8-byte records): a group's stage holds K records copied from a 16-byte-aligned
-// start, i.e. up to K + 2 records; stride/4 odd as above.
-__host__ __device__ __forceinline__ uint32_t frag3_cr_region_words(uint32_t K) {
-  const uint32_t base = 2u * K + 4u;
-  return ((base / 4u) % 2u == 0u) ? base + 4u : base;
 }
 
 // Records per group per stage for a launch's chunk_nnz (nonzeros per warp per stage).
@@ -222,6 +243,16 @@ inline uint32_t smem_staged_mask(const sf_launch_t& l) {
   return (l.flags & SF_LAUNCH_L2_TILES) ? 0u : l.staged_mask;
 }
 void launch_rows_op(float* Y, int R, const int64_t* rows, float* buf, int count, int op, cudaStream_t s);
+// ---- multi-GPU (sf_comm.cu) ----
+// Boundary-row exchange of a sharded plan's local block `out` (rows [row_begin, row_end)):
+// the first row goes to its owner (the lowest rank touching it) and is zeroed here; the
+// owner adds the partials in rank order.  No-op without a comm or at nranks == 1.
+void exchange_rows(Tensor& t, Plan& p, float* out, cudaStream_t s);
+// Every rank contributes rows [blk[2k], blk[2k+1]) of an I x R matrix from `local`
+// (this rank's rows starting at blk[2*rank]); full (I x R, every rank) receives them all.
+void allgather_blocks(Tensor& t, const std::vector<uint64_t>& blk, const float* local, float* full, int R,
+                      cudaStream_t s);
+void ensure_ranges(Tensor& t, Plan& p, cudaStream_t s);
 void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
                       uint32_t* const* inds, int* d_flag, cudaStream_t s);
 

@@ -128,6 +128,8 @@ struct CooParams {
   const float* val;
   const float* fac[SF_MAX_MODES];
   float* out;
+  uint64_t dims[SF_MAX_MODES];  // a nonzero with some index >= dims[m] is skipped (the streamed
+                                // path range-checks segments concurrently with this kernel)
   uint64_t nnz;
   int nmodes, mode, rank;
 };
@@ -141,15 +143,17 @@ __global__ void __launch_bounds__(256) coo_kernel(CooParams p) {
   for (uint64_t e = group; e < p.nnz; e += ngroups) {
     const float v = __ldg(p.val + e);
     float4 acc = make_float4(v, v, v, v);
+    bool ok = true;
 #pragma unroll
     for (int m = 0; m < SF_MAX_MODES; ++m) {
       if (m >= p.nmodes) break;
       if (m == p.mode) continue;
       const uint32_t im = __ldg(p.ind[m] + e);
-      acc = f4mul(acc, ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub));
+      ok = ok && im < p.dims[m];
+      if (ok) acc = f4mul(acc, ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub));
     }
     const uint32_t in = __ldg(p.ind[p.mode] + e);
-    red_add_v4(p.out + (size_t)in * R + 4 * sub, acc);
+    if (ok && in < p.dims[p.mode]) red_add_v4(p.out + (size_t)in * R + 4 * sub, acc);
   }
 }
 
@@ -161,21 +165,22 @@ __global__ void coo_generic_kernel(CooParams p) {
     const uint64_t e = t / p.rank;
     const int r = (int)(t - e * p.rank);
     float acc = __ldg(p.val + e);
-    for (int m = 0; m < p.nmodes; ++m) {
-      if (m == p.mode) continue;
-      acc *= __ldg(p.fac[m] + (size_t)__ldg(p.ind[m] + e) * p.rank + r);
+    bool ok = true;
+    for (int m = 0; m < p.nmodes && ok; ++m) {
+      const uint32_t im = __ldg(p.ind[m] + e);
+      ok = im < p.dims[m];
+      if (ok && m != p.mode) acc *= __ldg(p.fac[m] + (size_t)im * p.rank + r);
     }
-    atomicAdd(p.out + (size_t)__ldg(p.ind[p.mode] + e) * p.rank + r, acc);
+    if (ok) atomicAdd(p.out + (size_t)__ldg(p.ind[p.mode] + e) * p.rank + r, acc);
   }
 }
 
 void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* const* inds,
                 const float* vals, const float* const* factors, int rank, int mode, float* out,
                 cudaStream_t s) {
-  (void)dims;
   if (nnz == 0) return;
   CooParams p{};
-  for (int m = 0; m < nmodes; ++m) { p.ind[m] = inds[m]; p.fac[m] = factors[m]; }
+  for (int m = 0; m < nmodes; ++m) { p.ind[m] = inds[m]; p.fac[m] = factors[m]; p.dims[m] = dims[m]; }
   p.val = vals;
   p.out = out;
   p.nnz = nnz;
@@ -209,7 +214,7 @@ __global__ void rows_op_kernel(float* __restrict__ Y, int R, const int64_t* __re
   for (int c = threadIdx.x; c < R; c += blockDim.x) {
     float* y = Y + (size_t)r * R + c;
     if (op == 0) buf[(size_t)k * R + c] = *y;
-    else if (op == 1) *y += buf[(size_t)k * R + c];
+    else if (op == 1) atomicAdd(y, buf[(size_t)k * R + c]);  // several entries may target one row
     else *y = 0.f;
   }
 }
@@ -235,6 +240,28 @@ int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode) 
   return S;
 }
 
+// Hot-row cache fill: cache[begin[k] + j, :] = src[k][rows[k][j], :] (float4 per thread).
+struct HotFill {
+  const float* src[SF_MAX_MODES];
+  const uint32_t* rows[SF_MAX_MODES];
+  uint64_t begin[SF_MAX_MODES + 1];
+  int nslots;
+};
+
+__global__ void hot_fill_kernel(const HotFill h, int R4, float* __restrict__ cache) {
+  const uint64_t total = h.begin[h.nslots] * (uint64_t)R4;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += stride) {
+    const uint64_t r = e / R4;
+    const int c = (int)(e - r * R4);
+    int k = 0;
+    while (k + 1 < h.nslots && r >= h.begin[k + 1]) ++k;
+    const uint32_t src_row = __ldg(h.rows[k] + (r - h.begin[k]));
+    const float4 v = __ldg(reinterpret_cast<const float4*>(h.src[k] + (size_t)src_row * R4 * 4) + c);
+    reinterpret_cast<float4*>(cache)[e] = v;
+  }
+}
+
 static int frag3_occ(int N, int R, int S, int threads, size_t smem) {
   switch (R) {
     case 16: return frag3_occ_r16(N, S, threads, smem);
@@ -254,7 +281,6 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     fp.dims[m] = (uint32_t)t.dims[m];
   }
   fp.rec = p.rec.as<uint32_t>();
-  fp.rowid = p.rowid.as<uint32_t>();
   fp.out = out;
   fp.chunk_begin = p.chunk_begin.as<uint32_t>();
   fp.chunk_tile = p.chunk_tile.as<uint64_t>();
@@ -264,7 +290,6 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   fp.nnz = (uint32_t)p.nnz_local;
   const uint32_t gpw = (uint32_t)frag_groups_per_warp(R);
   fp.K = frag3_K((uint32_t)p.launch.chunk_nnz, gpw);
-  if (p.rec_compact) fp.K &= ~1u;  // CR stages keep the parity of the sub-range start (K even)
   fp.W = (uint32_t)p.rec_words;
   fp.out_mask = p.rec_packed ? p.rec_bmask[0] : 0xFFFFFFFFu;
   for (int f = 0; f < SF_MAX_MODES; ++f) {
@@ -273,6 +298,31 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   }
   fp.owner = owner ? 1u : 0u;
   const int S = frag_slot_order(N, n, smem_staged_mask(p.launch), fp.slot_mode);
+  if (p.hot_total) {  // hot-row cache: this call's copy of every slot's hot rows
+    HotFill hf{};
+    int k = 0;
+    for (int q = 0; q < N - 1; ++q) {
+      if (!p.hot_bit[q] || !p.hot_count[q]) continue;
+      hf.src[k] = factors[fp.slot_mode[q]];
+      hf.rows[k] = p.hot_rows[q].as<uint32_t>();
+      hf.begin[k] = p.hot_off[q];
+      ++k;
+    }
+    hf.nslots = k;
+    hf.begin[k] = p.hot_total;
+    float* cache = p.hot_cache.as<float>();
+    const uint64_t items = p.hot_total * (uint64_t)(R / 4);
+    const int g = (int)std::max<uint64_t>(1, std::min<uint64_t>((items + 255) / 256, (uint64_t)t.num_sms * 16));
+    hot_fill_kernel<<<g, 256, 0, s>>>(hf, R / 4, cache);
+    count_launch();
+    SF_CUDA(cudaGetLastError());
+    for (int q = 0; q < N - 1; ++q) {
+      fp.hot_bit[q] = p.hot_bit[q];
+      if (p.hot_bit[q])
+        fp.hot_delta[q] = (int64_t)((reinterpret_cast<intptr_t>(cache + p.hot_off[q] * (uint64_t)R) -
+                                     reinterpret_cast<intptr_t>(factors[fp.slot_mode[q]])) / 16);
+    }
+  }
   fp.l2tiles = (p.launch.flags & SF_LAUNCH_L2_TILES) ? 1u : 0u;
   uint32_t off = 0;
   for (int q = 0; q < S; ++q) {
@@ -345,9 +395,9 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   }
 }
 
-void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out,
+void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, float* out_block,
                    cudaStream_t s) {
-  const int N = t.nmodes, R = p.rank, n = p.mode;
+  const int N = t.nmodes, R = p.rank;
   const bool frag = p.launch.kernel == SF_KERNEL_FRAG && frag_supported(N, R) && p.rec_words;
   // A5: unstaged fragment plans run in owner mode (whole runs stored, gaps zeroed by
   // their owner, only run-crossing rows pre-zeroed by launch_frag3); everything else
@@ -355,18 +405,22 @@ void launch_mttkrp(const Tensor& t, const Plan& p, const float* const* factors, 
   const bool owner = frag && p.launch.staged_mask == 0 && p.nnz_local > 0 &&
                      !(p.launch.flags & SF_LAUNCH_NO_OWNER_STORES);
   const size_t row_bytes = sizeof(float) * (size_t)R;
+  // the caller's block holds rows [out_row0, out_row0 + out_rows); the kernels index Y by
+  // absolute row and only touch rows in [row_begin, row_end), inside the block
+  float* out = out_block - p.out_row0 * (size_t)R;
+  const uint64_t blk_end = p.out_row0 + p.out_rows;
   if (!owner) {
-    SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * t.dims[n], s));
-  } else {  // rows outside this shard's row range
-    if (p.row_begin > 0) SF_CUDA(cudaMemsetAsync(out, 0, row_bytes * p.row_begin, s));
-    if (p.row_end < t.dims[n])
-      SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (t.dims[n] - p.row_end), s));
+    SF_CUDA(cudaMemsetAsync(out_block, 0, row_bytes * p.out_rows, s));
+  } else {  // block rows no nonzero of this shard touches (unsharded: rows before/after)
+    if (p.row_begin > p.out_row0) SF_CUDA(cudaMemsetAsync(out_block, 0, row_bytes * (p.row_begin - p.out_row0), s));
+    if (p.row_end < blk_end)
+      SF_CUDA(cudaMemsetAsync(out + p.row_end * (size_t)R, 0, row_bytes * (blk_end - p.row_end), s));
   }
   if (p.nnz_local == 0) return;
   if (frag) return launch_frag3(t, p, factors, out, s, owner);
   uint32_t* ind[SF_MAX_MODES];
   for (int m = 0; m < N; ++m) ind[m] = p.ind[m].as<uint32_t>();
-  launch_coo(N, t.dims, p.nnz_local, ind, p.val.as<float>(), factors, R, n, out, s);
+  launch_coo(N, t.dims, p.nnz_local, ind, p.val.as<float>(), factors, R, p.mode, out, s);
 }
 
 }  // namespace sf

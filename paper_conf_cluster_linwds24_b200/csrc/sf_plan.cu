@@ -399,6 +399,60 @@ __global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32
   }
 }
 
+// ---- hot-row cache (launch.hot_kb; DESIGN.md §5 "hot-row cache") ----
+// cnt[x] = nonzeros of this plan whose gathered index (mode m) is x
+__global__ void hot_count_kernel(const uint32_t* __restrict__ ind, const uint32_t* __restrict__ perm, uint64_t n,
+                                 uint32_t* __restrict__ cnt) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride)
+    atomicAdd(cnt + __ldg(ind + __ldg(perm + k)), 1u);
+}
+
+struct HotCount {
+  const uint32_t* cnt[SF_MAX_MODES];
+  uint64_t dim[SF_MAX_MODES];
+  int n;
+  uint32_t tau[32];
+};
+
+// above[j] = rows (over every hot-enabled factor) with cnt > tau[j], for 32 thresholds at once
+__global__ void hot_above_kernel(const HotCount h, unsigned long long* __restrict__ above) {
+  __shared__ unsigned long long acc[32];
+  if (threadIdx.x < 32) acc[threadIdx.x] = 0;
+  __syncthreads();
+  uint32_t c[32];
+#pragma unroll
+  for (int j = 0; j < 32; ++j) c[j] = 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (int q = 0; q < h.n; ++q)
+    for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < h.dim[q]; x += stride) {
+      const uint32_t v = __ldg(h.cnt[q] + x);
+#pragma unroll
+      for (int j = 0; j < 32; ++j) c[j] += v > h.tau[j];
+    }
+#pragma unroll
+  for (int j = 0; j < 32; ++j) {
+    uint32_t v = c[j];
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(&acc[j], (unsigned long long)v);
+  }
+  __syncthreads();
+  if (threadIdx.x < 32 && acc[threadIdx.x]) atomicAdd(above + threadIdx.x, acc[threadIdx.x]);
+}
+
+__global__ void hot_flag_kernel(const uint32_t* __restrict__ cnt, uint64_t dim, uint32_t tau, uint32_t* __restrict__ flag) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < dim; x += stride)
+    flag[x] = __ldg(cnt + x) > tau ? 1u : 0u;
+}
+
+__global__ void hot_rows_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ slot, uint64_t dim,
+                                uint32_t tau, uint32_t* __restrict__ rows) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < dim; x += stride)
+    if (__ldg(cnt + x) > tau) rows[__ldg(slot + x)] = (uint32_t)x;
+}
+
 // frag3 records: kernel-order record k = [raw field fmap[0], ..., fmap[WK-1]] of the raw
 // AoS record perm[k] (fmap < 0: zero padding).  Slot order: i_n, gathered slots, value.
 // Packed (nfields > 0): fields f < nfields (raw word fmap[f]) are OR-ed in at bit boff[f]
@@ -407,6 +461,12 @@ struct RecParams {
   int fmap[8];
   int nfields;
   uint32_t boff[8];
+  // hot-row cache: field d (a gathered slot) with hcnt[d] != nullptr becomes
+  // hslot[d][x] | hbit[d] when the row x has hcnt[d][x] > htau
+  const uint32_t* hcnt[8];
+  const uint32_t* hslot[8];
+  uint32_t hbit[8];
+  uint32_t htau;
 };
 
 template <int WR, int WK>
@@ -427,6 +487,7 @@ __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32
       uint32_t x = 0;
 #pragma unroll
       for (int q = 0; q < WR; ++q) x = (rp.fmap[d] == q) ? w[q] : x;
+      if (rp.hcnt[d] && __ldg(rp.hcnt[d] + x) > rp.htau) x = __ldg(rp.hslot[d] + x) | rp.hbit[d];
       o[d] = x;
     }
     if (WK == 8 && rp.nfields > 0) {  // packed 16-byte record
@@ -450,60 +511,6 @@ __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32
   }
 }
 
-// CR records (8 bytes): word 0 = the gathered slots' indices bit-packed (staged slots: row
-// inside the block, idx % block_rows), word 1 = v; rowid[k] = i_n.  cr_delta_kernel then
-// writes the run delta d into the top bits (sf_frag3.cuh kRecCompact).
-struct CrParams {
-  int in_word;               // raw AoS word of i_n
-  int nslots;                // gathered slots (N - 1)
-  int slot_word[SF_MAX_MODES];
-  uint32_t slot_mod[SF_MAX_MODES];  // 0 = full index, else block rows (staged slot)
-  uint32_t boff[SF_MAX_MODES];
-  int val_word;
-};
-
-template <int WR>
-__global__ void gather_rec_cr_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
-                                     uint64_t n, CrParams cp, uint32_t* __restrict__ rec,
-                                     uint32_t* __restrict__ rowid) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)perm[k] * WR);
-    uint32_t w[WR];
-#pragma unroll
-    for (int q = 0; q < WR / 4; ++q) {
-      const uint4 v = __ldg(src + q);
-      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
-    }
-    auto word = [&](int i) {
-      uint32_t x = 0;
-#pragma unroll
-      for (int q = 0; q < WR; ++q) x = (i == q) ? w[q] : x;
-      return x;
-    };
-    uint32_t x = 0;
-    for (int q = 0; q < cp.nslots; ++q) {
-      uint32_t idx = word(cp.slot_word[q]);
-      if (cp.slot_mod[q]) idx %= cp.slot_mod[q];
-      x |= idx << cp.boff[q];
-    }
-    reinterpret_cast<uint2*>(rec)[k] = make_uint2(x, word(cp.val_word));
-    rowid[k] = word(cp.in_word);
-  }
-}
-
-__global__ void cr_delta_kernel(const uint32_t* __restrict__ rowid, uint64_t n, uint32_t shift, uint32_t esc,
-                                uint32_t* __restrict__ rec) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    uint32_t d = esc;
-    if (k > 0) {
-      const uint32_t a = rowid[k - 1], b = rowid[k];
-      d = (b == a) ? 0u : ((b > a && b - a < esc) ? b - a : esc);
-    }
-    rec[2 * k] |= d << shift;
-  }
-}
 
 struct GatherParams {
   const uint32_t* src[SF_MAX_MODES];
@@ -593,6 +600,9 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     p.row_begin = kb / t.dims[s];
     p.row_end = ke / t.dims[s] + 1;
   }
+  // the caller's out block: whole Y unsharded, the touched rows of a shard
+  p.out_row0 = t.nranks > 1 ? p.row_begin : 0;
+  p.out_rows = t.nranks > 1 ? p.row_end - p.row_begin : t.dims[mode];
   trace_mark("build: shard range");
   const bool staged_is_secondary = launch.kernel == SF_KERNEL_FRAG && launch.staged_mask == (1u << s);
   if (!staged_is_secondary) keys.release();  // else kept for the tile keys
@@ -660,61 +670,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   }
   const bool use_rec = launch.kernel == SF_KERNEL_FRAG && frag_supported(N, rank);
   p.rec_words = 0;
-  p.rec_compact = false;
-  p.rowid.release();
-  // CR records: non-owner plans (staged or L2-tiled or NO_OWNER_STORES; the owner path
-  // needs i_n at every run edge) with N = 3 whose gathered fields leave >= 2 bits for d.
-  bool compact = false;
-  int cr_bits[SF_MAX_MODES] = {};
-  if (use_rec && N == 3 && (launch.flags & SF_LAUNCH_COMPACT) && !(launch.flags & SF_LAUNCH_DETERMINISTIC) &&
-      (launch.staged_mask != 0 || (launch.flags & SF_LAUNCH_NO_OWNER_STORES))) {
-    int slot_mode[SF_MAX_MODES];
-    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
-    int total = 0;
-    for (int q = 0; q < N - 1; ++q) {
-      const int m = slot_mode[q];
-      const bool in_smem = smem_staged_mask(launch) & (1u << m);
-      cr_bits[q] = index_bits(in_smem ? (uint64_t)launch.block_rows[m] : t.dims[m]);
-      total += cr_bits[q];
-    }
-    compact = total <= 30;
-  }
-  if (use_rec && compact) {
-    int slot_mode[SF_MAX_MODES];
-    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
-    p.rec_words = 2;
-    p.rec_compact = true;
-    p.rec.alloc(nl * 8 + kPadBytes);
-    p.rowid.alloc(nl * 4 + kPadBytes);
-    SF_CUDA(cudaMemsetAsync(p.rec.as<uint32_t>() + nl * 2, 0, kPadBytes, t.stream));
-    CrParams cp{};
-    cp.in_word = mode;
-    cp.nslots = N - 1;
-    cp.val_word = N;
-    uint32_t off = 0;
-    int total = 0;
-    for (int q = 0; q < N - 1; ++q) total += cr_bits[q];
-    const uint32_t dbits = (uint32_t)std::min(16, 32 - total);
-    p.rec_boff[0] = 32u - dbits;        // run delta d in the top dbits bits
-    p.rec_bmask[0] = (1u << dbits) - 1u;  // escape value E
-    for (int q = 0; q < N - 1; ++q) {
-      const int m = slot_mode[q];
-      cp.slot_word[q] = m;
-      cp.slot_mod[q] = (smem_staged_mask(launch) & (1u << m)) ? launch.block_rows[m] : 0u;
-      cp.boff[q] = off;
-      p.rec_boff[1 + q] = off;
-      p.rec_bmask[1 + q] = (1u << cr_bits[q]) - 1u;
-      off += (uint32_t)cr_bits[q];
-    }
-    if (nl) {
-      gather_rec_cr_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, cp,
-                                                                p.rec.as<uint32_t>(), p.rowid.as<uint32_t>());
-      cr_delta_kernel<<<grid_for(nl), 256, 0, t.stream>>>(p.rowid.as<uint32_t>(), nl, p.rec_boff[0], p.rec_bmask[0],
-                                                          p.rec.as<uint32_t>());
-      count_launch(2);
-      SF_CUDA(cudaGetLastError());
-    }
-  } else if (use_rec) {
+  if (use_rec) {
     // frag3 records in slot order [i_n, staged slots, other gathered slots, value, 0...]
     const bool packed = N >= 4 && rec_packable(t);
     const int WK = packed ? 4 : rec_words_for(N);
@@ -725,15 +681,116 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     RecParams rp{};
     for (int d = 0; d < 8; ++d) rp.fmap[d] = -1;
     int slot_mode[SF_MAX_MODES];
-    frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
+    const int Ssm = frag_slot_order(N, mode, smem_staged_mask(launch), slot_mode);
     rp.fmap[0] = mode;
     for (int q = 0; q < N - 1; ++q) rp.fmap[1 + q] = slot_mode[q];
     rp.fmap[N] = N;  // value word of the raw record
     rp.nfields = 0;
-    if (packed) {  // fields in slot order, i_n at bit 0
+    // hot-row cache: eligible gathered slots are gathered from L2/HBM (not staged in shared
+    // memory, not the L2-tiled mode) and large enough for their rows to be scattered
+    bool hot_q[SF_MAX_MODES] = {};
+    std::vector<DevBuf> hcnt(SF_MAX_MODES), hslot(SF_MAX_MODES);
+    p.hot_total = 0;
+    for (int q = 0; q < SF_MAX_MODES; ++q) {
+      p.hot_bit[q] = 0;
+      p.hot_count[q] = p.hot_off[q] = 0;
+      p.hot_rows[q].release();
+    }
+    p.hot_cache.release();
+    if (launch.hot_kb > 0 && nl) {
+      int bits_used = 0;
+      if (packed)
+        for (int f = 0; f < N; ++f) bits_used += index_bits(t.dims[rp.fmap[f]]);
+      for (int q = Ssm; q < N - 1; ++q) {
+        const int m = slot_mode[q];
+        if (launch.staged_mask & (1u << m)) continue;
+        if (t.dims[m] >= (1ull << 31)) continue;
+        if (packed && bits_used + 1 > 96) continue;
+        bits_used += packed ? 1 : 0;
+        hot_q[q] = true;
+      }
+      HotCount hc{};
+      for (int q = 0; q < N - 1; ++q) {
+        if (!hot_q[q]) continue;
+        const int m = slot_mode[q];
+        hcnt[q].alloc(t.dims[m] * 4 + 16);
+        SF_CUDA(cudaMemsetAsync(hcnt[q].p, 0, t.dims[m] * 4, t.stream));
+        hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
+                                                             hcnt[q].as<uint32_t>());
+        count_launch();
+        hc.cnt[hc.n] = hcnt[q].as<uint32_t>();
+        hc.dim[hc.n] = t.dims[m];
+        ++hc.n;
+      }
+      if (hc.n) {
+        // one global threshold tau (rows with count > tau are hot) so the hot rows of every
+        // slot fit the budget: the static cache of the most frequently gathered rows
+        const uint64_t budget = (uint64_t)launch.hot_kb * 1024ull / ((uint64_t)rank * 4);
+        DevBuf above(32 * 8);
+        uint64_t dimmax = 0;
+        for (int q = 0; q < hc.n; ++q) dimmax = std::max(dimmax, hc.dim[q]);
+        auto count_above = [&](unsigned long long* h) {
+          SF_CUDA(cudaMemsetAsync(above.p, 0, 32 * 8, t.stream));
+          hot_above_kernel<<<grid_for(dimmax), 256, 0, t.stream>>>(hc, above.as<unsigned long long>());
+          count_launch();
+          SF_CUDA(cudaMemcpyAsync(h, above.p, 32 * 8, cudaMemcpyDeviceToHost, t.stream));
+          SF_CUDA(cudaStreamSynchronize(t.stream));
+        };
+        unsigned long long h[32];
+        for (int j = 0; j < 32; ++j) hc.tau[j] = (j == 31) ? 0xFFFFFFFFu : ((1u << j) - 1u);  // 0, 1, 3, 7, ...
+        count_above(h);
+        int j = 0;
+        while (j < 31 && h[j] > budget) ++j;
+        uint32_t tau = hc.tau[j];
+        if (j > 0) {  // refine inside (tau[j-1], tau[j]]
+          const uint64_t lo = (uint64_t)hc.tau[j - 1] + 1, hi = hc.tau[j];
+          for (int i = 0; i < 32; ++i) hc.tau[i] = (uint32_t)std::min<uint64_t>(hi, lo + ((hi - lo) * i + 30) / 31);
+          count_above(h);
+          for (int i = 0; i < 32; ++i)
+            if (h[i] <= budget) { tau = hc.tau[i]; break; }
+        }
+        uint64_t total = 0;
+        for (int q = 0; q < N - 1; ++q) {
+          if (!hot_q[q]) continue;
+          const int m = slot_mode[q];
+          const uint64_t I = t.dims[m];
+          hslot[q].alloc(I * 4 + 16);
+          hot_flag_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt[q].as<uint32_t>(), I, tau, hslot[q].as<uint32_t>());
+          uint32_t last_flag = 0, last_slot = 0;
+          SF_CUDA(cudaMemcpyAsync(&last_flag, hslot[q].as<uint32_t>() + I - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+          size_t tb = 0;
+          SF_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, hslot[q].as<uint32_t>(), hslot[q].as<uint32_t>(),
+                                                (int64_t)I, t.stream));
+          DevBuf tmp(tb + 16);
+          SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, tb, hslot[q].as<uint32_t>(), hslot[q].as<uint32_t>(),
+                                                (int64_t)I, t.stream));
+          SF_CUDA(cudaMemcpyAsync(&last_slot, hslot[q].as<uint32_t>() + I - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+          SF_CUDA(cudaStreamSynchronize(t.stream));
+          const uint64_t cnt = (uint64_t)last_slot + last_flag;
+          count_launch(2);
+          if (cnt == 0) continue;
+          p.hot_rows[q].alloc(cnt * 4 + 16);
+          hot_rows_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt[q].as<uint32_t>(), hslot[q].as<uint32_t>(), I, tau,
+                                                             p.hot_rows[q].as<uint32_t>());
+          count_launch();
+          p.hot_bit[q] = packed ? (1u << index_bits(I)) : 0x80000000u;
+          p.hot_count[q] = cnt;
+          p.hot_off[q] = total;
+          total += cnt;
+          rp.hcnt[1 + q] = hcnt[q].as<uint32_t>();
+          rp.hslot[1 + q] = hslot[q].as<uint32_t>();
+          rp.hbit[1 + q] = p.hot_bit[q];
+        }
+        rp.htau = tau;
+        p.hot_total = total;
+        if (total) p.hot_cache.alloc(total * rank * 4 + 64);
+        SF_CUDA(cudaGetLastError());
+      }
+    }
+    if (packed) {  // fields in slot order, i_n at bit 0 (a hot slot's field has one more bit)
       uint32_t off = 0;
       for (int f = 0; f < N; ++f) {
-        const int b = index_bits(t.dims[rp.fmap[f]]);
+        const int b = index_bits(t.dims[rp.fmap[f]]) + ((f >= 1 && p.hot_bit[f - 1]) ? 1 : 0);
         rp.boff[f] = off;
         p.rec_boff[f] = off;
         p.rec_bmask[f] = (b >= 32) ? 0xFFFFFFFFu : ((1u << b) - 1u);
@@ -752,6 +809,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       else throw StatusError{SF_ERR_UNSUPPORTED, "frag3 records: unsupported record width"};
       count_launch();
       SF_CUDA(cudaGetLastError());
+      if (p.hot_total) SF_CUDA(cudaStreamSynchronize(t.stream));  // hcnt / hslot are freed on return
     }
   } else {
     // Gather the kernel-order SoA arrays (padded for aligned bulk copies).

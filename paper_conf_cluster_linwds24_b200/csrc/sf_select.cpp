@@ -64,6 +64,9 @@ void normalize_launch(const Tensor& t, int mode, int rank, sf_launch_t& l) {
     l.flags &= ~(SF_LAUNCH_NO_OWNER_STORES | SF_LAUNCH_L2_TILES);
   }
   if (l.staged_mask == 0u) l.flags &= ~SF_LAUNCH_L2_TILES;
+  l.flags &= (SF_LAUNCH_NO_OWNER_STORES | SF_LAUNCH_DETERMINISTIC | SF_LAUNCH_L2_TILES);
+  if (l.kernel != SF_KERNEL_FRAG) l.hot_kb = 0;
+  l.hot_kb = std::min<uint32_t>(l.hot_kb, 4u << 20);  // 4 GiB
 }
 
 // Selector rules, calibrated on the sweeps in profiles/:
@@ -89,7 +92,6 @@ static sf_launch_t select_rules(const Tensor& t, const sf_features_t& f, int mod
   l.ctas_per_sm = 0;
   l.chunk_nnz = 128;
   l.staged_mask = 0;
-  l.flags = SF_LAUNCH_L1_NO_ALLOCATE;  // measured: -1..-8% time on every config swept
   if (l.kernel != SF_KERNEL_FRAG || nnz_local == 0) {
     normalize_launch(t, mode, rank, l);
     return l;
@@ -189,7 +191,6 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out) {
   base.kernel = frag_supported(t.nmodes, rank) ? SF_KERNEL_FRAG : SF_KERNEL_COO;
   base.block_threads = 512;
   base.chunk_nnz = 128;
-  base.flags = SF_LAUNCH_L1_NO_ALLOCATE;
   int n = 0;
   auto add = [&](int stage_mode, uint32_t rows, uint32_t flags) {
     sf_launch_t l = base;
@@ -226,6 +227,16 @@ struct TreeModel {
 };
 static TreeModel g_model;
 static bool g_have_model = false;
+
+// The deployed model (selector_model.json) is compiled in (build/sf_selector_model.inc,
+// written by _build.py) and installed when the library loads, so a C caller gets the same
+// launch as the tests and the bench; sf_set_selector_model replaces it (n_nodes = 0: rules).
+#include "sf_selector_model.inc"
+static const bool g_default_model_installed = [] {
+  set_selector_model(kModel_feature, kModel_threshold, kModel_left, kModel_right, kModel_value, kModelNodes,
+                     kModelFeatures);
+  return true;
+}();
 
 void set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
                         const int32_t* right, const int32_t* value, int n_nodes, int n_features) {
@@ -316,6 +327,30 @@ static bool l2_refine_enabled() {
   return !(e && e[0] == '0');
 }
 
+// ---------------------------------------------------------------------------
+// Hot-row cache (launch.hot_kb; DESIGN.md §5 "hot-row cache").  Random 128-byte row gathers
+// from a factor spread over hundreds of MB run at ~4.6 TB/s whether or not the rows hit L2,
+// while the same gathers from a dense 32 MB block run at ~15 TB/s (tools/micro/l2_hot.cu,
+// profiles/r02/micro_l2hot.txt): the scattered hot rows cost TLB reach, not DRAM bytes.
+// Copying the most frequent rows into one dense block per call (64-128 MB, a few tens of us)
+// gave 1.3-1.5x on nell-1- and amazon-shaped gathers in the microbenchmark.  Enabled when the
+// gathered factors that are neither staged nor L2-tiled total more than ~1.3x L2.
+// ---------------------------------------------------------------------------
+static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
+static constexpr uint32_t kHotKB = 128 * 1024, kHotKBTiled = 64 * 1024;
+
+static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
+  if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC)) return;
+  double gathered = 0;
+  for (int m = 0; m < t.nmodes; ++m) {
+    if (m == mode || (l.staged_mask & (1u << m))) continue;
+    const double F = (double)t.dims[m] * rank * 4.0;
+    if (F >= 16.0 * 1024 * 1024) gathered += F;
+  }
+  if (gathered < kHotMinGatheredBytes) return;
+  l.hot_kb = (l.flags & SF_LAUNCH_L2_TILES) ? kHotKBTiled : kHotKB;
+}
+
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local) {
   sf_launch_t l{};
   bool picked = false;
@@ -335,6 +370,7 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
   if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
   // the hand rule refines picks of a selector that cannot choose L2 tiles itself
   if (l2_refine_enabled() && !(picked && g_model.l2_classes)) l2_tile_refine(t, f, mode, rank, nnz_local, l);
+  hot_refine(t, mode, rank, l);
   return l;
 }
 

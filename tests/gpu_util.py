@@ -35,11 +35,16 @@ def run(dims, inds, vals, facs, R, modes=None, launch=None, device_input=True, s
                 t.set_launch(n, R, L)
             else:
                 t.plan(n, R)
-            y = torch.full((dims[n], R), float("nan"), dtype=torch.float32, device=dev)
+            info = t.plan_info(n, R)
+            # the library writes the plan's out block (all of Y unsharded, the local row block of
+            # a shard); NaN-filled so any row it fails to write is caught; embedded in a full Y
+            y = torch.full((info["out_rows"], R), float("nan"), dtype=torch.float32, device=dev)
             t.mttkrp(n, tf, y)
             torch.cuda.synchronize()
-            out[n] = y.cpu().numpy()
-            infos[n] = t.plan_info(n, R)
+            full = np.zeros((dims[n], R), np.float32)
+            full[info["out_row0"]:info["out_row0"] + info["out_rows"]] = y.cpu().numpy()
+            out[n] = full
+            infos[n] = info
     return out, infos
 
 

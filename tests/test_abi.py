@@ -40,12 +40,19 @@ def test_status_strings_and_version():
     assert sf.kernel_launches() == 0  # nothing launched on a CPU box
 
 
-def test_struct_layouts_match_header():
-    # sizes implied by include/scalfrag.h on LP64
-    assert ctypes.sizeof(sf.Launch) == 4 * 5 + 4 * 8 + 4
-    assert ctypes.sizeof(sf.Features) == 8 * 7 + 8 * 40 + 4 * 4 + 8 * 5
-    head = ctypes.sizeof(sf.Features) + ctypes.sizeof(sf.Launch)
-    assert ctypes.sizeof(sf.PlanInfo) == head + (-head % 8) + 8 * 7
+def test_struct_layouts_match_header(tmp_path):
+    """ctypes mirrors == the C compiler's layout of include/scalfrag.h (sizes and offsets)."""
+    src = tmp_path / "sz.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "scalfrag.h"\n'
+                   'int main(void) { printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(sf_launch_t), '
+                   'sizeof(sf_features_t), sizeof(sf_plan_info_t), offsetof(sf_launch_t, hot_kb), '
+                   'offsetof(sf_plan_info_t, out_rows), offsetof(sf_plan_info_t, plan_ms)); return 0; }\n')
+    exe = tmp_path / "sz"
+    subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    got = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
+    want = [ctypes.sizeof(sf.Launch), ctypes.sizeof(sf.Features), ctypes.sizeof(sf.PlanInfo),
+            sf.Launch.hot_kb.offset, sf.PlanInfo.out_rows.offset, sf.PlanInfo.plan_ms.offset]
+    assert got == want
 
 
 def test_no_oracle_in_product_path():

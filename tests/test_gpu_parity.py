@@ -52,11 +52,14 @@ def _launches(dims, n):
                          flags=sf.LAUNCH_L2_TILES)
     yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, block_threads=256,
                          staged={m: max(1, dims[m] // 3 + 1) for m in others}, flags=sf.LAUNCH_L2_TILES)
-    # compact 8-byte records (SF_LAUNCH_COMPACT, N = 3 non-owner plans): staged, L2 tiles, unstaged
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=48, staged={others[0]: 7}, flags=sf.LAUNCH_COMPACT)
+    # hot-row cache (launch.hot_kb): a budget of a few rows (only the most frequent rows are
+    # hot), every row hot, with L2 tiles, with shared-memory staging, with memset + atomics
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=48, hot_kb=1)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, hot_kb=1 << 16)
     yield sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={others[-1]: max(1, dims[others[-1]] // 4 + 1)},
-                         flags=sf.LAUNCH_COMPACT | sf.LAUNCH_L2_TILES)
-    yield sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=sf.LAUNCH_COMPACT | sf.LAUNCH_NO_OWNER_STORES)
+                         flags=sf.LAUNCH_L2_TILES, hot_kb=2)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=48, staged={others[0]: 7}, hot_kb=2)
+    yield sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=sf.LAUNCH_NO_OWNER_STORES, hot_kb=3)
 
 
 @pytest.mark.parametrize("name", ["tiny", "tiny_skew"])
@@ -77,12 +80,16 @@ def test_ranks_and_orders(cuda_device, R, dims):
     nnz = 3001  # ragged
     inds, vals = synth.gen_coo(dims, nnz, 99, zipf=(0.8,) * len(dims), val_kind="signed")
     facs = synth.gen_factors(dims, R, 77, "signed")
-    for staged, flags in ((False, 0), (True, 0), (True, sf.LAUNCH_L2_TILES), (True, sf.LAUNCH_COMPACT)):
+    for staged, flags, hot in ((False, 0, 0), (True, 0, 0), (True, sf.LAUNCH_L2_TILES, 0), (False, 0, 1),
+                               (True, sf.LAUNCH_L2_TILES, 1)):
         def L(n):
             if not staged:
-                return sf.Launch.make(kernel=FRAG, chunk_nnz=100)
-            return sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=flags,
-                                  staged={m: max(1, dims[m] // 2) for m in range(len(dims)) if m != n})
+                return sf.Launch.make(kernel=FRAG, chunk_nnz=100, hot_kb=hot)
+            # L2 tiles: one tiled mode, so the others can take hot rows
+            st = {m: max(1, dims[m] // 2) for m in range(len(dims)) if m != n}
+            if flags:
+                st = {max(st): st[max(st)]}
+            return sf.Launch.make(kernel=FRAG, chunk_nnz=100, flags=flags, staged=st, hot_kb=hot)
         Y, _ = G.run(dims, inds, vals, facs, R, launch=L)
         for n in range(len(dims)):
             G.assert_parity(Y[n], dims, inds, vals, facs, R, n)
@@ -273,9 +280,9 @@ def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
                 G.assert_parity(y.cpu().numpy(), dims, inds, vals, facs, 16, n)
 
 
-@pytest.mark.parametrize("kind", ["l2tiles", "staged", "compact"])
+@pytest.mark.parametrize("kind", ["l2tiles", "staged", "hot"])
 def test_shards_with_tiled_plans(cuda_device, kind):
-    """§8(e) with tiled plans: each shard's L2-tiled / shared-memory-tiled / compact-record
+    """§8(e) with tiled plans: each shard's L2-tiled / shared-memory-tiled / hot-row-cache
     plan covers only its slice of the matricized order; the P partial outputs sum to the
     full result exactly (integer data) and to the oracle; host input (upload || presort)."""
     dims, R = (150, 110, 90), 32
@@ -283,9 +290,9 @@ def test_shards_with_tiled_plans(cuda_device, kind):
     facs = synth.gen_factors(dims, R, 32, "int")
     for n in range(3):
         others = [m for m in range(3) if m != n]
-        flags = {"l2tiles": sf.LAUNCH_L2_TILES, "staged": 0, "compact": sf.LAUNCH_COMPACT}[kind]
+        flags = {"l2tiles": sf.LAUNCH_L2_TILES, "staged": 0, "hot": sf.LAUNCH_L2_TILES}[kind]
         L = sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={others[-1]: max(1, dims[others[-1]] // 3)},
-                           flags=flags)
+                           flags=flags, hot_kb=2 if kind == "hot" else 0)
         Yfull, _ = oracle.mttkrp(dims, inds, vals, facs, R, n)
         for P in (2, 5):
             acc = np.zeros_like(Yfull)

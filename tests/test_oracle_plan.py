@@ -97,3 +97,25 @@ def test_features_brute():
         assert np.array_equal(f["slice_hist"], h)
         assert f["slice_ratio"] == len(sl) / dims[n]
         assert f["fiber_ratio"] == len(fb) / len(sl)
+
+
+def _golden_plan():
+    import json
+    import os
+    return json.load(open(os.path.join(os.path.dirname(__file__), "golden", "plan_chunks_shards.json")))
+
+
+@pytest.mark.parametrize("case", _golden_plan()["chunks"], ids=lambda c: str(c["tiles"])[:24] + f"/C{c['C']}")
+def test_chunks_golden(case):
+    """Hand-computed chunk lists (tests/golden/plan_chunks_shards.json, R9)."""
+    got = plan.chunks(np.array(case["tiles"], dtype=np.uint64), case["C"])
+    assert got.tolist() == case["expect"], case["why"]
+
+
+@pytest.mark.parametrize("case", _golden_plan()["shard_range"], ids=lambda c: f"{c['nnz']}/{c['P']}")
+def test_shard_range_golden(case):
+    """Hand-computed floor(p*nnz/P) cuts, incl. the nell-1 / amazon 8-GPU cuts."""
+    P = case["P"]
+    got = [plan.shard_range(case["nnz"], P, p) for p in range(P)]
+    cuts = case["cuts"]
+    assert got == [(cuts[p], cuts[p + 1]) for p in range(P)], case["why"]

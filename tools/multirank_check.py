@@ -1,6 +1,10 @@
-"""Run under torchrun (any world size; SF_SAME_GPU=1 puts every rank on cuda:0 with gloo):
-each rank plans its shard of every mode, runs sf_mttkrp, exchanges boundary rows, and the
-gathered row-sharded Y must equal the single-rank result bit-exactly (integer data)."""
+"""Run under torchrun (any world size; SF_SAME_GPU=1 puts every rank on cuda:0 with the gloo
+transport, else NCCL): each rank plans its shard of every mode, runs sf_mttkrp (which ends with
+the boundary exchange inside libscalfrag), and
+  * the row-sharded local blocks must equal the single-rank result bit-exactly on the rows
+    each rank owns and be 0 elsewhere (integer data), every row owned at most once;
+  * sf_allgather_rows must rebuild the full single-rank Y on every rank;
+  * sf_cpals on the shards must give the same fits and factors as on one rank."""
 import os
 import sys
 
@@ -11,7 +15,7 @@ import torch.distributed as dist
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import synth  # noqa: E402
 import paper_conf_cluster_linwds24_b200 as sf  # noqa: E402
-from paper_conf_cluster_linwds24_b200.dist import BoundaryExchange, owner_maps  # noqa: E402
+from paper_conf_cluster_linwds24_b200 import dist as sfdist  # noqa: E402
 
 
 def main():
@@ -19,40 +23,72 @@ def main():
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
     dev = torch.device("cuda", 0 if same else int(os.environ.get("LOCAL_RANK", 0)))
     torch.cuda.set_device(dev)
-    dist.init_process_group("gloo" if same else "nccl")
+    dist.init_process_group("gloo" if same else "nccl", device_id=None if same else dev)
     dims, R = (3000, 2000, 1500), 32
+    # heavy first mode so one row spans several shards at world >= 3
     inds, vals = synth.gen_coo_device(dims, 2_000_000, 77, zipf=(1.3, 0.5, 0.5), val_kind="int")
     facs = synth.gen_factors_device(dims, R, 78, "int")
     ok = True
+    msgs = []
     for n in range(3):
         with sf.Tensor(dims, inds, vals) as T1:
             T1.plan(n, R)
             full = torch.empty((dims[n], R), device=dev)
             T1.mttkrp(n, facs, full)
         with sf.Tensor(dims, inds, vals) as T:
-            T.set_shard(world, rank)
+            sfdist.attach(T, world, rank)
             T.plan(n, R)
             info = T.plan_info(n, R)
-            y = torch.empty((dims[n], R), device=dev)
+            y = torch.full((info["out_rows"], R), float("nan"), device=dev)
             T.mttkrp(n, facs, y)
-            ex = BoundaryExchange(world, rank, R, dev, host_staging=same)
-            ex.combine(y, info["row_begin"], info["row_end"])
             torch.cuda.synchronize()
             ranges = [None] * world
             dist.all_gather_object(ranges, (info["row_begin"], info["row_end"]))
-            zero_rows, _ = owner_maps(ranges)
+            send_first, owner = sf.exchange_map(ranges)
             lo, hi = ranges[rank]
-            mine = torch.zeros(dims[n], dtype=torch.bool, device=dev)
-            mine[lo:hi] = True
-            for r in zero_rows[rank]:
-                mine[r] = False
-            ok &= bool(torch.equal(y[mine], full[mine]))
-            ok &= bool((y[~mine] == 0).all())
-            cover = mine.to(torch.int32).cpu()
+            mine = torch.zeros(hi - lo, dtype=torch.bool, device=dev)
+            mine[:] = True
+            if send_first[rank] and hi > lo:
+                mine[0] = False
+            yf = full[lo:hi]
+            ok_n = bool(torch.equal(y[mine], yf[mine])) and bool((y[~mine] == 0).all())
+            cover = torch.zeros(dims[n], dtype=torch.int32)
+            cover[lo:hi] = mine.to(torch.int32).cpu()
             dist.all_reduce(cover)
-            ok &= bool((cover[torch.from_numpy(np.arange(dims[n]))] <= 1).all())
+            ok_n &= bool((cover <= 1).all())
+            # replicated Y from the row-sharded blocks
+            rep = torch.empty((dims[n], R), device=dev)
+            T.allgather_rows(n, y, rep)
+            torch.cuda.synchronize()
+            ok_n &= bool(torch.equal(rep, full))
+            if not ok_n:
+                msgs.append(f"mode {n} rank {rank} ranges {ranges}")
+            ok &= ok_n
+    # CP-ALS on the shards == CP-ALS on one rank (same initial factors)
+    fd = [torch.rand((d, 16), device=dev, generator=torch.Generator(device=dev).manual_seed(5 + m))
+          for m, d in enumerate(dims)]
+    vals_f = torch.rand(vals.shape, device=dev, generator=torch.Generator(device=dev).manual_seed(9))
+    with sf.Tensor(dims, inds, vals_f) as T1:
+        a1 = [f.clone() for f in fd]
+        fits1 = T1.cp_als(a1, iters=3)
+    with sf.Tensor(dims, inds, vals_f) as T:
+        sfdist.attach(T, world, rank)
+        a2 = [f.clone() for f in fd]
+        fits2 = T.cp_als(a2, iters=3)
+    torch.cuda.synchronize()
+    for k in range(3):
+        if abs(fits1[k] - fits2[k]) > 1e-6:
+            ok = False
+            msgs.append(f"cpals fit {k}: {fits1[k]} vs {fits2[k]}")
+    for m in range(3):
+        rel = float((a1[m] - a2[m]).abs().max() / a1[m].abs().max())
+        if not rel < 1e-3:
+            ok = False
+            msgs.append(f"cpals factor {m}: rel diff {rel}")
     flag = torch.tensor([1 if ok else 0])
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+    for mm in msgs:
+        print(mm, flush=True)
     if rank == 0:
         print("MULTIRANK OK" if flag.item() == 1 else "MULTIRANK MISMATCH", flush=True)
     dist.destroy_process_group()
