@@ -28,6 +28,10 @@
  *     `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
  *   - Asynchronous kernel faults surface at the caller's next synchronization
  *     (as in cuBLAS); the library itself synchronizes only where stated.
+ *   - Environment: the library reads nothing but SF_DEBUG, a debug / A-B aid that is never
+ *     needed in production: a comma-separated list of trace (sf_plan phase marks on
+ *     stderr), no_presort, no_l2tiles, no_hot, no_cpals_fused (disable one optimisation)
+ *     and l2_revisit=<x> (calibration of the L2-tile rule).
  */
 #ifndef SCALFRAG_H
 #define SCALFRAG_H
@@ -221,9 +225,12 @@ sf_status sf_mttkrp(sf_tensor_t t, int mode, const float* const* factors, int ra
                     void* stream);
 
 /* One-shot streamed path (the paper's pipeline; §8(a) A8 (ii)):
- * host COO is uploaded in `segments` pieces over `streams` streams while the
- * nnz-parallel kernel consumes finished segments; Y (device) is overwritten.
- * No handle, no sort.  Synchronizes before returning. */
+ * host COO is uploaded in `segments` pieces over `streams` streams while finished
+ * segments are computed; Y (device, I_mode x rank) is overwritten.  No handle.  For rank
+ * 16/32/64 each segment is sorted by i_n on the device and reduced in registers along its
+ * runs (one atomic per run piece: heavy rows keep short fp32 chains); other ranks use one
+ * atomic per nonzero.  Synchronizes before returning.  On SF_ERR_INDEX_OUT_OF_RANGE the
+ * offending nonzeros were skipped and Y holds the sum of the others. */
 sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
                              const uint32_t* const* inds_host, const float* vals_host,
                              const float* const* factors, int rank, int mode, float* out,

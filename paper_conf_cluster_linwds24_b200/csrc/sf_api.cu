@@ -28,12 +28,28 @@ static thread_local std::string g_err;
 
 void set_error(const std::string& msg) { g_err = msg; }
 
+const char* debug_opt(const char* key) {
+  static thread_local std::string val;
+  const char* e = std::getenv("SF_DEBUG");
+  if (!e || !*e) return nullptr;
+  const std::string all(e);
+  const size_t klen = strlen(key);
+  size_t pos = 0;
+  while (pos <= all.size()) {
+    size_t end = all.find(',', pos);
+    if (end == std::string::npos) end = all.size();
+    const std::string item = all.substr(pos, end - pos);
+    if (item.compare(0, klen, key) == 0 && (item.size() == klen || item[klen] == '=')) {
+      val = item.size() == klen ? std::string() : item.substr(klen + 1);
+      return val.c_str();
+    }
+    pos = end + 1;
+  }
+  return nullptr;
+}
+
 void trace_mark(const char* phase) {
-  static const bool on = [] {
-    const char* e = std::getenv("SF_PLAN_TRACE");
-    return e && e[0] == '1';
-  }();
-  if (!on) return;
+  if (!debug_opt("trace")) return;
   static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
   const auto now = std::chrono::steady_clock::now();
   fprintf(stderr, "[sf trace] %-24s +%.3f ms\n", phase, std::chrono::duration<double, std::milli>(now - last).count());
@@ -578,6 +594,14 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
     segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, nnz)));
     streams = std::max(1, std::min(streams, segments));
     const uint64_t seg_len = (nnz + segments - 1) / segments;
+    // sorted segments (A8 (ii) + pre-reduction): rank 16/32/64 sort every segment by i_n on
+    // the device and reduce runs in registers; other ranks keep one atomic per nonzero
+    const bool sorted = seg_sorted_supported(rank);
+    int kbits = 1;
+    for (uint64_t x = dims[mode] - 1; x; x >>= 1) ++kbits;
+    const size_t raw_bytes = (size_t)seg_len * 4 * (nmodes + 1) + 64;
+    const size_t sort_temp = sorted ? seg_sort_temp_bytes(seg_len, kbits) : 0;
+    const size_t sort_bytes = sorted ? (size_t)seg_len * 12 + 3 * 64 + sort_temp : 0;
     std::vector<cudaStream_t> st(streams);
     for (auto& s : st) SF_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     std::vector<DevBuf> ring;
@@ -585,7 +609,7 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
     cudaEvent_t zeroed = nullptr;
     try {
       ring.reserve(streams);
-      for (int s = 0; s < streams; ++s) ring.emplace_back((size_t)seg_len * 4 * (nmodes + 1) + 64);
+      for (int s = 0; s < streams; ++s) ring.emplace_back(raw_bytes + sort_bytes);
       SF_CUDA(cudaEventCreateWithFlags(&zeroed, cudaEventDisableTiming));
       SF_CUDA(cudaMemsetAsync(flag.p, 0, 16, st[0]));
       SF_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * dims[mode] * (size_t)rank, st[0]));
@@ -605,7 +629,18 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
         float* dv = reinterpret_cast<float*>(base + (size_t)nmodes * seg_len * 4);
         SF_CUDA(cudaMemcpyAsync(dv, vals_host + a, len * 4, cudaMemcpyHostToDevice, st[s]));
         validate_indices(nmodes, dims, len, di, flag.as<int>(), st[s]);
-        launch_coo(nmodes, dims, len, di, dv, factors, rank, mode, out, st[s]);
+        if (sorted) {
+          char* sb = base + raw_bytes;
+          uint32_t* skey = reinterpret_cast<uint32_t*>(sb);
+          uint32_t* spos = reinterpret_cast<uint32_t*>(sb + ((seg_len * 4 + 63) & ~(size_t)63));
+          uint32_t* iota = reinterpret_cast<uint32_t*>(sb + 2 * ((seg_len * 4 + 63) & ~(size_t)63));
+          void* temp = sb + 3 * ((seg_len * 4 + 63) & ~(size_t)63);
+          launch_iota(iota, len, st[s]);
+          seg_sort(di[mode], skey, iota, spos, len, kbits, temp, sort_temp, st[s]);
+          launch_seg_sorted(nmodes, dims, len, di, dv, skey, spos, factors, rank, mode, out, st[s]);
+        } else {
+          launch_coo(nmodes, dims, len, di, dv, factors, rank, mode, out, st[s]);
+        }
       }
       for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
       int bad = 0;

@@ -429,8 +429,7 @@ static void update_one(const float* M, uint64_t I, const float* Vinv, float* A, 
 
 static bool update_fused(const float* M, uint64_t I, int R, const float* Vinv, float* A, double* G, double* dot,
                          cudaStream_t s) {
-  const char* env = std::getenv("SF_CPALS_FUSED");  // "0": separate kernels (A/B)
-  if (env && env[0] == '0') return false;
+  if (debug_opt("no_cpals_fused")) return false;  // SF_DEBUG A/B: separate kernels
   SF_CUDA(cudaMemsetAsync(G, 0, sizeof(double) * R * R, s));
   switch (R) {
     case 16: update_one<16>(M, I, Vinv, A, G, dot, s); break;

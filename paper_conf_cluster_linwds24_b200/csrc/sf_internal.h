@@ -14,7 +14,11 @@
 
 namespace sf {
 
-// SF_PLAN_TRACE=1: host wall-clock phase marks of sf_plan on stderr (profiling aid).
+// The library's only environment input (debug / A-B aid, include/scalfrag.h "SF_DEBUG"):
+// SF_DEBUG is a comma-separated list of key or key=value; debug_opt returns the value of
+// `key` ("" for a bare key) or nullptr when absent.  Read at every call (in-process A/B).
+const char* debug_opt(const char* key);
+// SF_DEBUG=trace: host wall-clock phase marks of sf_plan on stderr (profiling aid).
 void trace_mark(const char* phase);
 
 // Thread-local error detail + status plumbing.
@@ -236,6 +240,14 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
                 const float* vals, const float* const* factors, int rank, int mode, float* out,
                 cudaStream_t s);
 bool frag_supported(int nmodes, int rank);
+bool seg_sorted_supported(int rank);
+void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* const* inds,
+                       const float* vals, const uint32_t* skey, const uint32_t* spos, const float* const* factors,
+                       int rank, int mode, float* out, cudaStream_t s);
+void launch_iota(uint32_t* x, uint64_t n, cudaStream_t s);
+size_t seg_sort_temp_bytes(uint64_t len, int bits);
+void seg_sort(const uint32_t* keys_in, uint32_t* keys_out, const uint32_t* vals_in, uint32_t* vals_out, uint64_t len,
+              int bits, void* temp, size_t temp_bytes, cudaStream_t s);
 // gathered slot order of a plan: staged modes ascending, then the other gathered modes
 int frag_slot_order(int nmodes, int mode, uint32_t staged_mask, int* slot_mode);
 // modes whose factor blocks are copied into shared memory (L2-tiled plans stage none)

@@ -203,6 +203,104 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
 }
 
 // ---------------------------------------------------------------------------
+// Sorted-segment kernel (the one-shot streamed path, §8(a) A8 (ii)).  A segment of the raw
+// COO, once on the device, is sorted by i_n (keys = i_n, payload = position in the segment);
+// each lane group then walks a contiguous range of the sorted positions, accumulating in
+// registers while i_n is unchanged and adding one vector atomic per run piece -- a heavy row
+// gets one atomic per (segment, group) instead of one per nonzero, which keeps the fp32
+// chain short (SURVEY C-2: amazon's 1.2e8-nonzero row).  Out-of-range nonzeros are skipped
+// (the segment's range check runs concurrently and is reported at the end).
+// ---------------------------------------------------------------------------
+struct SegParams {
+  const uint32_t* ind[SF_MAX_MODES];  // segment arrays (input order)
+  const float* val;
+  const uint32_t* skey;               // sorted i_n
+  const uint32_t* spos;               // position of the sorted slot in the segment
+  const float* fac[SF_MAX_MODES];
+  float* out;
+  uint64_t dims[SF_MAX_MODES];
+  uint64_t len;
+  int nmodes, mode;
+};
+
+template <int R>
+__global__ void __launch_bounds__(256) seg_sorted_kernel(SegParams p) {
+  constexpr int LPN = R / 4;
+  const int sub = threadIdx.x % LPN;
+  const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / LPN;
+  const uint64_t G = ((uint64_t)gridDim.x * blockDim.x) / LPN;
+  const uint64_t k0 = g * p.len / G, k1 = (g + 1) * p.len / G;
+  uint32_t cur = 0xFFFFFFFFu;
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (uint64_t k = k0; k < k1; ++k) {
+    const uint32_t i = __ldg(p.skey + k);
+    const uint32_t e = __ldg(p.spos + k);
+    if (i != cur) {
+      if (cur != 0xFFFFFFFFu) red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
+      acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      cur = i < p.dims[p.mode] ? i : 0xFFFFFFFFu;
+    }
+    if (cur == 0xFFFFFFFFu) continue;
+    const float v = __ldg(p.val + e);
+    float4 prod = make_float4(v, v, v, v);
+    bool ok = true;
+#pragma unroll
+    for (int m = 0; m < SF_MAX_MODES; ++m) {
+      if (m >= p.nmodes) break;
+      if (m == p.mode) continue;
+      const uint32_t im = __ldg(p.ind[m] + e);
+      ok = ok && im < p.dims[m];
+      if (ok) prod = f4mul(prod, ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub));
+    }
+    if (ok) {
+      acc.x += prod.x; acc.y += prod.y; acc.z += prod.z; acc.w += prod.w;
+    }
+  }
+  if (cur != 0xFFFFFFFFu) red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
+}
+
+bool seg_sorted_supported(int rank) { return rank == 16 || rank == 32 || rank == 64; }
+
+void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* const* inds,
+                       const float* vals, const uint32_t* skey, const uint32_t* spos, const float* const* factors,
+                       int rank, int mode, float* out, cudaStream_t s) {
+  if (len == 0) return;
+  SegParams p{};
+  for (int m = 0; m < nmodes; ++m) { p.ind[m] = inds[m]; p.fac[m] = factors[m]; p.dims[m] = dims[m]; }
+  p.val = vals;
+  p.skey = skey;
+  p.spos = spos;
+  p.out = out;
+  p.len = len;
+  p.nmodes = nmodes;
+  p.mode = mode;
+  // ~64 nonzeros per lane group: long runs per group, enough groups to fill the GPU
+  auto grid_for = [&](int lpn) {
+    const uint64_t groups = std::max<uint64_t>(1, len / 64);
+    return (int)std::max<uint64_t>(1, std::min<uint64_t>((groups * lpn + 255) / 256, (uint64_t)148 * 16));
+  };
+  switch (rank) {
+    case 16: seg_sorted_kernel<16><<<grid_for(4), 256, 0, s>>>(p); break;
+    case 32: seg_sorted_kernel<32><<<grid_for(8), 256, 0, s>>>(p); break;
+    default: seg_sorted_kernel<64><<<grid_for(16), 256, 0, s>>>(p); break;
+  }
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+__global__ void iota_kernel(uint32_t* __restrict__ x, uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    x[i] = (uint32_t)i;
+}
+
+void launch_iota(uint32_t* x, uint64_t n, cudaStream_t s) {
+  if (!n) return;
+  iota_kernel<<<(int)std::min<uint64_t>((n + 255) / 256, 148 * 16), 256, 0, s>>>(x, n);
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+// ---------------------------------------------------------------------------
 // Boundary-row helper (multi-GPU exchange, §8(e))
 // ---------------------------------------------------------------------------
 __global__ void rows_op_kernel(float* __restrict__ Y, int R, const int64_t* __restrict__ rows,

@@ -84,8 +84,7 @@ __global__ void split_key_kernel(const uint64_t* __restrict__ c, uint64_t n, int
 static void aos_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t st);  // below
 
 bool presort_begin(Tensor& t, uint64_t seg_len) {
-  const char* env = std::getenv("SF_PRESORT");
-  if (env && env[0] == '0') return false;
+  if (debug_opt("no_presort")) return false;  // SF_DEBUG A/B
   const uint64_t n = t.nnz;
   if (n < 2 || seg_len >= n || n >= (1ull << 30)) return false;
   const int pb = std::max(1, bitlen(n - 1));
@@ -920,6 +919,24 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   p.plan_ms = ms;
   cudaEventDestroy(ev0);
   cudaEventDestroy(ev1);
+}
+
+// Segment sort of the one-shot streamed path (sf_mttkrp_streamed): stable radix sort of a
+// segment's i_n (the low `bits` bits) with the segment positions as payload.
+size_t seg_sort_temp_bytes(uint64_t len, int bits) {
+  size_t tb = 0;
+  SF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint32_t*)nullptr, (uint32_t*)nullptr,
+                                          (const uint32_t*)nullptr, (uint32_t*)nullptr, (int64_t)len, 0,
+                                          std::max(1, bits)));
+  return tb;
+}
+
+void seg_sort(const uint32_t* keys_in, uint32_t* keys_out, const uint32_t* vals_in, uint32_t* vals_out, uint64_t len,
+              int bits, void* temp, size_t temp_bytes, cudaStream_t s) {
+  if (!len) return;
+  SF_CUDA(cub::DeviceRadixSort::SortPairs(temp, temp_bytes, keys_in, keys_out, vals_in, vals_out, (int64_t)len, 0,
+                                          std::max(1, bits), s));
+  count_launch((uint64_t)((std::max(1, bits) + 7) / 8) + 1);
 }
 
 }  // namespace sf

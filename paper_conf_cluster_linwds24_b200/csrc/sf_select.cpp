@@ -293,8 +293,8 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
       f.nnz == 0)
     return;
   const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
-  const char* env = std::getenv("SF_L2_MAX_REVISIT");  // calibration override of kL2MaxRevisit
-  const double max_revisit = env ? std::atof(env) : kL2MaxRevisit;
+  const char* env = debug_opt("l2_revisit");  // SF_DEBUG calibration override of kL2MaxRevisit
+  const double max_revisit = (env && *env) ? std::atof(env) : kL2MaxRevisit;
   int best = -1;
   double bestF = 0;
   for (int m = 0; m < t.nmodes; ++m) {
@@ -323,8 +323,7 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
 }
 
 static bool l2_refine_enabled() {
-  const char* e = std::getenv("SF_L2_TILES");  // "0": keep the selector's unstaged pick (A/B)
-  return !(e && e[0] == '0');
+  return !debug_opt("no_l2tiles");  // SF_DEBUG A/B: keep the selector's unstaged pick
 }
 
 // ---------------------------------------------------------------------------
@@ -332,22 +331,24 @@ static bool l2_refine_enabled() {
 // from a factor spread over hundreds of MB run at ~4.6 TB/s whether or not the rows hit L2,
 // while the same gathers from a dense 32 MB block run at ~15 TB/s (tools/micro/l2_hot.cu,
 // profiles/r02/micro_l2hot.txt): the scattered hot rows cost TLB reach, not DRAM bytes.
-// Copying the most frequent rows into one dense block per call (64-128 MB, a few tens of us)
-// gave 1.3-1.5x on nell-1- and amazon-shaped gathers in the microbenchmark.  Enabled when the
-// gathered factors that are neither staged nor L2-tiled total more than ~1.3x L2.
+// Copying the most frequent rows into one dense block per call (a few tens of us) gave
+// 1.3-1.5x on nell-1- and amazon-shaped gathers in the microbenchmark; in frag3 on nell-1
+// 16-32 MB blocks are best (mode 2: 7.01 -> 4.68 ms; 128 MB 4.86, 256 MB 6.02;
+// profiles/r02/hot_sweep_*.jsonl).  Enabled when the gathered factors that are neither
+// staged nor L2-tiled total more than ~1.3x L2.
 // ---------------------------------------------------------------------------
 static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
-static constexpr uint32_t kHotKB = 128 * 1024, kHotKBTiled = 64 * 1024;
+static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 32 * 1024;
 
 static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
-  if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC)) return;
+  if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC) || l.staged_mask != 0) return;
   double gathered = 0;
   for (int m = 0; m < t.nmodes; ++m) {
     if (m == mode || (l.staged_mask & (1u << m))) continue;
     const double F = (double)t.dims[m] * rank * 4.0;
     if (F >= 16.0 * 1024 * 1024) gathered += F;
   }
-  if (gathered < kHotMinGatheredBytes) return;
+  if (gathered < kHotMinGatheredBytes || debug_opt("no_hot")) return;  // SF_DEBUG A/B
   l.hot_kb = (l.flags & SF_LAUNCH_L2_TILES) ? kHotKBTiled : kHotKB;
 }
 
@@ -369,8 +370,11 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
   }
   if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
   // the hand rule refines picks of a selector that cannot choose L2 tiles itself
-  if (l2_refine_enabled() && !(picked && g_model.l2_classes)) l2_tile_refine(t, f, mode, rank, nnz_local, l);
+  // hot-row cache first: where it applies to an unstaged pick it beats L2 tiles (deli-4d 1.2-1.8x,
+  // flickr-3d 1.2x per mode) or ties them within 3 % (nell-1), profiles/r02/hot_sweep_g06.jsonl
   hot_refine(t, mode, rank, l);
+  if (l.hot_kb == 0 && l2_refine_enabled() && !(picked && g_model.l2_classes))
+    l2_tile_refine(t, f, mode, rank, nnz_local, l);
   return l;
 }
 

@@ -53,8 +53,8 @@ def grid(dims, n, R, quick):
         opts = {m: sorted(set(row_opts + ([dims[m]] if dims[m] <= 2048 else []))) for m in st}
         rows_choices = [()] if not st else itertools.product(*[opts[m] for m in st])
         for rows in rows_choices:
-            for C, th, fl in itertools.product(chunks, threads, (2,) if not st else (10,)):
-                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl,
+            for C, th, fl in itertools.product(chunks, threads, (0,) if not st else (8,)):
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl & ~8,
                        "staged": {m: min(r, dims[m]) for m, r in zip(st, rows)}}
     # L2-tiled plans (SF_LAUNCH_L2_TILES = 64): one gathered factor >= 16 MB in 16/32/64 MB blocks
     for m in others:
@@ -66,7 +66,38 @@ def grid(dims, n, R, quick):
             if rows >= dims[m]:
                 continue
             for C, th in itertools.product(chunks, threads):
-                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": 2 | 64, "staged": {m: rows}}
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": 64, "staged": {m: rows}}
+    yield {"kernel": 1}
+
+
+def grid_sparse(dims, n, R):
+    """Exhaustive grid for hyper-sparse modes (gathered factors >> L2, SURVEY C-6): unstaged
+    (owner stores / memset + atomics), L2 tiles of every gathered factor >= 16 MB in
+    16/32/64/128 MB blocks (one mode, and two modes), each with hot-row caches of
+    0/8/16/32/64/128 MB, x chunk length x threads; shared-memory block staging for contrast."""
+    others = [m for m in range(len(dims)) if m != n]
+    hots = [0, 8, 16, 32, 64, 128]
+    for fl in (0, 4):
+        for C, th, hb in itertools.product([64, 128, 256], [512, 1024], hots):
+            yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": fl, "staged": {}, "hot_kb": hb * 1024}
+    big = [m for m in others if dims[m] * R * 4 >= 16 * 2**20]
+    for m in big:
+        for mb in (16, 32, 64, 128):
+            rows = int(mb * 2**20 / (R * 4))
+            if rows >= dims[m]:
+                continue
+            for C, th, hb in itertools.product([128, 256], [512, 1024], hots):
+                yield {"kernel": 2, "block_threads": th, "chunk_nnz": C, "flags": 64, "staged": {m: rows},
+                       "hot_kb": hb * 1024}
+    for a, b in itertools.combinations(big, 2):
+        for mb in (32, 64):
+            ra, rb = (min(int(mb * 2**20 / (R * 4)), dims[x]) for x in (a, b))
+            for hb in (0, 16, 32):
+                yield {"kernel": 2, "block_threads": 512, "chunk_nnz": 128, "flags": 64, "staged": {a: ra, b: rb},
+                       "hot_kb": hb * 1024}
+    for m in others:
+        for rows in (256, 512):
+            yield {"kernel": 2, "block_threads": 512, "chunk_nnz": 128, "flags": 0, "staged": {m: min(rows, dims[m])}}
     yield {"kernel": 1}
 
 
@@ -75,6 +106,7 @@ def main():
     ap.add_argument("--config", default="nell2")
     ap.add_argument("--modes", default=None)
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--sparse", action="store_true", help="the hyper-sparse grid (grid_sparse)")
     ap.add_argument("--out", default=None)
     ap.add_argument("--only-staged", default=None, help="restrict to this staged set, e.g. '1:256'")
     args = ap.parse_args()
@@ -82,10 +114,12 @@ def main():
 
     import paper_conf_cluster_linwds24_b200 as sf
     cfg = synth.CONFIGS[args.config]
-    inds, vals = synth.config_tensor(cfg)
-    facs = [torch.from_numpy(f).cuda() for f in synth.config_factors(cfg)]
+    inds, vals = synth.config_tensor_device(cfg)
+    facs = synth.config_factors_device(cfg)
     R = cfg.rank
-    T = sf.Tensor(cfg.dims, [torch.from_numpy(a.view(np.int32)) for a in inds], torch.from_numpy(vals))
+    T = sf.Tensor(cfg.dims, inds, vals)
+    del inds, vals
+    torch.cuda.empty_cache()
     modes = [int(x) for x in args.modes.split(",")] if args.modes else range(cfg.nmodes)
     outf = open(args.out, "w") if args.out else None
     flops = cfg.nmodes * cfg.nnz * R
@@ -97,11 +131,11 @@ def main():
             kernel=2 if pick["kernel"] == "frag" else 1, block_threads=pick["block_threads"],
             ctas_per_sm=pick["ctas_per_sm"], chunk_nnz=pick["chunk_nnz"],
             staged={m: r for m, r in enumerate(pick["block_rows"]) if pick["staged_mask"] >> m & 1},
-            flags=pick.get("flags", 0)),
+            flags=pick.get("flags", 0), hot_kb=pick.get("hot_kb", 0)),
             sf, torch)
         results = []
         t0 = time.time()
-        for g in grid(cfg.dims, n, R, args.quick):
+        for g in (grid_sparse(cfg.dims, n, R) if args.sparse else grid(cfg.dims, n, R, args.quick)):
             if args.only_staged is not None:
                 want = {} if args.only_staged == "none" else {int(a): int(b) for a, b in
                                                               (x.split(":") for x in args.only_staged.split(","))}

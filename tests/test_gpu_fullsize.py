@@ -58,3 +58,44 @@ def test_fullsize_sampled_rows(cuda_device, name):
             if len(empty):
                 assert not y[torch.from_numpy(empty).cuda()].any()
             assert torch.isfinite(y).all()
+
+
+def _streamed_check(dims, inds, vals, facs, R, n, rows, segments=8, streams=4):
+    h_inds = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    h_vals = torch.from_numpy(vals).pin_memory()
+    d_facs = [torch.from_numpy(f).cuda() for f in facs]
+    y = torch.full((dims[n], R), float("nan"), device="cuda")
+    sf.mttkrp_streamed(dims, h_inds, h_vals, d_facs, n, y, segments, streams)
+    Yr, Sr = oracle.mttkrp_rows(dims, inds, vals, facs, R, n, rows)
+    got = y[torch.from_numpy(rows).cuda()].cpu().numpy()
+    rel, zv = oracle.max_rel_err(got, Yr, Sr)
+    assert torch.isfinite(y).all()
+    return rel
+
+
+def test_streamed_fullsize_nell2(cuda_device):
+    """A8 (ii) at BASELINE.json configs[1] size: the sorted-segment streamed path from pinned
+    host COO, sampled rows (incl. the heaviest) within the north-star tolerance."""
+    cfg = synth.CONFIGS["nell2"]
+    inds, vals = synth.config_tensor(cfg)
+    facs = synth.config_factors(cfg)
+    rng = np.random.default_rng(3)
+    for n in range(cfg.nmodes):
+        rows, _, _ = _sample_rows(rng, inds[n], cfg.dims[n], k=24)
+        rel = _streamed_check(cfg.dims, inds, vals, facs, cfg.rank, n, rows)
+        assert rel <= G.TOL, (n, rel)
+
+
+def test_streamed_heavy_row(cuda_device):
+    """SURVEY C-2: one row holding a large share of 2e7 nonzeros (amazon mode 3 has 1.2e8 in one
+    row) -- the sorted-segment kernel pre-reduces it in registers, so the fp32 atomic chain
+    stays short and the row meets 1e-4."""
+    dims, R, nnz = (50, 4000, 3000), 16, 20_000_000
+    inds, vals = synth.gen_coo(dims, nnz, 41, zipf=(2.5, 0.5, 0.5))
+    facs = synth.gen_factors(dims, R, 42)
+    cnt = np.bincount(inds[0], minlength=dims[0])
+    assert cnt.max() > 0.3 * nnz  # a genuinely heavy row
+    rows = np.array(sorted({int(np.argmax(cnt)), 0, 1, 2, int(np.argmin(cnt))}))
+    for segments, streams in ((8, 4), (3, 2)):
+        rel = _streamed_check(dims, inds, vals, facs, R, 0, rows, segments, streams)
+        assert rel <= G.TOL, (segments, rel)

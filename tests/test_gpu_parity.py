@@ -260,8 +260,8 @@ def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
     ti = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
     tv = torch.from_numpy(vals).pin_memory()
     tf = [G.dev_f(f) for f in facs]
-    for flag in ("1", "0"):
-        monkeypatch.setenv("SF_PRESORT", flag)
+    for flag in ("", "no_presort"):
+        monkeypatch.setenv("SF_DEBUG", flag)
         with sf.Tensor(dims, ti, tv, segments=segments, streams=streams) as t:
             for n in range(3):
                 others = [m for m in range(3) if m != n]

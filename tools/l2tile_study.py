@@ -73,7 +73,7 @@ def main():
         for n in range(cfg.nmodes):
             out = torch.empty((cfg.dims[n], R), dtype=torch.float32, device="cuda")
             # the selector without the L2-tile rule is the reference ("auto"); with it: "rule"
-            os.environ["SF_L2_TILES"] = "0"
+            os.environ["SF_DEBUG"] = "no_l2tiles"
             T.plan(n, R)
             auto = timed(n, out)
             ref = out.clone()
@@ -81,7 +81,7 @@ def main():
             print(json.dumps({"config": name, "dims": list(cfg.dims), "nnz": cfg.nnz, "rank": R, "mode": n,
                               "launch": "auto", "ms": auto, "picked": info["launch"]}), flush=True)
             T.plan_release(n, R)
-            os.environ["SF_L2_TILES"] = "1"
+            os.environ.pop("SF_DEBUG", None)
             T.plan(n, R)
             ms = timed(n, out)
             print(json.dumps({"config": name, "mode": n, "launch": "rule", "ms": ms, "speedup_vs_auto": auto / ms,

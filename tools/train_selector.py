@@ -166,6 +166,64 @@ def train(args):
         json.dump(report, open(args.report, "w"), indent=1)
 
 
+def compare(args):
+    """"DecisionTree ... compared with other models (SVM, AdaBoost, Bagging ...)".
+    5-fold CV on the same training corpus for each model family, as the deployed CLASSIFIER
+    (achieved / best time, accuracy) and as per-class time REGRESSORS (the paper's MAPE), with
+    training time and per-call inference time."""
+    from sklearn.ensemble import AdaBoostClassifier, AdaBoostRegressor, BaggingClassifier, BaggingRegressor
+    from sklearn.model_selection import KFold
+    from sklearn.pipeline import make_pipeline
+    from sklearn.preprocessing import StandardScaler
+    from sklearn.svm import SVC, SVR
+    from sklearn.tree import DecisionTreeClassifier, DecisionTreeRegressor
+    X, T = load_many(args.data)
+    y = np.argmin(T, axis=1)
+    best = T[np.arange(len(T)), y]
+    d = args.depth
+    fams = {
+        "DecisionTree": (lambda: DecisionTreeClassifier(max_depth=d, min_samples_leaf=2, random_state=0),
+                         lambda: DecisionTreeRegressor(max_depth=d, random_state=0)),
+        "SVM": (lambda: make_pipeline(StandardScaler(), SVC(C=10.0, gamma="scale")),
+                lambda: make_pipeline(StandardScaler(), SVR(C=10.0, gamma="scale"))),
+        "AdaBoost": (lambda: AdaBoostClassifier(DecisionTreeClassifier(max_depth=3), n_estimators=50, random_state=0),
+                     lambda: AdaBoostRegressor(DecisionTreeRegressor(max_depth=d), n_estimators=50, random_state=0)),
+        "Bagging": (lambda: BaggingClassifier(DecisionTreeClassifier(max_depth=d), n_estimators=30, random_state=0),
+                    lambda: BaggingRegressor(DecisionTreeRegressor(max_depth=d), n_estimators=30, random_state=0)),
+    }
+    kf = KFold(n_splits=5, shuffle=True, random_state=0)
+    out = {"samples": int(len(X)), "classes": int(T.shape[1]), "data": args.data, "models": {}}
+    for name, (mk_c, mk_r) in fams.items():
+        ratios, acc, mape = [], [], []
+        for tr, te in kf.split(X):
+            clf = mk_c().fit(X[tr], y[tr])
+            p = clf.predict(X[te])
+            ratios += list(best[te] / T[te, p])
+            acc += list(p == y[te])
+            for c in range(T.shape[1]):
+                ok = np.isfinite(T[:, c])
+                trc, tec = tr[ok[tr]], te[ok[te]]
+                if len(trc) < 4 or len(tec) == 0:
+                    continue
+                reg = mk_r().fit(X[trc], np.log(T[trc, c]))
+                pred = np.exp(reg.predict(X[tec]))
+                mape += list(np.abs(pred - T[tec, c]) / T[tec, c])
+        t0 = time.perf_counter()
+        clf = mk_c().fit(X, y)
+        train_s = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        for _ in range(200):
+            clf.predict(X[:1])
+        infer_ms = (time.perf_counter() - t0) / 200 * 1e3
+        out["models"][name] = {"cv_pick_over_best_mean": float(np.mean(ratios)),
+                               "cv_pick_over_best_min": float(np.min(ratios)),
+                               "cv_accuracy": float(np.mean(acc)), "cv_regressor_mape": float(np.mean(mape)),
+                               "train_s": train_s, "infer_ms_per_call": infer_ms}
+        print(name, json.dumps(out["models"][name]), flush=True)
+    if args.report:
+        json.dump(out, open(args.report, "w"), indent=1)
+
+
 def evaluate(args):
     import torch
 
@@ -203,7 +261,7 @@ def evaluate(args):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("cmd", choices=["collect", "train", "eval"])
+    ap.add_argument("cmd", choices=["collect", "train", "eval", "compare"])
     ap.add_argument("--count", type=int, default=40)
     ap.add_argument("--nnz-log10", default="6.0,7.5")
     ap.add_argument("--dims-log10", default="2.5,7.2")
@@ -220,7 +278,7 @@ def main():
     args_prefix, args_seed_base = args.prefix, args.seed_base
     args_nnz_lo, args_nnz_hi = (float(x) for x in args.nnz_log10.split(","))
     args_dims_log10 = tuple(float(x) for x in args.dims_log10.split(","))
-    {"collect": collect, "train": train, "eval": evaluate}[args.cmd](args)
+    {"collect": collect, "train": train, "eval": evaluate, "compare": compare}[args.cmd](args)
 
 
 if __name__ == "__main__":
