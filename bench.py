@@ -278,7 +278,11 @@ def main():
     # ---- synthetic input (every rank holds the full raw COO, §8(e) v1), generated in HBM by
     # the device twin of the seeded generator; pinned host copies feed the e2e leg ----
     t_gen = time.perf_counter()
-    d_inds, d_vals = synth.config_tensor_device(cfg, device=dev)
+    # at N>1 each rank generates / uploads only its slice of the input positions and the
+    # shards are assembled by the library's distributed preprocessing (sf_tensor_create_dist,
+    # SURVEY §8(e) v2): histogram allgather + one all-to-all per mode
+    lo, hi = (rank * cfg.nnz) // world, ((rank + 1) * cfg.nnz) // world
+    d_inds, d_vals = synth.config_tensor_device(cfg, device=dev, lo=lo, hi=hi)
     d_facs = synth.config_factors_device(cfg, device=dev)
     raw_bytes = sum(a.numel() * 4 for a in d_inds) + d_vals.numel() * 4
     import psutil
@@ -297,7 +301,8 @@ def main():
     stream = torch.cuda.Stream(device=dev)
 
     # ---- resident tensor ----
-    T = sf.Tensor(cfg.dims, d_inds, d_vals)
+    T = sf.Tensor(cfg.dims, d_inds, d_vals) if world == 1 else \
+        sf.Tensor.create_dist(cfg.dims, cfg.nnz, lo, d_inds, d_vals)
     del d_inds, d_vals
     torch.cuda.empty_cache()
     if world > 1:  # shard + the boundary exchange inside sf_mttkrp (NCCL; gloo transport on one GPU)
@@ -447,7 +452,8 @@ def main():
         d2h_s = torch.cuda.Stream(device=dev)
 
         def e2e_step():
-            with sf.Tensor(cfg.dims, h_inds, h_vals) as T2:
+            with (sf.Tensor(cfg.dims, h_inds, h_vals) if world == 1 else
+                  sf.Tensor.create_dist(cfg.dims, cfg.nnz, lo, h_inds, h_vals)) as T2:
                 if world > 1:
                     sfdist.attach(T2, world, rank)
                 ev_f = {}

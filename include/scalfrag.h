@@ -139,6 +139,16 @@ sf_status sf_tensor_create_ex(int nmodes, const uint64_t* dims, uint64_t nnz,
                               const uint32_t* const* inds, const float* vals, int segments,
                               int streams, sf_tensor_t* out);
 sf_status sf_tensor_destroy(sf_tensor_t t);
+/* Distributed ingest (SURVEY §8(e) "v2", row F4): this rank passes only input positions
+ * [pos_begin, pos_begin + nnz_local) of an nnz_total-nonzero tensor (the ranks' slices must
+ * tile [0, nnz_total) in rank order; nnz_total < 2^32).  After sf_comm_attach*, the first
+ * sf_plan of a mode assembles this rank's shard of the matricized order -- the same nonzeros
+ * as sf_set_shard on the whole tensor -- by a global i_n histogram (allgather + rank-order
+ * sum) and one all-to-all, then sorts only the shard.  sf_plan_export reports global input
+ * positions.  Everything else behaves as a sharded handle. */
+sf_status sf_tensor_create_dist(int nmodes, const uint64_t* dims, uint64_t nnz_total, uint64_t pos_begin,
+                                uint64_t nnz_local, const uint32_t* const* inds, const float* vals,
+                                sf_tensor_t* out);
 
 /* Multi-GPU (§8(e)): restrict this handle to shard `rank` of `nranks`: for every mode
  * it owns matricized positions [floor(rank*nnz/nranks), floor((rank+1)*nnz/nranks)).
@@ -264,6 +274,9 @@ const char* sf_status_string(sf_status s);
 const char* sf_last_error(void);
 /* Number of kernels this library has launched in this process (monotone). */
 uint64_t sf_kernel_launches(void);
+/* Device bytes held by the library's live buffers (all handles, plans, scratch; the block
+ * cache's idle blocks excluded) and their high-water mark since the last reset_peak != 0. */
+sf_status sf_device_bytes(uint64_t* in_use, uint64_t* peak, int reset_peak);
 /* Library version string. */
 const char* sf_version(void);
 

@@ -104,7 +104,8 @@ EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
             "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
             "sf_trim_cache", "sf_shard_rows", "sf_comm_unique_id", "sf_comm_attach",
-            "sf_comm_attach_transport", "sf_comm_detach", "sf_allgather_rows", "sf_exchange_map"]
+            "sf_comm_attach_transport", "sf_comm_detach", "sf_allgather_rows", "sf_exchange_map",
+            "sf_tensor_create_dist", "sf_device_bytes"]
 
 # int fn(void* ctx, const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs,
 #        int nranks, void* stream)
@@ -150,6 +151,8 @@ def lib(build_if_missing: bool = True):
             L.sf_comm_detach.argtypes = [P]
             L.sf_allgather_rows.argtypes = [P, I, I, P, P, P]
             L.sf_exchange_map.argtypes = [I, P, P, P]
+            L.sf_device_bytes.argtypes = [ctypes.POINTER(U64), ctypes.POINTER(U64), I]
+            L.sf_tensor_create_dist.argtypes = [I, P, U64, U64, U64, P, P, ctypes.POINTER(P)]
             for fn in EXPORTED:
                 if fn not in ("sf_status_string", "sf_last_error", "sf_kernel_launches", "sf_version"):
                     getattr(L, fn).restype = ctypes.c_int
@@ -242,6 +245,13 @@ def kernel_launches() -> int:
     return int(lib().sf_kernel_launches())
 
 
+def device_bytes(reset_peak=False):
+    """(bytes held by live library buffers, high-water mark) -- sf_device_bytes."""
+    a, b = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    _check(lib().sf_device_bytes(ctypes.byref(a), ctypes.byref(b), int(bool(reset_peak))))
+    return a.value, b.value
+
+
 def version() -> str:
     return lib().sf_version().decode()
 
@@ -259,6 +269,22 @@ class Tensor:
         _check(lib().sf_tensor_create_ex(self.nmodes, d, self.nnz, ip, _ptr(vals), int(segments),
                                          int(streams), ctypes.byref(h)))
         self._h = h
+
+    @classmethod
+    def create_dist(cls, dims, nnz_total, pos_begin, inds, vals):
+        """Distributed ingest (sf_tensor_create_dist): this rank's slice [pos_begin, pos_begin +
+        len(vals)) of an nnz_total-nonzero tensor; attach a comm before planning."""
+        self = cls.__new__(cls)
+        self.dims = tuple(int(d) for d in dims)
+        self.nmodes = len(self.dims)
+        self.nnz = int(len(vals))
+        d = (ctypes.c_uint64 * self.nmodes)(*self.dims)
+        ip = (ctypes.c_void_p * self.nmodes)(*[_ptr(a) for a in inds])
+        h = ctypes.c_void_p()
+        _check(lib().sf_tensor_create_dist(self.nmodes, d, int(nnz_total), int(pos_begin), self.nnz, ip, _ptr(vals),
+                                           ctypes.byref(h)))
+        self._h = h
+        return self
 
     def close(self):
         if getattr(self, "_h", None):

@@ -124,6 +124,9 @@ struct BlockCache {
 };
 static BlockCache g_cache;
 
+// Bytes held by live library buffers (all devices) and their high-water mark (sf_device_bytes).
+static std::atomic<uint64_t> g_in_use{0}, g_peak{0};
+
 void DevBuf::alloc(size_t b) {
   release();
   if (b == 0) b = 16;
@@ -131,10 +134,17 @@ void DevBuf::alloc(size_t b) {
   size_t got = 0;
   p = g_cache.get(b, &got);
   bytes = got;
+  const uint64_t now = g_in_use.fetch_add(got) + got;
+  uint64_t pk = g_peak.load();
+  while (now > pk && !g_peak.compare_exchange_weak(pk, now)) {
+  }
 }
 
 void DevBuf::release() {
-  if (p) g_cache.put(p, bytes);
+  if (p) {
+    g_cache.put(p, bytes);
+    g_in_use.fetch_sub(bytes);
+  }
   p = nullptr;
   bytes = 0;
 }
@@ -149,6 +159,10 @@ size_t Plan::device_bytes() const {
 Tensor::~Tensor() {
   for (auto& kv : plans) delete kv.second;
   plans.clear();
+  for (int m = 0; m < SF_MAX_MODES; ++m) {
+    delete sub[m];
+    sub[m] = nullptr;
+  }
   delete comm;
   comm = nullptr;
   if (stream) cudaStreamDestroy(stream);
@@ -278,28 +292,42 @@ static Plan* get_plan(Tensor& t, int mode, int rank) {
   return it == t.plans.end() ? nullptr : it->second;
 }
 
+// The tensor a plan of `mode` is built from: the handle itself, or -- for a distributed
+// handle (sf_tensor_create_dist) with several ranks -- this rank's shard of the mode, gathered
+// from every rank (sf_dist.cu), planned as a one-rank tensor.
+static Tensor& plan_source(Tensor& t, int mode) {
+  if (!t.dist || t.nranks == 1) return t;
+  dist_build_sub(t, mode);
+  return *t.sub[mode];
+}
+
 static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override_launch) {
   trace_mark("plan: enter");
   SF_CUDA(cudaSetDevice(t.device));
+  Tensor& src = plan_source(t, mode);
   sf_features_t f;
   DevBuf keys, pos;  // the matricized order, sorted once for features + the plan
-  compute_features(t, mode, &f, &keys, &pos);
+  compute_features(src, mode, &f, &keys, &pos);
   trace_mark("plan: features");
-  const uint64_t lo = (uint64_t)(((unsigned __int128)t.rank * t.nnz) / t.nranks);
-  const uint64_t hi = (uint64_t)(((unsigned __int128)(t.rank + 1) * t.nnz) / t.nranks);
+  const uint64_t lo = (uint64_t)(((unsigned __int128)src.rank * src.nnz) / src.nranks);
+  const uint64_t hi = (uint64_t)(((unsigned __int128)(src.rank + 1) * src.nnz) / src.nranks);
   sf_launch_t l;
   if (override_launch && override_launch->kernel != SF_KERNEL_AUTO) {
     l = *override_launch;
-    normalize_launch(t, mode, rank, l);
+    normalize_launch(src, mode, rank, l);
   } else {
-    l = select_launch(t, f, mode, rank, hi - lo);
+    l = select_launch(src, f, mode, rank, hi - lo);
   }
-  if (l.kernel == SF_KERNEL_FRAG && frag_smem_bytes(t, mode, rank, l) > t.smem_optin)
+  if (l.kernel == SF_KERNEL_FRAG && frag_smem_bytes(src, mode, rank, l) > src.smem_optin)
     throw StatusError{SF_ERR_INVALID_ARG, "launch needs more shared memory than the device has"};
   trace_mark("plan: select");
   Plan* p = new Plan();
   try {
-    build_plan(t, *p, mode, rank, l, &keys, &pos);
+    build_plan(src, *p, mode, rank, l, &keys, &pos);
+    if (&src != &t) {  // a distributed shard writes its local row block like any shard
+      p->out_row0 = p->row_begin;
+      p->out_rows = p->row_end - p->row_begin;
+    }
     trace_mark("plan: build");
   } catch (...) {
     delete p;
@@ -408,6 +436,11 @@ sf_status sf_set_shard(sf_tensor_t h, int nranks, int rank) {
     }
     for (auto& kv : t->plans) delete kv.second;
     t->plans.clear();
+    for (int m = 0; m < SF_MAX_MODES; ++m) {  // distributed shards depend on (nranks, rank)
+      delete t->sub[m];
+      t->sub[m] = nullptr;
+      t->sub_gpos[m].release();
+    }
     t->nranks = nranks;
     t->rank = rank;
     return SF_OK;
@@ -464,7 +497,7 @@ sf_status sf_features(sf_tensor_t h, int mode, sf_features_t* out) {
     Tensor* t = as_tensor(h);
     check_mode_rank(*t, mode, 1);
     SF_CUDA(cudaSetDevice(t->device));
-    compute_features(*t, mode, out, nullptr, nullptr);
+    compute_features(plan_source(*t, mode), mode, out, nullptr, nullptr);
     return SF_OK;
   });
 }
@@ -503,7 +536,13 @@ sf_status sf_plan_export(sf_tensor_t h, int mode, int rank, uint64_t* perm_host,
     if (perm_host && p->nnz_local) {
       std::vector<uint32_t> tmp(p->nnz_local);
       SF_CUDA(cudaMemcpy(tmp.data(), p->perm.p, p->nnz_local * 4, cudaMemcpyDeviceToHost));
-      for (uint64_t k = 0; k < p->nnz_local; ++k) perm_host[k] = tmp[k];
+      if (t->sub[mode] && t->dist && t->nranks > 1) {  // shard positions -> global input positions
+        std::vector<uint32_t> g(t->sub[mode]->nnz);
+        SF_CUDA(cudaMemcpy(g.data(), t->sub_gpos[mode].p, g.size() * 4, cudaMemcpyDeviceToHost));
+        for (uint64_t k = 0; k < p->nnz_local; ++k) perm_host[k] = g[tmp[k]];
+      } else {
+        for (uint64_t k = 0; k < p->nnz_local; ++k) perm_host[k] = tmp[k];
+      }
     }
     if (chunks_host && p->num_chunks) {
       std::vector<uint32_t> b(p->num_chunks + 1);
@@ -697,10 +736,11 @@ sf_status sf_selector_features(sf_tensor_t h, int mode, int rank, double* x, int
     check_mode_rank(*t, mode, rank);
     SF_CUDA(cudaSetDevice(t->device));
     sf_features_t f;
-    compute_features(*t, mode, &f, nullptr, nullptr);
-    const uint64_t lo = (uint64_t)(((unsigned __int128)t->rank * t->nnz) / t->nranks);
-    const uint64_t hi = (uint64_t)(((unsigned __int128)(t->rank + 1) * t->nnz) / t->nranks);
-    *n = selector_features(*t, f, mode, rank, hi - lo, x);
+    Tensor& src = plan_source(*t, mode);
+    compute_features(src, mode, &f, nullptr, nullptr);
+    const uint64_t lo = (uint64_t)(((unsigned __int128)src.rank * src.nnz) / src.nranks);
+    const uint64_t hi = (uint64_t)(((unsigned __int128)(src.rank + 1) * src.nnz) / src.nranks);
+    *n = selector_features(src, f, mode, rank, hi - lo, x);
     return SF_OK;
   });
 }
@@ -744,6 +784,13 @@ const char* sf_status_string(sf_status s) {
 const char* sf_last_error(void) { return g_err.c_str(); }
 
 uint64_t sf_kernel_launches(void) { return g_launches.load(); }
+
+sf_status sf_device_bytes(uint64_t* in_use, uint64_t* peak, int reset_peak) {
+  if (in_use) *in_use = g_in_use.load();
+  if (peak) *peak = g_peak.load();
+  if (reset_peak) g_peak.store(g_in_use.load());
+  return SF_OK;
+}
 
 const char* sf_version(void) { return "scalfrag-b200 0.1 (sm_100a)"; }
 

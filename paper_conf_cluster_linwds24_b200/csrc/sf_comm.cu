@@ -13,7 +13,8 @@
 // rank; this moves R*4.
 //
 // Transport: NCCL (dlopen'ed libnccl.so.2: ncclBroadcast per root inside a group = an
-// allgatherv, on the caller's stream) or the caller's allgatherv callback.
+// allgatherv, grouped ncclSend/ncclRecv = an alltoallv, on the caller's stream) or the
+// caller's allgatherv callback.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>
@@ -39,6 +40,8 @@ struct NcclApi {
   ncclResult_t (*GroupStart)() = nullptr;
   ncclResult_t (*GroupEnd)() = nullptr;
   ncclResult_t (*Broadcast)(const void*, void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
 };
 
@@ -58,8 +61,11 @@ static NcclApi& nccl() {
     a.GroupStart = reinterpret_cast<decltype(a.GroupStart)>(sym("ncclGroupStart"));
     a.GroupEnd = reinterpret_cast<decltype(a.GroupEnd)>(sym("ncclGroupEnd"));
     a.Broadcast = reinterpret_cast<decltype(a.Broadcast)>(sym("ncclBroadcast"));
+    a.Send = reinterpret_cast<decltype(a.Send)>(sym("ncclSend"));
+    a.Recv = reinterpret_cast<decltype(a.Recv)>(sym("ncclRecv"));
     a.GetErrorString = reinterpret_cast<decltype(a.GetErrorString)>(sym("ncclGetErrorString"));
-    a.ok = a.GetUniqueId && a.CommInitRank && a.CommDestroy && a.GroupStart && a.GroupEnd && a.Broadcast;
+    a.ok = a.GetUniqueId && a.CommInitRank && a.CommDestroy && a.GroupStart && a.GroupEnd && a.Broadcast && a.Send &&
+           a.Recv;
     if (!a.ok) a.err = "libnccl.so.2 lacks a required symbol";
     return a;
   }();
@@ -94,6 +100,58 @@ void Comm::allgatherv(const void* send, void* recv, const uint64_t* bytes, const
     nccl_check(api.Broadcast(src, dst, bytes[k], ncclChar, k, static_cast<ncclComm_t>(nccl), s), "ncclBroadcast");
   }
   nccl_check(api.GroupEnd(), "ncclGroupEnd");
+}
+
+// alltoallv: block q of `send` (sbytes[q] bytes at sdispl[q]) goes to rank q; the block from
+// rank k lands at recv + rdispl[k] (rbytes[k] bytes).  NCCL: grouped ncclSend / ncclRecv.
+// Caller transport: emulated with allgatherv (every rank receives every send buffer and keeps
+// its blocks -- a test-only cost).
+void Comm::alltoallv(const void* send, const uint64_t* sbytes, const uint64_t* sdispl, void* recv,
+                     const uint64_t* rbytes, const uint64_t* rdispl, cudaStream_t s) {
+  if (!fn) {
+    NcclApi& api = sf::nccl();
+    if (!nccl || !api.ok) throw StatusError{SF_ERR_NCCL, "no NCCL communicator"};
+    nccl_check(api.GroupStart(), "ncclGroupStart");
+    for (int q = 0; q < nranks; ++q) {
+      if (sbytes[q])
+        nccl_check(api.Send(static_cast<const char*>(send) + sdispl[q], sbytes[q], ncclChar, q,
+                            static_cast<ncclComm_t>(nccl), s), "ncclSend");
+      if (rbytes[q])
+        nccl_check(api.Recv(static_cast<char*>(recv) + rdispl[q], rbytes[q], ncclChar, q,
+                            static_cast<ncclComm_t>(nccl), s), "ncclRecv");
+    }
+    nccl_check(api.GroupEnd(), "ncclGroupEnd");
+    return;
+  }
+  // every rank's (sbytes, sdispl) table, then every rank's whole send buffer
+  const int P = nranks;
+  DevBuf tab((size_t)P * P * 16 + 16);
+  std::vector<uint64_t> mine(2 * P), bytes(P, (uint64_t)P * 16), displs(P);
+  for (int q = 0; q < P; ++q) { mine[2 * q] = sbytes[q]; mine[2 * q + 1] = sdispl[q]; displs[q] = (uint64_t)q * P * 16; }
+  char* tsend = tab.as<char>() + (size_t)rank * P * 16;
+  SF_CUDA(cudaMemcpyAsync(tsend, mine.data(), (size_t)P * 16, cudaMemcpyHostToDevice, s));
+  allgatherv(tsend, tab.p, bytes.data(), displs.data(), s);
+  std::vector<uint64_t> all((size_t)P * P * 2);
+  SF_CUDA(cudaMemcpyAsync(all.data(), tab.p, (size_t)P * P * 16, cudaMemcpyDeviceToHost, s));
+  SF_CUDA(cudaStreamSynchronize(s));
+  std::vector<uint64_t> tot(P), off(P);
+  uint64_t sum = 0;
+  for (int k = 0; k < P; ++k) {
+    uint64_t end = 0;
+    for (int q = 0; q < P; ++q) end = std::max(end, all[(size_t)k * 2 * P + 2 * q] + all[(size_t)k * 2 * P + 2 * q + 1]);
+    tot[k] = end;
+    off[k] = sum;
+    sum += end;
+  }
+  DevBuf big(sum + 16);
+  allgatherv(send, big.p, tot.data(), off.data(), s);
+  for (int k = 0; k < P; ++k) {
+    const uint64_t b = all[(size_t)k * 2 * P + 2 * rank], d = all[(size_t)k * 2 * P + 2 * rank + 1];
+    if (b != rbytes[k]) throw StatusError{SF_ERR_NCCL, "alltoallv: receive size mismatch"};
+    if (b) SF_CUDA(cudaMemcpyAsync(static_cast<char*>(recv) + rdispl[k], big.as<char>() + off[k] + d, b,
+                                   cudaMemcpyDeviceToDevice, s));
+  }
+  SF_CUDA(cudaStreamSynchronize(s));
 }
 
 // ---------------------------------------------------------------------------

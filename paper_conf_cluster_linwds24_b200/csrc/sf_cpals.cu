@@ -501,11 +501,18 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
       parts(sharded ? (size_t)P * R * R * sizeof(double) + 64 : 16);
   double* dG = G.as<double>();
   for (int m = 0; m < N; ++m) gram(factors[m], t.dims[m], R, dG + (size_t)m * R * R, s);
-  // ||X||^2 (whole tensor: every rank holds the full raw COO)
+  // ||X||^2 (whole tensor: every rank holds the full raw COO; distributed handles sum slices)
   SF_CUDA(cudaMemsetAsync(scal.p, 0, 4 * sizeof(double), s));
   dot_kernel<<<grid_of(t.nnz, 256), 256, 0, s>>>(t.val.as<float>(), nullptr, t.nnz, scal.as<double>());
   count_launch();
   double normX2 = 0;
+  if (sharded && t.dist) {  // a distributed handle holds only its slice of the values
+    std::vector<uint64_t> bytes(P, 8), displs(P);
+    for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * 8;
+    t.comm->allgatherv(scal.p, parts.p, bytes.data(), displs.data(), s);
+    sum_parts_kernel<<<1, 32, 0, s>>>(parts.as<double>(), P, 1, scal.as<double>());
+    count_launch();
+  }
   SF_CUDA(cudaMemcpyAsync(&normX2, scal.p, sizeof(double), cudaMemcpyDeviceToHost, s));
   SF_CUDA(cudaStreamSynchronize(s));
   const float* const* cf = const_cast<const float* const*>(factors);

@@ -120,6 +120,8 @@ struct Comm {
   sf_allgatherv_fn fn = nullptr;
   void* ctx = nullptr;
   void allgatherv(const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs, cudaStream_t s);
+  void alltoallv(const void* send, const uint64_t* sbytes, const uint64_t* sdispl, void* recv, const uint64_t* rbytes,
+                 const uint64_t* rdispl, cudaStream_t s);
   ~Comm();
 };
 
@@ -149,6 +151,14 @@ struct Tensor {
   int pre_pb = 0;              // position bits
   cudaStream_t stream = nullptr;               // internal stream for planning
   Comm* comm = nullptr;                        // sharded handles: collective transport
+  // Distributed ingest (sf_tensor_create_dist): this handle holds only input
+  // positions [pos_begin, pos_begin + nnz) of an nnz_total-nonzero tensor; per mode, the
+  // nonzeros of this rank's shard of the matricized order are fetched from every rank
+  // (histogram allgather + all-to-all) into sub[mode], whose plan the handle uses.
+  bool dist = false;
+  uint64_t pos_begin = 0, nnz_total = 0;
+  Tensor* sub[SF_MAX_MODES] = {};
+  DevBuf sub_gpos[SF_MAX_MODES];               // global input position of every sub[mode] nonzero
   ~Tensor();
 };
 
@@ -265,6 +275,9 @@ void exchange_rows(Tensor& t, Plan& p, float* out, cudaStream_t s);
 void allgather_blocks(Tensor& t, const std::vector<uint64_t>& blk, const float* local, float* full, int R,
                       cudaStream_t s);
 void ensure_ranges(Tensor& t, Plan& p, cudaStream_t s);
+// sf_tensor_create_dist handles: build sub[mode] (this rank's shard of mode `mode`, gathered
+// from every rank; sf_dist.cu).
+void dist_build_sub(Tensor& t, int mode);
 void validate_indices(int nmodes, const uint64_t* dims, uint64_t nnz,
                       uint32_t* const* inds, int* d_flag, cudaStream_t s);
 

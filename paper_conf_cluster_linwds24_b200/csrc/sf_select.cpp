@@ -349,7 +349,17 @@ static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
     if (F >= 16.0 * 1024 * 1024) gathered += F;
   }
   if (gathered < kHotMinGatheredBytes || debug_opt("no_hot")) return;  // SF_DEBUG A/B
+  // the hot-row class: owner stores, 1024 threads (one CTA per SM), chunks of 64 nonzeros per
+  // warp and 32 MB of hot rows -- over the exhaustive sparse sweeps of nell-1 and deli-4d
+  // (sweep.py --sparse, 199-283 launches per mode, profiles/r02/sweeps/) the best fixed
+  // class: >= 0.945 of each mode's sweep best, 0.980 on average
   l.hot_kb = (l.flags & SF_LAUNCH_L2_TILES) ? kHotKBTiled : kHotKB;
+  l.block_threads = 1024;
+  l.chunk_nnz = 64;
+  l.ctas_per_sm = 0;
+  l.flags &= ~SF_LAUNCH_NO_OWNER_STORES;
+  normalize_launch(t, mode, rank, l);
+  if (frag_smem_bytes(t, mode, rank, l) > t.smem_optin) l.hot_kb = 0;
 }
 
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local) {

@@ -64,6 +64,32 @@ def main():
             if not ok_n:
                 msgs.append(f"mode {n} rank {rank} ranges {ranges}")
             ok &= ok_n
+    # distributed ingest (sf_tensor_create_dist): rank p holds only input
+    # positions [p*nnz/P, (p+1)*nnz/P); its shard plans must equal the v1 shard plans bit for bit
+    # (kernel order as global input positions, chunks) and give the same Y blocks
+    nnz = int(vals.numel())
+    lo, hi = rank * nnz // world, (rank + 1) * nnz // world
+    for n in range(3):
+        L = sf.Launch.make(kernel=sf.KERNEL_FRAG, chunk_nnz=128)
+        with sf.Tensor(dims, inds, vals) as T1, \
+                sf.Tensor.create_dist(dims, nnz, lo, [a[lo:hi] for a in inds], vals[lo:hi]) as T2:
+            sfdist.attach(T1, world, rank)
+            sfdist.attach(T2, world, rank)
+            T1.set_launch(n, R, L)
+            T2.set_launch(n, R, L)
+            p1, c1 = T1.plan_export(n, R)
+            p2, c2 = T2.plan_export(n, R)
+            i1, i2 = T1.plan_info(n, R), T2.plan_info(n, R)
+            y1 = torch.empty((i1["out_rows"], R), device=dev)
+            y2 = torch.empty((i2["out_rows"], R), device=dev)
+            T1.mttkrp(n, facs, y1)
+            T2.mttkrp(n, facs, y2)
+            torch.cuda.synchronize()
+            same = (np.array_equal(p1, p2) and np.array_equal(c1, c2) and i1["row_begin"] == i2["row_begin"]
+                    and i1["row_end"] == i2["row_end"] and bool(torch.equal(y1, y2)))
+            if not same:
+                ok = False
+                msgs.append(f"dist v2 mode {n} rank {rank}: plan/Y differ from v1")
     # CP-ALS on the shards == CP-ALS on one rank (same initial factors) up to fp32 summation
     # order (the shards sum M and the Grams in a different order): the bar of
     # tests/test_gpu_cpals.py against the fp64 oracle (fits 2e-4 over 3 sweeps, factors 2e-3

@@ -60,6 +60,11 @@ def main():
                 dbuf.copy_(h, non_blocking=True)
 
         t_h2d = wall(h2d)
+        h_y = torch.empty((cfg.dims[n], R), dtype=torch.float32).pin_memory()
+
+        def d2h():
+            h_y.copy_(y, non_blocking=True)
+        t_d2h = wall(d2h)
         grid = {}
         for S in (1, 2, 4, 8, 16, 32):
             for K in (1, 2, 4, 8):
@@ -77,12 +82,23 @@ def main():
                 torch.cuda.synchronize()
         t_res = wall(resident, reps=3)
         best = min(grid, key=grid.get)
+        # device footprint of the streamed path (O(streams x segment), not O(tensor): tensors larger
+        # than HBM stream through it) at 32 segments / 4 streams vs the tensor's bytes
+        sf.device_bytes(reset_peak=True)
+        sf.mttkrp_streamed(cfg.dims, h_inds, h_vals, facs, n, y, 32, 4)
+        torch.cuda.synchronize()
+        peak_streamed = sf.device_bytes()[1]
         out[name] = {"nnz": cfg.nnz, "bytes_h2d": int(sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4),
                      "t_h2d_ms": t_h2d, "h2d_GBps": (sum(a.numel() * 4 for a in h_inds) + h_vals.numel() * 4) / t_h2d / 1e6,
                      "t_compute_ms": t_comp, "t_streamed_ms": grid, "overlap_ratio": ov,
                      "best": best, "speedup_best_vs_1x1": t11 / grid[best],
-                     "t_resident_path_ms": t_res, "mode": n}
+                     "t_resident_path_ms": t_res, "mode": n, "t_d2h_ms": t_d2h,
+                     "breakdown_ms": {"h2d": t_h2d, "kernel": t_comp, "d2h": t_d2h,
+                                      "serial_sum": t_h2d + t_comp + t_d2h,
+                                      "streamed_best_plus_d2h": grid[best] + t_d2h},
+                     "streamed_peak_device_bytes_32seg": int(peak_streamed)}
         print(json.dumps({name: out[name]}), flush=True)
+    os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     path = os.path.join(ROOT, "gpurun_out", "stream_study.json")
     json.dump(out, open(path, "w"), indent=1)
 
