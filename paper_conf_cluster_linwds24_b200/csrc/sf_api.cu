@@ -149,6 +149,95 @@ void DevBuf::release() {
   bytes = 0;
 }
 
+// ---- small transfers through mapped pinned memory (no copy engine) ----
+__global__ void copy_bytes_kernel(unsigned char* __restrict__ dst, const unsigned char* __restrict__ src, size_t n) {
+  for (size_t i = threadIdx.x; i < n; i += blockDim.x) dst[i] = src[i];
+}
+
+static unsigned char* staging(size_t need) {
+  static thread_local unsigned char* buf = nullptr;
+  static thread_local size_t cap = 0;
+  if (need > cap) {
+    if (buf) cudaFreeHost(buf);
+    buf = nullptr;
+    cap = std::max<size_t>(need, 1 << 16);
+    SF_CUDA(cudaHostAlloc(reinterpret_cast<void**>(&buf), cap, cudaHostAllocMapped | cudaHostAllocPortable));
+  }
+  return buf;
+}
+
+void d2h_small(cudaStream_t s, int n, void* const* dst, const void* const* src, const size_t* bytes) {
+  size_t total = 0;
+  for (int i = 0; i < n; ++i) total += (bytes[i] + 15) & ~(size_t)15;
+  unsigned char* st = staging(total);
+  size_t off = 0;
+  for (int i = 0; i < n; ++i) {
+    if (!bytes[i]) continue;
+    copy_bytes_kernel<<<1, 256, 0, s>>>(st + off, static_cast<const unsigned char*>(src[i]), bytes[i]);
+    count_launch();
+    off += (bytes[i] + 15) & ~(size_t)15;
+  }
+  SF_CUDA(cudaGetLastError());
+  SF_CUDA(cudaStreamSynchronize(s));
+  off = 0;
+  for (int i = 0; i < n; ++i) {
+    if (!bytes[i]) continue;
+    memcpy(dst[i], st + off, bytes[i]);
+    off += (bytes[i] + 15) & ~(size_t)15;
+  }
+}
+
+void h2d_small(cudaStream_t s, void* dst, const void* src, size_t bytes) {
+  if (!bytes) return;
+  unsigned char* st = staging(bytes);
+  memcpy(st, src, bytes);
+  copy_bytes_kernel<<<1, 256, 0, s>>>(static_cast<unsigned char*>(dst), st, bytes);
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+  SF_CUDA(cudaStreamSynchronize(s));  // the staging buffer is reused by the next call
+}
+
+__global__ void d2d_vec_kernel(uint4* __restrict__ dst, const uint4* __restrict__ src, size_t n16) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += stride) dst[i] = src[i];
+}
+
+__global__ void d2d_bytes_kernel(unsigned char* __restrict__ dst, const unsigned char* __restrict__ src, size_t n,
+                                 int word) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x;
+  if (word) {  // 4-byte aligned
+    uint32_t* d = reinterpret_cast<uint32_t*>(dst);
+    const uint32_t* q = reinterpret_cast<const uint32_t*>(src);
+    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n / 4; i += stride) d[i] = q[i];
+    for (size_t i = (n / 4) * 4 + (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) dst[i] = src[i];
+  } else {
+    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) dst[i] = src[i];
+  }
+}
+
+void d2d_copy(void* dst, const void* src, size_t bytes, cudaStream_t s) {
+  if (!bytes) return;
+  const uintptr_t a = reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src);
+  unsigned char* d = static_cast<unsigned char*>(dst);
+  const unsigned char* q = static_cast<const unsigned char*>(src);
+  size_t done = 0;
+  if ((a & 15) == 0 && bytes >= 16) {
+    const size_t n16 = bytes / 16;
+    d2d_vec_kernel<<<(int)std::max<size_t>(1, std::min<size_t>((n16 + 255) / 256, 148 * 8)), 256, 0, s>>>(
+        reinterpret_cast<uint4*>(d), reinterpret_cast<const uint4*>(q), n16);
+    count_launch();
+    done = n16 * 16;
+  }
+  if (done < bytes) {
+    const size_t rest = bytes - done;
+    const int word = ((a & 3) == 0) ? 1 : 0;
+    d2d_bytes_kernel<<<(int)std::max<size_t>(1, std::min<size_t>((rest / 4 + 255) / 256, 148 * 8)), 256, 0, s>>>(
+        d + done, q + done, rest, word);
+    count_launch();
+  }
+  SF_CUDA(cudaGetLastError());
+}
+
 size_t Plan::device_bytes() const {
   size_t b = val.bytes + rec.bytes + perm.bytes + chunk_begin.bytes + chunk_tile.bytes + tile_chunk.bytes +
              hot_cache.bytes;

@@ -187,11 +187,10 @@ void ensure_ranges(Tensor& t, Plan& p, cudaStream_t s) {
   std::vector<uint64_t> bytes(P, 16), displs(P);
   for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * 16;
   char* send = buf.as<char>() + (size_t)t.rank * 16;
-  SF_CUDA(cudaMemcpyAsync(send, mine, 16, cudaMemcpyHostToDevice, s));
+  h2d_small(s, send, mine, 16);
   t.comm->allgatherv(send, buf.p, bytes.data(), displs.data(), s);
   std::vector<uint64_t> r(2 * P);
-  SF_CUDA(cudaMemcpyAsync(r.data(), buf.p, (size_t)P * 16, cudaMemcpyDeviceToHost, s));
-  SF_CUDA(cudaStreamSynchronize(s));
+  d2h_small(s, r.data(), buf.p, (size_t)P * 16);
   std::vector<int> owner;
   std::vector<char> sends;
   exchange_map(r, P, owner, sends);
@@ -221,14 +220,13 @@ void exchange_rows(Tensor& t, Plan& p, float* out, cudaStream_t s) {
     p.xbuf.alloc(need);
     std::vector<int> srcs(P, 0);
     for (size_t i = 0; i < p.add_srcs.size(); ++i) srcs[i] = p.add_srcs[i];
-    SF_CUDA(cudaMemcpyAsync(p.xbuf.as<char>() + (size_t)(P + 1) * R * 4, srcs.data(), (size_t)P * 4,
-                            cudaMemcpyHostToDevice, s));
+    h2d_small(s, p.xbuf.as<char>() + (size_t)(P + 1) * R * 4, srcs.data(), (size_t)P * 4);
   }
   float* send = p.xbuf.as<float>();
   float* recv = send + R;
   const int* srcs = reinterpret_cast<const int*>(p.xbuf.as<char>() + (size_t)(P + 1) * R * 4);
   const bool nonempty = p.row_end > p.row_begin;
-  if (p.send_first) SF_CUDA(cudaMemcpyAsync(send, out, (size_t)R * 4, cudaMemcpyDeviceToDevice, s));
+  if (p.send_first) d2d_copy(send, out, (size_t)R * 4, s);
   std::vector<uint64_t> bytes(P, (uint64_t)R * 4), displs(P);
   for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * R * 4;
   t.comm->allgatherv(send, recv, bytes.data(), displs.data(), s);

@@ -513,8 +513,7 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
     sum_parts_kernel<<<1, 32, 0, s>>>(parts.as<double>(), P, 1, scal.as<double>());
     count_launch();
   }
-  SF_CUDA(cudaMemcpyAsync(&normX2, scal.p, sizeof(double), cudaMemcpyDeviceToHost, s));
-  SF_CUDA(cudaStreamSynchronize(s));
+  d2h_small(s, &normX2, scal.p, sizeof(double));
   const float* const* cf = const_cast<const float* const*>(factors);
   // [V | I] in fp64: 64 KB at R = 64, above the 48 KB default dynamic shared-memory limit
   const size_t pinv_smem = (size_t)R * 2 * R * sizeof(double);
@@ -580,8 +579,7 @@ void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, doubl
     model_norm_kernel<<<1, 256, 0, s>>>(dG, N, R, scal.as<double>() + 2);
     count_launch();
     double h[3];
-    SF_CUDA(cudaMemcpyAsync(h, scal.p, 3 * sizeof(double), cudaMemcpyDeviceToHost, s));
-    SF_CUDA(cudaStreamSynchronize(s));
+    d2h_small(s, h, scal.p, 3 * sizeof(double));
     const double res2 = std::max(normX2 + h[2] - 2.0 * h[1], 0.0);
     const double fit = normX2 > 0 ? 1.0 - std::sqrt(res2) / std::sqrt(normX2) : 0.0;
     if (fits) fits[k] = fit;

@@ -127,11 +127,10 @@ void dist_build_sub(Tensor& t, int mode) {
     uint64_t mine[2] = {t.pos_begin, n};
     std::vector<uint64_t> bytes(P, 16), displs(P);
     for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * 16;
-    SF_CUDA(cudaMemcpyAsync(b.as<char>() + me * 16, mine, 16, cudaMemcpyHostToDevice, s));
+    h2d_small(s, b.as<char>() + me * 16, mine, 16);
     t.comm->allgatherv(b.as<char>() + me * 16, b.p, bytes.data(), displs.data(), s);
     std::vector<uint64_t> all(2 * P);
-    SF_CUDA(cudaMemcpyAsync(all.data(), b.p, (size_t)P * 16, cudaMemcpyDeviceToHost, s));
-    SF_CUDA(cudaStreamSynchronize(s));
+    d2h_small(s, all.data(), b.p, (size_t)P * 16);
     uint64_t at = 0;
     for (int k = 0; k < P; ++k) {
       if (all[2 * k] != at) throw StatusError{SF_ERR_INVALID_ARG, "distributed slices must tile the input in rank order"};
@@ -184,8 +183,7 @@ void dist_build_sub(Tensor& t, int mode) {
                                          nsel.as<uint64_t>(), (int64_t)n, s));
       count_launch(2);
       uint64_t c = 0;
-      SF_CUDA(cudaMemcpyAsync(&c, nsel.p, 8, cudaMemcpyDeviceToHost, s));
-      SF_CUDA(cudaStreamSynchronize(s));
+      d2h_small(s, &c, nsel.p, 8);
       scnt[q] = c;
     }
     sdis[q] = stot;
@@ -206,11 +204,10 @@ void dist_build_sub(Tensor& t, int mode) {
     DevBuf b((size_t)P * P * 8 + 16);
     std::vector<uint64_t> bytes(P, (uint64_t)P * 8), displs(P);
     for (int k = 0; k < P; ++k) displs[k] = (uint64_t)k * P * 8;
-    SF_CUDA(cudaMemcpyAsync(b.as<char>() + (size_t)me * P * 8, scnt.data(), (size_t)P * 8, cudaMemcpyHostToDevice, s));
+    h2d_small(s, b.as<char>() + (size_t)me * P * 8, scnt.data(), (size_t)P * 8);
     t.comm->allgatherv(b.as<char>() + (size_t)me * P * 8, b.p, bytes.data(), displs.data(), s);
     std::vector<uint64_t> all((size_t)P * P);
-    SF_CUDA(cudaMemcpyAsync(all.data(), b.p, (size_t)P * P * 8, cudaMemcpyDeviceToHost, s));
-    SF_CUDA(cudaStreamSynchronize(s));
+    d2h_small(s, all.data(), b.p, (size_t)P * P * 8);
     uint64_t at = 0;
     for (int k = 0; k < P; ++k) {
       rcnt[k] = all[(size_t)k * P + me];
@@ -248,10 +245,9 @@ void dist_build_sub(Tensor& t, int mode) {
     SF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, dk, dv, (int64_t)rtot, 0, end_bit, s));
     count_launch((uint64_t)(end_bit + 7) / 8 + 1);
     uint64_t k_first = 0;
-    SF_CUDA(cudaMemcpyAsync(&k_first, dk.Current(), 8, cudaMemcpyDeviceToHost, s));
-    SF_CUDA(cudaStreamSynchronize(s));
+    d2h_small(s, &k_first, dk.Current(), 8);
     uint32_t g0 = 0;
-    SF_CUDA(cudaMemcpy(&g0, gstart.as<uint32_t>() + k_first / Is, 4, cudaMemcpyDeviceToHost));
+    d2h_small(s, &g0, gstart.as<uint32_t>() + k_first / Is, 4);
     // sorted slot j is global matricized position g0 + j (complete rows were received)
     const uint64_t lo = cuts.c[me], hi = cuts.c[me + 1];
     first = lo > g0 ? lo - g0 : 0;

@@ -219,6 +219,19 @@ inline int frag_groups_per_warp(int R) {
   return lpn >= 1 && lpn <= 32 ? 32 / lpn : 1;
 }
 
+// Small host<->device transfers that must not queue behind bulk copies on the copy engines
+// (a plan's scalar reads would otherwise wait for a caller's multi-GB D2H on another stream):
+// a kernel moves the bytes through mapped pinned host memory, then the stream is synchronized.
+// Each call synchronizes `s`.  `n` pairs of (host dst, device src, bytes) for the reads.
+void d2h_small(cudaStream_t s, int n, void* const* dst, const void* const* src, const size_t* bytes);
+inline void d2h_small(cudaStream_t s, void* dst, const void* src, size_t bytes) {
+  d2h_small(s, 1, &dst, &src, &bytes);
+}
+void h2d_small(cudaStream_t s, void* dst, const void* src, size_t bytes);
+// Device-to-device copy by a kernel (any alignment; 16-byte vectors when both pointers allow):
+// keeps bulk plan copies off the copy engines a caller's H2D/D2H may be occupying.
+void d2d_copy(void* dst, const void* src, size_t bytes, cudaStream_t s);
+
 // ---- planning (sf_plan.cu) ----
 // upload || presort: decide and allocate (returns false: no mode qualifies / disabled by
 // SF_PRESORT=0 / not enough memory), per-segment work on the upload stream, CUB temp bytes

@@ -146,8 +146,7 @@ static void presort_finish(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_ou
     for (uint64_t a = 0; a < n; a += 2 * L) {
       const uint64_t b = std::min(n, a + L), c = std::min(n, a + 2 * L);
       if (b >= c) {  // odd run out: carried over
-        SF_CUDA(cudaMemcpyAsync(nxt.as<uint64_t>() + a, cur.as<uint64_t>() + a, (b - a) * 8,
-                                cudaMemcpyDeviceToDevice, t.stream));
+        d2d_copy(nxt.as<uint64_t>() + a, cur.as<uint64_t>() + a, (b - a) * 8, t.stream);
         continue;
       }
       size_t need = 0;
@@ -279,9 +278,12 @@ static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_f
     SF_CUDA(cudaGetLastError());
     uint32_t c[2];
     FeatAcc a;
-    SF_CUDA(cudaMemcpyAsync(c, nr.p, 8, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaMemcpyAsync(&a, accb.p, sizeof(FeatAcc), cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaStreamSynchronize(t.stream));
+    {
+      void* dst[2] = {c, &a};
+      const void* src[2] = {nr.p, accb.p};
+      const size_t nb[2] = {8, sizeof(FeatAcc)};
+      d2h_small(t.stream, 2, dst, src, nb);
+    }
     f->num_slices = c[0];
     f->num_fibers = c[1];
     f->max_nnz_per_slice = a.max_slice;
@@ -593,9 +595,12 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
   p.row_begin = p.row_end = 0;
   if (nl) {
     uint64_t kb, ke;
-    SF_CUDA(cudaMemcpyAsync(&kb, keys.as<uint64_t>() + lo, 8, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaMemcpyAsync(&ke, keys.as<uint64_t>() + hi - 1, 8, cudaMemcpyDeviceToHost, t.stream));
-    SF_CUDA(cudaStreamSynchronize(t.stream));
+    {
+      void* dst[2] = {&kb, &ke};
+      const void* src[2] = {keys.as<uint64_t>() + lo, keys.as<uint64_t>() + hi - 1};
+      const size_t nb[2] = {8, 8};
+      d2h_small(t.stream, 2, dst, src, nb);
+    }
     p.row_begin = kb / t.dims[s];
     p.row_end = ke / t.dims[s] + 1;
   }
@@ -646,7 +651,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       if (dk.Current() == k0.as<uint64_t>()) tkeys = std::move(k0); else tkeys = std::move(k1);
       if (dv.Current() != perm.as<uint32_t>()) perm = std::move(p1);
     } else {
-      SF_CUDA(cudaMemcpyAsync(perm.p, pos0.as<uint32_t>() + lo, nl * 4, cudaMemcpyDeviceToDevice, t.stream));
+      d2d_copy(perm.p, pos0.as<uint32_t>() + lo, nl * 4, t.stream);
       pos0.release();
     }
   }
@@ -732,8 +737,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
           SF_CUDA(cudaMemsetAsync(above.p, 0, 32 * 8, t.stream));
           hot_above_kernel<<<grid_for(dimmax), 256, 0, t.stream>>>(hc, above.as<unsigned long long>());
           count_launch();
-          SF_CUDA(cudaMemcpyAsync(h, above.p, 32 * 8, cudaMemcpyDeviceToHost, t.stream));
-          SF_CUDA(cudaStreamSynchronize(t.stream));
+          d2h_small(t.stream, h, above.p, 32 * 8);
         };
         unsigned long long h[32];
         for (int j = 0; j < 32; ++j) hc.tau[j] = (j == 31) ? 0xFFFFFFFFu : ((1u << j) - 1u);  // 0, 1, 3, 7, ...
@@ -756,15 +760,14 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
           hslot[q].alloc(I * 4 + 16);
           hot_flag_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt[q].as<uint32_t>(), I, tau, hslot[q].as<uint32_t>());
           uint32_t last_flag = 0, last_slot = 0;
-          SF_CUDA(cudaMemcpyAsync(&last_flag, hslot[q].as<uint32_t>() + I - 1, 4, cudaMemcpyDeviceToHost, t.stream));
+          d2h_small(t.stream, &last_flag, hslot[q].as<uint32_t>() + I - 1, 4);
           size_t tb = 0;
           SF_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, hslot[q].as<uint32_t>(), hslot[q].as<uint32_t>(),
                                                 (int64_t)I, t.stream));
           DevBuf tmp(tb + 16);
           SF_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, tb, hslot[q].as<uint32_t>(), hslot[q].as<uint32_t>(),
                                                 (int64_t)I, t.stream));
-          SF_CUDA(cudaMemcpyAsync(&last_slot, hslot[q].as<uint32_t>() + I - 1, 4, cudaMemcpyDeviceToHost, t.stream));
-          SF_CUDA(cudaStreamSynchronize(t.stream));
+          d2h_small(t.stream, &last_slot, hslot[q].as<uint32_t>() + I - 1, 4);
           const uint64_t cnt = (uint64_t)last_slot + last_flag;
           count_launch(2);
           if (cnt == 0) continue;
@@ -829,7 +832,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       DevBuf dptr(sizeof(uint32_t*) * SF_MAX_MODES);
       uint32_t* hptr[SF_MAX_MODES] = {};
       for (int m = 0; m < N; ++m) hptr[m] = g.dst[m];
-      SF_CUDA(cudaMemcpyAsync(dptr.p, hptr, sizeof(hptr), cudaMemcpyHostToDevice, t.stream));
+      h2d_small(t.stream, dptr.p, hptr, sizeof(hptr));
       uint32_t* const* dd = reinterpret_cast<uint32_t* const*>(dptr.p);
       switch (W) {
         case 4: gather_aos_kernel<4><<<grid_for(nl), 256, 0, t.stream>>>(t.aos.as<uint32_t>(), perm.as<uint32_t>(), nl, N, dd, g.vdst); break;
@@ -888,10 +891,12 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
                                             (int64_t)tiles_bound, t.stream));
       count_launch(5);
       uint32_t nr = 0, last_off = 0, last_n = 0;
-      SF_CUDA(cudaMemcpyAsync(&nr, nruns.p, 4, cudaMemcpyDeviceToHost, t.stream));
-      SF_CUDA(cudaMemcpyAsync(&last_off, coff.as<uint32_t>() + tiles_bound - 1, 4, cudaMemcpyDeviceToHost, t.stream));
-      SF_CUDA(cudaMemcpyAsync(&last_n, nch.as<uint32_t>() + tiles_bound - 1, 4, cudaMemcpyDeviceToHost, t.stream));
-      SF_CUDA(cudaStreamSynchronize(t.stream));
+      {
+        void* dst[3] = {&nr, &last_off, &last_n};
+        const void* src[3] = {nruns.p, coff.as<uint32_t>() + tiles_bound - 1, nch.as<uint32_t>() + tiles_bound - 1};
+        const size_t nb[3] = {4, 4, 4};
+        d2h_small(t.stream, 3, dst, src, nb);
+      }
       trace_mark("build: chunk count sync");
       p.num_tiles = nr;
       p.num_chunks = (uint64_t)last_off + last_n;

@@ -288,7 +288,7 @@ static constexpr double kL2MaxRevisit = 0.25;
 static constexpr double kL2YInCache = 32.0 * 1024 * 1024;
 
 static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local,
-                           sf_launch_t& l) {
+                           sf_launch_t& l, double max_tiles = 1e30) {
   if (l.kernel != SF_KERNEL_FRAG || l.staged_mask != 0 || (l.flags & SF_LAUNCH_DETERMINISTIC) || nnz_local == 0 ||
       f.nnz == 0)
     return;
@@ -302,6 +302,7 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
     const double F = (double)t.dims[m] * RB;
     if (F < kL2MinFactorBytes || F <= bestF) continue;
     const double T = std::ceil(F / kL2BlockBytes);
+    if (T > max_tiles) continue;
     double rho = 0;
     if (Yb > kL2YInCache) {
       double touched = 0;
@@ -338,7 +339,8 @@ static bool l2_refine_enabled() {
 // staged nor L2-tiled total more than ~1.3x L2.
 // ---------------------------------------------------------------------------
 static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
-static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 32 * 1024;
+static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 16 * 1024;
+static constexpr double kHotMaxTiles = 8;
 
 static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC) || l.staged_mask != 0) return;
@@ -349,13 +351,15 @@ static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
     if (F >= 16.0 * 1024 * 1024) gathered += F;
   }
   if (gathered < kHotMinGatheredBytes || debug_opt("no_hot")) return;  // SF_DEBUG A/B
-  // the hot-row class: owner stores, 1024 threads (one CTA per SM), chunks of 64 nonzeros per
-  // warp and 32 MB of hot rows -- over the exhaustive sparse sweeps of nell-1 and deli-4d
-  // (sweep.py --sparse, 199-283 launches per mode, profiles/r02/sweeps/) the best fixed
-  // class: >= 0.945 of each mode's sweep best, 0.980 on average
+  // the hot-row class: owner stores, 1024 threads (one CTA per SM), 32 MB of hot rows, no L2
+  // tiles, and stages of 4 register batches per lane group (chunk = 8 groups x 4 x U nonzeros:
+  // 64 at R >= 32 where U = 2, 128 at R = 16 where U = 4) -- the best fixed class over the
+  // exhaustive sparse sweeps (sweep.py --sparse, 143-283 launches per mode, nell-1, deli-4d,
+  // flickr-3d, deli-3d, flickr-4d: profiles/r02/sweeps/); L2 tiles on top of the hot rows won
+  // only 1-7 % on 6 of 17 modes and lost up to 20 % on others
   l.hot_kb = (l.flags & SF_LAUNCH_L2_TILES) ? kHotKBTiled : kHotKB;
   l.block_threads = 1024;
-  l.chunk_nnz = 64;
+  l.chunk_nnz = rank >= 32 ? 64 : 128;
   l.ctas_per_sm = 0;
   l.flags &= ~SF_LAUNCH_NO_OWNER_STORES;
   normalize_launch(t, mode, rank, l);
@@ -383,8 +387,21 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
   // hot-row cache first: where it applies to an unstaged pick it beats L2 tiles (deli-4d 1.2-1.8x,
   // flickr-3d 1.2x per mode) or ties them within 3 % (nell-1), profiles/r02/hot_sweep_g06.jsonl
   hot_refine(t, mode, rank, l);
-  if (l.hot_kb == 0 && l2_refine_enabled() && !(picked && g_model.l2_classes))
+  if (l.hot_kb != 0 && l2_refine_enabled()) {
+    // hot rows + L2 tiles when the tile rule holds with few tiles (a <= 512 MB factor in 64 MB
+    // blocks; long rows of a small Y): nell-1 modes 0/1 and amazon modes 1/2; many-tile
+    // picks (deli-4d, flickr: 28-35 tiles) lose to hot rows alone (profiles/r02/sweeps/)
+    sf_launch_t c = l;
+    l2_tile_refine(t, f, mode, rank, nnz_local, c, kHotMaxTiles);
+    if (c.flags & SF_LAUNCH_L2_TILES) {
+      c.hot_kb = kHotKBTiled;
+      c.chunk_nnz = 128;
+      normalize_launch(t, mode, rank, c);
+      if (frag_smem_bytes(t, mode, rank, c) <= t.smem_optin) l = c;
+    }
+  } else if (l.hot_kb == 0 && l2_refine_enabled() && !(picked && g_model.l2_classes)) {
     l2_tile_refine(t, f, mode, rank, nnz_local, l);
+  }
   return l;
 }
 

@@ -80,8 +80,10 @@ class TorchAllgatherv:
                         _dev_view(recv + displs[k], nbytes[k], self.device).copy_(blocks[k])
             s.synchronize()
             return 0
-        except Exception as e:  # never raise through the C ABI
+        except Exception as e:  # never raise through the C ABI: report, return failure
+            import sys
             self.errors.append(repr(e))
+            print(f"TorchAllgatherv: {e!r}", file=sys.stderr, flush=True)
             return 1
 
 

@@ -99,3 +99,22 @@ def test_streamed_heavy_row(cuda_device):
     for segments, streams in ((8, 4), (3, 2)):
         rel = _streamed_check(dims, inds, vals, facs, R, 0, rows, segments, streams)
         assert rel <= G.TOL, (segments, rel)
+
+
+def test_streamed_device_footprint(cuda_device):
+    """F2 (tensors larger than HBM): the streamed path holds only
+    streams x segment buffers on the device (sf_device_bytes), not the tensor."""
+    cfg = synth.CONFIGS["nell2"]
+    inds, vals = synth.config_tensor(cfg)
+    h_inds = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    h_vals = torch.from_numpy(vals).pin_memory()
+    d_facs = synth.config_factors_device(cfg)
+    y = torch.empty((cfg.dims[0], cfg.rank), device="cuda")
+    tensor_bytes = 4 * (cfg.nmodes + 1) * cfg.nnz
+    sf.device_bytes(reset_peak=True)
+    base, _ = sf.device_bytes()
+    sf.mttkrp_streamed(cfg.dims, h_inds, h_vals, d_facs, 0, y, 32, 4)
+    torch.cuda.synchronize()
+    _, peak = sf.device_bytes()
+    # 4 ring slots of one 1/32 segment each (raw arrays + sort scratch ~ 2.5x the raw bytes)
+    assert peak - base < 0.5 * tensor_bytes, (peak - base, tensor_bytes)
