@@ -482,28 +482,42 @@ void boundary_zero3_r16(const Frag3Params& fp, uint32_t ctas, uint32_t groups, f
 void boundary_zero3_r32(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out, cudaStream_t s);
 void boundary_zero3_r64(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out, cudaStream_t s);
 
+// Dynamic shared memory opted in per (device, instantiation, record format): only ever RAISED
+// (the occupancy query and the launch share it; lowering the attribute for a smaller plan
+// would make a later launch of a larger plan fail with "invalid argument").
+template <int N, int R, int S>
+size_t& frag3_smem_optin(int dev, int v) {
+  static size_t set[16][2] = {};
+  static size_t spill = 0;
+  return (dev < 16 && v < 2) ? set[dev][v] : spill;
+}
+
+template <int N, int R, int S, class K>
+void frag3_ensure_smem(K k, int v, size_t smem) {
+  int dev = 0;
+  SF_CUDA(cudaGetDevice(&dev));
+  size_t& cur = frag3_smem_optin<N, R, S>(dev, v);
+  if (dev >= 16 || smem > cur) {
+    SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (dev < 16) cur = smem;
+  }
+}
+
 template <int N, int R, int S>
 void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s) {
   auto k = frag3_kernel<N, R, S, kRecPlain>;
   if constexpr (N >= 4) {
     if (fp.W == 4) k = frag3_kernel<N, R, S, kRecPacked>;
   }
-  // opt-in shared memory once per (device, instantiation, size): host overhead of small launches
-  static size_t smem_set[16][2] = {};
-  int dev = 0;
-  SF_CUDA(cudaGetDevice(&dev));
   const int v = (fp.W == 4 && N >= 4) ? 1 : 0;
-  if (dev >= 16 || smem > smem_set[dev][v]) {
-    SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    if (dev < 16) smem_set[dev][v] = smem;
-  }
+  frag3_ensure_smem<N, R, S>(k, v, smem);
   k<<<grid, threads, smem, s>>>(fp);
 }
 
 template <int N, int R, int S>
 int frag3_occ_one(int threads, size_t smem) {
   auto k = frag3_kernel<N, R, S, kRecPlain>;
-  SF_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  frag3_ensure_smem<N, R, S>(k, 0, smem);
   int nb = 0;
   SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));
   return nb;

@@ -300,3 +300,25 @@ def test_shards_with_tiled_plans(cuda_device, kind):
                 Y, info = G.run(dims, inds, vals, facs, R, modes=[n], launch=L, shard=(P, p), device_input=False)
                 acc += Y[n]
             assert np.array_equal(acc, Yfull), (kind, n, P)
+
+
+def test_smem_optin_never_lowered(cuda_device):
+    """Two plans of the same kernel instantiation with different shared-memory needs: the
+    smaller plan's occupancy query / launch must not lower the opt-in below what the larger
+    plan needs (a later launch of the larger plan failed with "invalid argument")."""
+    dims, R = (300, 200, 100), 32
+    inds, vals = synth.gen_coo(dims, 20000, 3, zipf=(0.8, 0.8, 0.8))
+    facs = synth.gen_factors(dims, R, 4)
+    tf = [G.dev_f(f) for f in facs]
+    with sf.Tensor(dims, G.dev_inds(inds), G.dev_f(vals)) as t:
+        big = sf.Launch.make(kernel=FRAG, block_threads=1024, chunk_nnz=128)
+        small = sf.Launch.make(kernel=FRAG, block_threads=256, chunk_nnz=64)
+        ys = {}
+        for n, L in ((0, big), (1, small), (2, big)):
+            t.set_launch(n, R, L)
+        for n in (0, 1, 0, 2, 1, 0):
+            ys[n] = torch.empty((dims[n], R), device="cuda:0")
+            t.mttkrp(n, tf, ys[n])
+        torch.cuda.synchronize()
+        for n in range(3):
+            G.assert_parity(ys[n].cpu().numpy(), dims, inds, vals, facs, R, n)
