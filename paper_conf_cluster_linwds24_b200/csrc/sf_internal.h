@@ -147,6 +147,7 @@ struct Tensor {
   DevBuf pre[SF_MAX_MODES];
   bool have_pre[SF_MAX_MODES] = {};
   DevBuf pre_alt;              // composed keys of a segment before its sort (upload only)
+  DevBuf hot_cnt[SF_MAX_MODES];  // hot-row cache: nonzeros per row of mode m (whole handle), lazily
   uint64_t pre_seg_len = 0;
   int pre_pb = 0;              // position bits
   cudaStream_t stream = nullptr;               // internal stream for planning

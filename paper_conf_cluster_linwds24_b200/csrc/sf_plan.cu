@@ -401,6 +401,12 @@ __global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32
 }
 
 // ---- hot-row cache (launch.hot_kb; DESIGN.md §5 "hot-row cache") ----
+// cnt[x] = nonzeros of the handle whose mode-m index is x
+__global__ void hot_count_all_kernel(const uint32_t* __restrict__ ind, uint64_t n, uint32_t* __restrict__ cnt) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) atomicAdd(cnt + __ldg(ind + k), 1u);
+}
+
 // cnt[x] = nonzeros of this plan whose gathered index (mode m) is x
 __global__ void hot_count_kernel(const uint32_t* __restrict__ ind, const uint32_t* __restrict__ perm, uint64_t n,
                                  uint32_t* __restrict__ cnt) {
@@ -694,6 +700,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     // memory, not the L2-tiled mode) and large enough for their rows to be scattered
     bool hot_q[SF_MAX_MODES] = {};
     std::vector<DevBuf> hcnt(SF_MAX_MODES), hslot(SF_MAX_MODES);
+    const uint32_t* hcnt_ptr[SF_MAX_MODES] = {};
     p.hot_total = 0;
     for (int q = 0; q < SF_MAX_MODES; ++q) {
       p.hot_bit[q] = 0;
@@ -717,15 +724,27 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       for (int q = 0; q < N - 1; ++q) {
         if (!hot_q[q]) continue;
         const int m = slot_mode[q];
-        hcnt[q].alloc(t.dims[m] * 4 + 16);
-        SF_CUDA(cudaMemsetAsync(hcnt[q].p, 0, t.dims[m] * 4, t.stream));
-        hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
-                                                             hcnt[q].as<uint32_t>());
-        count_launch();
-        hc.cnt[hc.n] = hcnt[q].as<uint32_t>();
+        // row frequencies of mode m: over this plan's nonzeros when the handle is a shard,
+        // else over the whole tensor -- counted once per (handle, mode) and reused by every
+        // plan that gathers mode m
+        const bool whole = t.nranks == 1;
+        DevBuf* cnt = whole ? &t.hot_cnt[m] : &hcnt[q];
+        if (!cnt->p) {
+          cnt->alloc(t.dims[m] * 4 + 16);
+          SF_CUDA(cudaMemsetAsync(cnt->p, 0, t.dims[m] * 4, t.stream));
+          if (whole)
+            hot_count_all_kernel<<<grid_for(n), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), n, cnt->as<uint32_t>());
+          else
+            hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
+                                                                 cnt->as<uint32_t>());
+          count_launch();
+        }
+        hcnt_ptr[q] = cnt->as<uint32_t>();
+        hc.cnt[hc.n] = cnt->as<uint32_t>();
         hc.dim[hc.n] = t.dims[m];
         ++hc.n;
       }
+      trace_mark("build: hot counts");
       if (hc.n) {
         // one global threshold tau (rows with count > tau are hot) so the hot rows of every
         // slot fit the budget: the static cache of the most frequently gathered rows
@@ -758,7 +777,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
           const int m = slot_mode[q];
           const uint64_t I = t.dims[m];
           hslot[q].alloc(I * 4 + 16);
-          hot_flag_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt[q].as<uint32_t>(), I, tau, hslot[q].as<uint32_t>());
+          hot_flag_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt_ptr[q], I, tau, hslot[q].as<uint32_t>());
           uint32_t last_flag = 0, last_slot = 0;
           d2h_small(t.stream, &last_flag, hslot[q].as<uint32_t>() + I - 1, 4);
           size_t tb = 0;
@@ -772,19 +791,20 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
           count_launch(2);
           if (cnt == 0) continue;
           p.hot_rows[q].alloc(cnt * 4 + 16);
-          hot_rows_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt[q].as<uint32_t>(), hslot[q].as<uint32_t>(), I, tau,
+          hot_rows_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt_ptr[q], hslot[q].as<uint32_t>(), I, tau,
                                                              p.hot_rows[q].as<uint32_t>());
           count_launch();
           p.hot_bit[q] = packed ? (1u << index_bits(I)) : 0x80000000u;
           p.hot_count[q] = cnt;
           p.hot_off[q] = total;
           total += cnt;
-          rp.hcnt[1 + q] = hcnt[q].as<uint32_t>();
+          rp.hcnt[1 + q] = hcnt_ptr[q];
           rp.hslot[1 + q] = hslot[q].as<uint32_t>();
           rp.hbit[1 + q] = p.hot_bit[q];
         }
         rp.htau = tau;
         p.hot_total = total;
+        trace_mark("build: hot rows");
         if (total) p.hot_cache.alloc(total * rank * 4 + 64);
         SF_CUDA(cudaGetLastError());
       }
