@@ -287,8 +287,17 @@ static constexpr double kL2MinFactorBytes = 160.0 * 1024 * 1024;  // ~1.3x L2: s
 static constexpr double kL2MaxRevisit = 0.25;
 static constexpr double kL2YInCache = 32.0 * 1024 * 1024;
 
+// expected Y revisit ratio of tiling the order by T blocks: T * touched(T) / nnz, touched(T) =
+// the expected rows of Y a tile touches from the log2 slice-length histogram
+static double revisit_ratio(const sf_features_t& f, double T) {
+  double touched = 0;
+  for (int b = 0; b < SF_HIST_BINS; ++b)
+    touched += (double)f.slice_hist[b] * (1.0 - std::exp(-1.44 * std::ldexp(1.0, b) / T));
+  return f.nnz ? T * touched / (double)f.nnz : 0.0;
+}
+
 static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local,
-                           sf_launch_t& l, double max_tiles = 1e30) {
+                           sf_launch_t& l) {
   if (l.kernel != SF_KERNEL_FRAG || l.staged_mask != 0 || (l.flags & SF_LAUNCH_DETERMINISTIC) || nnz_local == 0 ||
       f.nnz == 0)
     return;
@@ -302,14 +311,7 @@ static void l2_tile_refine(const Tensor& t, const sf_features_t& f, int mode, in
     const double F = (double)t.dims[m] * RB;
     if (F < kL2MinFactorBytes || F <= bestF) continue;
     const double T = std::ceil(F / kL2BlockBytes);
-    if (T > max_tiles) continue;
-    double rho = 0;
-    if (Yb > kL2YInCache) {
-      double touched = 0;
-      for (int b = 0; b < SF_HIST_BINS; ++b)
-        touched += (double)f.slice_hist[b] * (1.0 - std::exp(-1.44 * std::ldexp(1.0, b) / T));
-      rho = T * touched / (double)f.nnz;
-    }
+    const double rho = (Yb > kL2YInCache) ? revisit_ratio(f, T) : 0.0;
     if (rho > max_revisit) continue;
     best = m;
     bestF = F;
@@ -340,7 +342,38 @@ static bool l2_refine_enabled() {
 // ---------------------------------------------------------------------------
 static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
 static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 16 * 1024;
-static constexpr double kHotMaxTiles = 8;
+// hot rows + L2 tiles (3-way tensors): tile one gathered factor of 64-512 MB in 64 MB blocks
+// (16 MB blocks below 256 MB) when that gives <= 8 tiles and the Y revisit ratio <= 0.25
+static constexpr double kHotTileMinBytes = 64.0 * 1024 * 1024, kHotTileMaxBytes = 512.0 * 1024 * 1024;
+static constexpr double kHotTileMaxTiles = 8, kHotTileMaxRevisit = 0.25;
+
+static void hot_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, sf_launch_t& l) {
+  if (l.hot_kb == 0 || l.staged_mask != 0 || t.nmodes != 3 || f.nnz == 0) return;
+  const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
+  int best = -1;
+  double bestF = 0, bestBlock = 0;
+  for (int m = 0; m < t.nmodes; ++m) {
+    if (m == mode) continue;
+    const double F = (double)t.dims[m] * RB;
+    if (F < kHotTileMinBytes || F > kHotTileMaxBytes || F <= bestF) continue;
+    const double block = F >= 256.0 * 1024 * 1024 ? 64.0 * 1024 * 1024 : 16.0 * 1024 * 1024;
+    const double T = std::ceil(F / block);
+    if (T > kHotTileMaxTiles) continue;
+    if ((Yb > kL2YInCache ? revisit_ratio(f, T) : 0.0) > kHotTileMaxRevisit) continue;
+    best = m;
+    bestF = F;
+    bestBlock = block;
+  }
+  if (best < 0) return;
+  sf_launch_t c = l;
+  c.staged_mask = 1u << best;
+  c.block_rows[best] = (uint32_t)std::max(1.0, bestBlock / RB);
+  c.flags = (c.flags | SF_LAUNCH_L2_TILES) & ~SF_LAUNCH_NO_OWNER_STORES;
+  c.hot_kb = kHotKBTiled;
+  c.chunk_nnz = 128;
+  normalize_launch(t, mode, rank, c);
+  if (frag_smem_bytes(t, mode, rank, c) <= t.smem_optin) l = c;
+}
 
 static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
   if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC) || l.staged_mask != 0) return;
@@ -369,7 +402,10 @@ static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
 sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int rank, uint64_t nnz_local) {
   sf_launch_t l{};
   bool picked = false;
-  if (g_have_model && frag_supported(t.nmodes, rank) && nnz_local > 0) {
+  // the tree was trained on 1e6..3e7-nonzero tensors; below 2^20 nonzeros the launch is latency-
+  // bound (~10 us) and the rule selector (stage every small factor whole) is within 5 % of the
+  // sweep best on configs[0] (profiles/r02/sweeps/sweep_tiny.jsonl), the tree's picks 0.55-0.87
+  if (g_have_model && frag_supported(t.nmodes, rank) && nnz_local >= (1u << 20)) {
     double x[32];
     const int nx = selector_features(t, f, mode, rank, nnz_local, x);
     if (nx == g_model.nfeat) {
@@ -383,23 +419,16 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
     }
   }
   if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
-  // the hand rule refines picks of a selector that cannot choose L2 tiles itself
-  // hot-row cache first: where it applies to an unstaged pick it beats L2 tiles (deli-4d 1.2-1.8x,
-  // flickr-3d 1.2x per mode) or ties them within 3 % (nell-1), profiles/r02/hot_sweep_g06.jsonl
+  // hot-row cache first: where it applies to an unstaged pick it beats L2 tiles alone (deli-4d
+  // 1.2-1.8x, flickr-3d 1.2x per mode) or ties them (nell-1), profiles/r02/hot_sweep_g06.jsonl;
+  // then, for 3-way tensors, L2 tiles of one mid-size factor on top (hot_tile_refine): amazon
+  // 0.81x / nell-1 0.96-0.99x the hot-only time; 4-way tensors lose 3-15 % with any tiling
+  // (deli-4d), profiles/r02/sweeps/
   hot_refine(t, mode, rank, l);
-  if (l.hot_kb != 0 && l2_refine_enabled()) {
-    // hot rows + L2 tiles when the tile rule holds with few tiles (a <= 512 MB factor in 64 MB
-    // blocks; long rows of a small Y): nell-1 modes 0/1 and amazon modes 1/2; many-tile
-    // picks (deli-4d, flickr: 28-35 tiles) lose to hot rows alone (profiles/r02/sweeps/)
-    sf_launch_t c = l;
-    l2_tile_refine(t, f, mode, rank, nnz_local, c, kHotMaxTiles);
-    if (c.flags & SF_LAUNCH_L2_TILES) {
-      c.hot_kb = kHotKBTiled;
-      c.chunk_nnz = 128;
-      normalize_launch(t, mode, rank, c);
-      if (frag_smem_bytes(t, mode, rank, c) <= t.smem_optin) l = c;
-    }
-  } else if (l.hot_kb == 0 && l2_refine_enabled() && !(picked && g_model.l2_classes)) {
+  if (l.hot_kb != 0) {
+    if (l2_refine_enabled()) hot_tile_refine(t, f, mode, rank, l);
+  } else if (l2_refine_enabled() && !(picked && g_model.l2_classes)) {
+    // the hand rule refines picks of a selector that cannot choose L2 tiles itself
     l2_tile_refine(t, f, mode, rank, nnz_local, l);
   }
   return l;

@@ -150,6 +150,7 @@ def main():
             print(line, flush=True)
             if outf:
                 outf.write(line + "\n")
+                outf.flush()
         ok = sorted([r for r in results if r["ms"]], key=lambda r: r["ms"])
         best = ok[0]
         rank_of_pick = sum(1 for r in ok if r["ms"] < t_pick) + 1
@@ -159,6 +160,10 @@ def main():
         print(json.dumps(summ), flush=True)
         if outf:
             outf.write(json.dumps(summ) + "\n")
+            outf.flush()
+        T.plan_release(n, R)  # one plan resident at a time (amazon: 1.74 B nonzeros)
+        del out
+        torch.cuda.empty_cache()
     T.close()
 
 

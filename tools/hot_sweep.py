@@ -23,6 +23,9 @@ def main():
     ap.add_argument("--budgets", default="0,16,32,64,128,256")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--modes", default=None)
+    ap.add_argument("--persist", action="store_true",
+                    help="also time every variant with the hot block persisting in L2 (SF_DEBUG=l2_persist)")
+    ap.add_argument("--no-tiles-variant", action="store_true", help="only the selector's tiling choice")
     args = ap.parse_args()
     import torch
 
@@ -36,14 +39,15 @@ def main():
         T = sf.Tensor(cfg.dims, inds, vals)
         del inds, vals
         torch.cuda.empty_cache()
-        s = torch.cuda.current_stream()
+        s = torch.cuda.Stream()
         modes = range(N) if args.modes is None else [int(x) for x in args.modes.split(",")]
         for n in modes:
             T.plan(n, R)
             base = T.plan_info(n, R)["launch"]
             out = torch.empty((cfg.dims[n], R), dtype=torch.float32, device="cuda")
             variants = []
-            for tiles in ([True, False] if base["flags"] & sf.LAUNCH_L2_TILES else [None]):
+            tv = [True, False] if (base["flags"] & sf.LAUNCH_L2_TILES) and not args.no_tiles_variant else [None]
+            for tiles in tv:
                 for hb in budgets:
                     variants.append((tiles, hb))
             for tiles, hb in variants:
@@ -56,18 +60,24 @@ def main():
                                    flags=flags, hot_kb=hb * 1024)
                 T.set_launch(n, R, L)
                 info = T.plan_info(n, R)
-                for _ in range(3):
-                    T.mttkrp(n, facs, out)
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record(s)
-                for _ in range(args.reps):
-                    T.mttkrp(n, facs, out)
-                e1.record(s)
-                torch.cuda.synchronize()
-                ms = e0.elapsed_time(e1) / args.reps
-                print(json.dumps({"config": name, "mode": n, "l2tiles": bool(flags & sf.LAUNCH_L2_TILES),
-                                  "hot_mb": hb, "ms": round(ms, 4), "plan_ms": round(info["plan_ms"], 2),
-                                  "selector": base}), flush=True)
+                for persist in ([False, True] if args.persist else [False]):
+                    if persist:
+                        os.environ["SF_DEBUG"] = "l2_persist"
+                    else:
+                        os.environ.pop("SF_DEBUG", None)
+                    for _ in range(3):
+                        T.mttkrp(n, facs, out, stream=s)
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(s)
+                    for _ in range(args.reps):
+                        T.mttkrp(n, facs, out, stream=s)
+                    e1.record(s)
+                    torch.cuda.synchronize()
+                    ms = e0.elapsed_time(e1) / args.reps
+                    print(json.dumps({"config": name, "mode": n, "l2tiles": bool(flags & sf.LAUNCH_L2_TILES),
+                                      "hot_mb": hb, "persist": persist, "ms": round(ms, 4),
+                                      "plan_ms": round(info["plan_ms"], 2), "selector": base}), flush=True)
+                os.environ.pop("SF_DEBUG", None)
             T.plan_release(n, R)
             del out
             torch.cuda.empty_cache()

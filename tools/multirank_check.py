@@ -90,6 +90,20 @@ def main():
             if not same:
                 ok = False
                 msgs.append(f"dist v2 mode {n} rank {rank}: plan/Y differ from v1")
+            # the selector's own launches (hot rows where they apply) on both: integer data, so
+            # any summation order gives the same Y bit for bit
+            T1.plan_release(n, R)
+            T2.plan_release(n, R)
+            T1.plan(n, R)
+            T2.plan(n, R)
+            y1.zero_()
+            y2.zero_()
+            T1.mttkrp(n, facs, y1)
+            T2.mttkrp(n, facs, y2)
+            torch.cuda.synchronize()
+            if not torch.equal(y1, y2):
+                ok = False
+                msgs.append(f"dist v2 mode {n} rank {rank}: auto-planned Y differs from v1")
     # CP-ALS on the shards == CP-ALS on one rank (same initial factors) up to fp32 summation
     # order (the shards sum M and the Grams in a different order): the bar of
     # tests/test_gpu_cpals.py against the fp64 oracle (fits 2e-4 over 3 sweeps, factors 2e-3
