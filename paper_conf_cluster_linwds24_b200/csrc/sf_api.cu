@@ -19,9 +19,18 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "sf_internal.h"
 
 namespace sf {
+
+// NVTX ranges around every public entry point (visible in nsys / ncu timelines; a no-op
+// without a profiler attached).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 std::atomic<uint64_t> g_launches{0};
 static thread_local std::string g_err;
@@ -439,6 +448,7 @@ extern "C" {
 sf_status sf_tensor_create_ex(int nmodes, const uint64_t* dims, uint64_t nnz,
                               const uint32_t* const* inds, const float* vals, int segments,
                               int streams, sf_tensor_t* out) {
+  NvtxRange nvtx_("sf_tensor_create_ex");
   return guard([&]() -> sf_status {
     if (!out) throw StatusError{SF_ERR_INVALID_ARG, "out is NULL"};
     *out = nullptr;
@@ -537,6 +547,7 @@ sf_status sf_set_shard(sf_tensor_t h, int nranks, int rank) {
 }
 
 sf_status sf_plan(sf_tensor_t h, int mode, int rank) {
+  NvtxRange nvtx_("sf_plan");
   return guard([&]() -> sf_status {
     if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
     Tensor* t = as_tensor(h);
@@ -548,6 +559,7 @@ sf_status sf_plan(sf_tensor_t h, int mode, int rank) {
 }
 
 sf_status sf_plan_release(sf_tensor_t h, int mode, int rank) {
+  NvtxRange nvtx_("sf_plan_release");
   return guard([&]() -> sf_status {
     if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
     Tensor* t = as_tensor(h);
@@ -571,6 +583,7 @@ sf_status sf_trim_cache(void) {
 }
 
 sf_status sf_set_launch(sf_tensor_t h, int mode, int rank, const sf_launch_t* launch) {
+  NvtxRange nvtx_("sf_set_launch");
   return guard([&]() -> sf_status {
     if (!h || !launch) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
     Tensor* t = as_tensor(h);
@@ -650,6 +663,7 @@ sf_status sf_plan_export(sf_tensor_t h, int mode, int rank, uint64_t* perm_host,
 
 sf_status sf_mttkrp(sf_tensor_t h, int mode, const float* const* factors, int rank, float* out,
                     void* stream) {
+  NvtxRange nvtx_("sf_mttkrp");
   return guard([&]() -> sf_status {
     if (!h || !factors || !out) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
     Tensor* t = as_tensor(h);
@@ -678,6 +692,7 @@ sf_status sf_shard_rows(sf_tensor_t h, int mode, int rank, uint64_t* row_begin, 
 }
 
 sf_status sf_allgather_rows(sf_tensor_t h, int mode, int rank, const float* local, float* full, void* stream) {
+  NvtxRange nvtx_("sf_allgather_rows");
   return guard([&]() -> sf_status {
     if (!h || !full || !local) throw StatusError{SF_ERR_INVALID_ARG, "NULL argument"};
     Tensor* t = as_tensor(h);
@@ -710,6 +725,7 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
                              const uint32_t* const* inds_host, const float* vals_host,
                              const float* const* factors, int rank, int mode, float* out,
                              int segments, int streams) {
+  NvtxRange nvtx_("sf_mttkrp_streamed");
   return guard([&]() -> sf_status {
     if (nmodes < 2 || nmodes > SF_MAX_MODES || !dims || !factors || !out)
       throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
@@ -798,6 +814,7 @@ sf_status sf_rows_op(float* Y, int rank, const int64_t* rows, float* buf, int co
 
 sf_status sf_cpals(sf_tensor_t h, int rank, float* const* factors, int iters, double tol, double* fits,
                    int* iters_done, void* stream) {
+  NvtxRange nvtx_("sf_cpals");
   return guard([&]() -> sf_status {
     if (!h || !factors || iters < 0) throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
     Tensor* t = as_tensor(h);
