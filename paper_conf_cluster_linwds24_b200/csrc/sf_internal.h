@@ -148,6 +148,8 @@ struct Tensor {
   bool have_pre[SF_MAX_MODES] = {};
   DevBuf pre_alt;              // composed keys of a segment before its sort (upload only)
   DevBuf hot_cnt[SF_MAX_MODES];  // hot-row cache: nonzeros per row of mode m (whole handle), lazily
+  double hot_cover[SF_MAX_MODES] = {-1, -1, -1, -1, -1, -1, -1, -1};  // share of nonzeros in the
+                                 // hottest 2^18 rows of mode m (hot_coverage), -1 = not measured
   uint64_t pre_seg_len = 0;
   int pre_pb = 0;              // position bits
   cudaStream_t stream = nullptr;               // internal stream for planning
@@ -254,6 +256,10 @@ int selector_candidates(const Tensor& t, int mode, int rank, sf_launch_t* out);
 void set_selector_model(const int32_t* feature, const double* threshold, const int32_t* left,
                         const int32_t* right, const int32_t* value, int n_nodes, int n_features);
 size_t frag_smem_bytes(const Tensor& t, int mode, int rank, const sf_launch_t& l);
+bool hot_tile_candidate(const Tensor& t, int mode, int rank, int m);
+// share of the handle's nonzeros whose mode-m index is among the hottest `rows` rows (cached in
+// t.hot_cover[m]; counts in t.hot_cnt[m]) -- how well a hot-row cache would serve mode m
+void hot_coverage(Tensor& t, int m, uint64_t rows);
 // ---- CP-ALS (sf_cpals.cu) ----
 void cpals(Tensor& t, int R, float* const* factors, int iters, double tol, double* fits, int* done,
            cudaStream_t s, Plan* const* plans);

@@ -471,37 +471,12 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
     count_launch();
     SF_CUDA(cudaGetLastError());
   }
-  // (experiment, SF_DEBUG=l2_persist) keep the hot-row block persisting in L2 during the launch
-  // through the stream's access-policy window (restored afterwards)
-  const bool persist = p.hot_total && s != nullptr && debug_opt("l2_persist");
-  cudaStreamAttrValue old_attr{};
-  if (persist) {
-    int dev = 0, maxp = 0, maxw = 0;
-    SF_CUDA(cudaGetDevice(&dev));
-    SF_CUDA(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev));
-    SF_CUDA(cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev));
-    const size_t bytes = std::min<size_t>({p.hot_total * (size_t)R * 4, (size_t)maxp, (size_t)maxw});
-    static size_t limit_set[16] = {};
-    if (dev < 16 && limit_set[dev] < bytes) {
-      SF_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes));
-      limit_set[dev] = bytes;
-    }
-    SF_CUDA(cudaStreamGetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &old_attr));
-    cudaStreamAttrValue a{};
-    a.accessPolicyWindow.base_ptr = p.hot_cache.p;
-    a.accessPolicyWindow.num_bytes = bytes;
-    a.accessPolicyWindow.hitRatio = 1.0f;
-    a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    SF_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &a));
-  }
   switch (R) {
     case 16: frag3_launch_r16(N, S, fp, grid, threads, smem, s); break;
     case 32: frag3_launch_r32(N, S, fp, grid, threads, smem, s); break;
     case 64: frag3_launch_r64(N, S, fp, grid, threads, smem, s); break;
     default: throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: unsupported rank"};
   }
-  if (persist) SF_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &old_attr));
   count_launch();
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) {

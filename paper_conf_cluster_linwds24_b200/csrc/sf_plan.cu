@@ -460,6 +460,73 @@ __global__ void hot_rows_kernel(const uint32_t* __restrict__ cnt, const uint32_t
     if (__ldg(cnt + x) > tau) rows[__ldg(slot + x)] = (uint32_t)x;
 }
 
+// The smallest threshold tau with #{rows of every slot in hc with count > tau} <= budget: 32
+// geometric candidates (0, 1, 3, 7, ...), then 32 linear ones inside the bracketing interval.
+static uint32_t hot_threshold(Tensor& t, HotCount hc, uint64_t budget) {
+  DevBuf above(32 * 8);
+  uint64_t dimmax = 0;
+  for (int q = 0; q < hc.n; ++q) dimmax = std::max(dimmax, hc.dim[q]);
+  auto count_above = [&](unsigned long long* h) {
+    SF_CUDA(cudaMemsetAsync(above.p, 0, 32 * 8, t.stream));
+    hot_above_kernel<<<grid_for(dimmax), 256, 0, t.stream>>>(hc, above.as<unsigned long long>());
+    count_launch();
+    d2h_small(t.stream, h, above.p, 32 * 8);
+  };
+  unsigned long long h[32];
+  for (int j = 0; j < 32; ++j) hc.tau[j] = (j == 31) ? 0xFFFFFFFFu : ((1u << j) - 1u);
+  count_above(h);
+  int j = 0;
+  while (j < 31 && h[j] > budget) ++j;
+  uint32_t tau = hc.tau[j];
+  if (j > 0) {  // refine inside (tau[j-1], tau[j]]
+    const uint64_t lo = (uint64_t)hc.tau[j - 1] + 1, hi = hc.tau[j];
+    for (int i = 0; i < 32; ++i) hc.tau[i] = (uint32_t)std::min<uint64_t>(hi, lo + ((hi - lo) * i + 30) / 31);
+    count_above(h);
+    for (int i = 0; i < 32; ++i)
+      if (h[i] <= budget) { tau = hc.tau[i]; break; }
+  }
+  return tau;
+}
+
+__global__ void hot_sum_kernel(const uint32_t* __restrict__ cnt, uint64_t dim, uint32_t tau,
+                               unsigned long long* __restrict__ sum) {
+  unsigned long long a = 0;
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < dim; x += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = __ldg(cnt + x);
+    if (c > tau) a += c;
+  }
+  for (int o = 16; o; o >>= 1) a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
+  if ((threadIdx.x & 31) == 0 && a) atomicAdd(sum, a);
+}
+
+static void ensure_hot_counts(Tensor& t, int m) {
+  if (t.hot_cnt[m].p) return;
+  t.hot_cnt[m].alloc(t.dims[m] * 4 + 16);
+  SF_CUDA(cudaMemsetAsync(t.hot_cnt[m].p, 0, t.dims[m] * 4, t.stream));
+  if (t.nnz)
+    hot_count_all_kernel<<<grid_for(t.nnz), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), t.nnz,
+                                                               t.hot_cnt[m].as<uint32_t>());
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+void hot_coverage(Tensor& t, int m, uint64_t rows) {
+  if (t.hot_cover[m] >= 0) return;
+  ensure_hot_counts(t, m);
+  HotCount hc{};
+  hc.cnt[0] = t.hot_cnt[m].as<uint32_t>();
+  hc.dim[0] = t.dims[m];
+  hc.n = 1;
+  const uint32_t tau = hot_threshold(t, hc, rows);
+  DevBuf sum(16);
+  SF_CUDA(cudaMemsetAsync(sum.p, 0, 8, t.stream));
+  hot_sum_kernel<<<grid_for(t.dims[m]), 256, 0, t.stream>>>(hc.cnt[0], t.dims[m], tau, sum.as<unsigned long long>());
+  count_launch();
+  unsigned long long v = 0;
+  d2h_small(t.stream, &v, sum.p, 8);
+  t.hot_cover[m] = t.nnz ? (double)v / (double)t.nnz : 0.0;
+}
+
 // frag3 records: kernel-order record k = [raw field fmap[0], ..., fmap[WK-1]] of the raw
 // AoS record perm[k] (fmap < 0: zero padding).  Slot order: i_n, gathered slots, value.
 // Packed (nfields > 0): fields f < nfields (raw word fmap[f]) are OR-ed in at bit boff[f]
@@ -729,14 +796,13 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
         // plan that gathers mode m
         const bool whole = t.nranks == 1;
         DevBuf* cnt = whole ? &t.hot_cnt[m] : &hcnt[q];
-        if (!cnt->p) {
+        if (whole) {
+          ensure_hot_counts(t, m);
+        } else {
           cnt->alloc(t.dims[m] * 4 + 16);
           SF_CUDA(cudaMemsetAsync(cnt->p, 0, t.dims[m] * 4, t.stream));
-          if (whole)
-            hot_count_all_kernel<<<grid_for(n), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), n, cnt->as<uint32_t>());
-          else
-            hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
-                                                                 cnt->as<uint32_t>());
+          hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
+                                                               cnt->as<uint32_t>());
           count_launch();
         }
         hcnt_ptr[q] = cnt->as<uint32_t>();
@@ -749,28 +815,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
         // one global threshold tau (rows with count > tau are hot) so the hot rows of every
         // slot fit the budget: the static cache of the most frequently gathered rows
         const uint64_t budget = (uint64_t)launch.hot_kb * 1024ull / ((uint64_t)rank * 4);
-        DevBuf above(32 * 8);
-        uint64_t dimmax = 0;
-        for (int q = 0; q < hc.n; ++q) dimmax = std::max(dimmax, hc.dim[q]);
-        auto count_above = [&](unsigned long long* h) {
-          SF_CUDA(cudaMemsetAsync(above.p, 0, 32 * 8, t.stream));
-          hot_above_kernel<<<grid_for(dimmax), 256, 0, t.stream>>>(hc, above.as<unsigned long long>());
-          count_launch();
-          d2h_small(t.stream, h, above.p, 32 * 8);
-        };
-        unsigned long long h[32];
-        for (int j = 0; j < 32; ++j) hc.tau[j] = (j == 31) ? 0xFFFFFFFFu : ((1u << j) - 1u);  // 0, 1, 3, 7, ...
-        count_above(h);
-        int j = 0;
-        while (j < 31 && h[j] > budget) ++j;
-        uint32_t tau = hc.tau[j];
-        if (j > 0) {  // refine inside (tau[j-1], tau[j]]
-          const uint64_t lo = (uint64_t)hc.tau[j - 1] + 1, hi = hc.tau[j];
-          for (int i = 0; i < 32; ++i) hc.tau[i] = (uint32_t)std::min<uint64_t>(hi, lo + ((hi - lo) * i + 30) / 31);
-          count_above(h);
-          for (int i = 0; i < 32; ++i)
-            if (h[i] <= budget) { tau = hc.tau[i]; break; }
-        }
+        const uint32_t tau = hot_threshold(t, hc, budget);
         uint64_t total = 0;
         for (int q = 0; q < N - 1; ++q) {
           if (!hot_q[q]) continue;

@@ -342,32 +342,43 @@ static bool l2_refine_enabled() {
 // ---------------------------------------------------------------------------
 static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
 static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 16 * 1024;
-// hot rows + L2 tiles (3-way tensors): tile one gathered factor of 64-512 MB in 64 MB blocks
-// (16 MB blocks below 256 MB) when that gives <= 8 tiles and the Y revisit ratio <= 0.25
+// hot rows + L2 tiles (3-way tensors): tile one gathered factor of 64-512 MB by blocks of 2^19
+// rows (64 MB at R = 32, 32 MB at R = 16; <= 16 tiles, Y revisit ratio <= 0.25) and hot-cache
+// the other.  Of two candidates, tile the one the hot-row cache would serve worse (lower share
+// of nonzeros in its hottest rows, t.hot_cover, measured by the planner): amazon mode 0 tiles
+// mode 1 (Zipf 0.8) and caches mode 2 (Zipf 1.0), 0.81x vs 0.94x the hot-only time.
 static constexpr double kHotTileMinBytes = 64.0 * 1024 * 1024, kHotTileMaxBytes = 512.0 * 1024 * 1024;
-static constexpr double kHotTileMaxTiles = 8, kHotTileMaxRevisit = 0.25;
+static constexpr double kHotTileMaxTiles = 16, kHotTileMaxRevisit = 0.25;
+static constexpr uint32_t kHotTileRows = 1u << 19;
+
+bool hot_tile_candidate(const Tensor& t, int mode, int rank, int m) {
+  if (t.nmodes != 3 || m == mode) return false;
+  const double F = (double)t.dims[m] * rank * 4.0;
+  return F >= kHotTileMinBytes && F <= kHotTileMaxBytes &&
+         std::ceil((double)t.dims[m] / kHotTileRows) <= kHotTileMaxTiles;
+}
 
 static void hot_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, sf_launch_t& l) {
   if (l.hot_kb == 0 || l.staged_mask != 0 || t.nmodes != 3 || f.nnz == 0) return;
   const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
   int best = -1;
-  double bestF = 0, bestBlock = 0;
+  double bestF = 0, bestCover = 2.0;
   for (int m = 0; m < t.nmodes; ++m) {
-    if (m == mode) continue;
+    if (!hot_tile_candidate(t, mode, rank, m)) continue;
     const double F = (double)t.dims[m] * RB;
-    if (F < kHotTileMinBytes || F > kHotTileMaxBytes || F <= bestF) continue;
-    const double block = F >= 256.0 * 1024 * 1024 ? 64.0 * 1024 * 1024 : 16.0 * 1024 * 1024;
-    const double T = std::ceil(F / block);
-    if (T > kHotTileMaxTiles) continue;
+    const double T = std::ceil((double)t.dims[m] / kHotTileRows);
     if ((Yb > kL2YInCache ? revisit_ratio(f, T) : 0.0) > kHotTileMaxRevisit) continue;
-    best = m;
-    bestF = F;
-    bestBlock = block;
+    const double cover = t.hot_cover[m] >= 0 ? t.hot_cover[m] : 1.0;
+    if (cover < bestCover - 1e-3 || (std::fabs(cover - bestCover) <= 1e-3 && F > bestF)) {
+      best = m;
+      bestF = F;
+      bestCover = cover;
+    }
   }
   if (best < 0) return;
   sf_launch_t c = l;
   c.staged_mask = 1u << best;
-  c.block_rows[best] = (uint32_t)std::max(1.0, bestBlock / RB);
+  c.block_rows[best] = kHotTileRows;
   c.flags = (c.flags | SF_LAUNCH_L2_TILES) & ~SF_LAUNCH_NO_OWNER_STORES;
   c.hot_kb = kHotKBTiled;
   c.chunk_nnz = 128;

@@ -23,8 +23,6 @@ def main():
     ap.add_argument("--budgets", default="0,16,32,64,128,256")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--modes", default=None)
-    ap.add_argument("--persist", action="store_true",
-                    help="also time every variant with the hot block persisting in L2 (SF_DEBUG=l2_persist)")
     ap.add_argument("--no-tiles-variant", action="store_true", help="only the selector's tiling choice")
     args = ap.parse_args()
     import torch
@@ -60,11 +58,7 @@ def main():
                                    flags=flags, hot_kb=hb * 1024)
                 T.set_launch(n, R, L)
                 info = T.plan_info(n, R)
-                for persist in ([False, True] if args.persist else [False]):
-                    if persist:
-                        os.environ["SF_DEBUG"] = "l2_persist"
-                    else:
-                        os.environ.pop("SF_DEBUG", None)
+                for persist in [False]:
                     for _ in range(3):
                         T.mttkrp(n, facs, out, stream=s)
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -75,9 +69,8 @@ def main():
                     torch.cuda.synchronize()
                     ms = e0.elapsed_time(e1) / args.reps
                     print(json.dumps({"config": name, "mode": n, "l2tiles": bool(flags & sf.LAUNCH_L2_TILES),
-                                      "hot_mb": hb, "persist": persist, "ms": round(ms, 4),
+                                      "hot_mb": hb, "ms": round(ms, 4),
                                       "plan_ms": round(info["plan_ms"], 2), "selector": base}), flush=True)
-                os.environ.pop("SF_DEBUG", None)
             T.plan_release(n, R)
             del out
             torch.cuda.empty_cache()
