@@ -28,6 +28,10 @@
  *     `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
  *   - Asynchronous kernel faults surface at the caller's next synchronization
  *     (as in cuBLAS); the library itself synchronizes only where stated.
+ *   - Arithmetic: fp32 products and sums; the vector reductions at run boundaries
+ *     (red.global.add.v4.f32) flush subnormal results to zero, so a row whose |.|-scale
+ *     S = sum |v * prod A| is itself subnormal (< 1.2e-38) may come back as 0 -- such
+ *     inputs are outside the 1e-4 relative contract (reading R8).
  *   - Environment: the library reads nothing but SF_DEBUG, a debug / A-B aid that is never
  *     needed in production: a comma-separated list of trace (sf_plan phase marks on
  *     stderr), no_presort, no_l2tiles, no_hot, no_cpals_fused (disable one optimisation)
