@@ -30,6 +30,10 @@
 
 #include "sf_frag.cuh"
 
+#ifndef SF_FRAG_U_WIDE
+#define SF_FRAG_U_WIDE 2  // U for N >= 4 at R >= 32 (A/B builds: -DSF_FRAG_U_WIDE=1)
+#endif
+
 namespace sf {
 
 // First position of group gam (of Gam) inside the tile segment [a, a + len).
@@ -119,7 +123,8 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   static_assert(!PK || N >= 4, "packed records are for N >= 4");
   constexpr int RB = R * 4;     // bytes per factor row
   constexpr int R4 = R / 4;     // float4 per factor row
-  constexpr int U = (VEC == 8) ? 2 : kFragUnroll;  // batch (register budget: 64 at 1024 thr)
+  // batch of nonzeros in flight per lane group (register budget: 64 at 1024 threads)
+  constexpr int U = (VEC == 8) ? (N >= 4 ? SF_FRAG_U_WIDE : 2) : kFragUnroll;
   extern __shared__ __align__(128) unsigned char smem_raw[];
 
   const int tid = threadIdx.x;
