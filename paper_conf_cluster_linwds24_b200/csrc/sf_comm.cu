@@ -21,6 +21,9 @@
 
 #include <algorithm>
 #include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -79,9 +82,34 @@ static void nccl_check(ncclResult_t r, const char* what) {
   }
 }
 
-Comm::~Comm() {
-  if (nccl && sf::nccl().ok) sf::nccl().CommDestroy(static_cast<ncclComm_t>(nccl));
+// NCCL communicators are shared by every handle attached with the same (unique id, nranks,
+// rank, device): ncclCommInitRank is a collective costing tens to hundreds of ms, and a user
+// (or bench.py's e2e leg) creates a handle per tensor.  Destroyed with the last handle.
+struct NcclHandle {
+  ncclComm_t comm = nullptr;
+  ~NcclHandle() {
+    if (comm && sf::nccl().ok) sf::nccl().CommDestroy(comm);
+  }
+};
+
+static std::mutex g_comm_mu;
+static std::map<std::string, std::weak_ptr<NcclHandle>> g_comms;
+
+static std::shared_ptr<NcclHandle> nccl_comm_for(const void* id128, int nranks, int rank, int device) {
+  std::string key(static_cast<const char*>(id128), 128);
+  key += ":" + std::to_string(nranks) + ":" + std::to_string(rank) + ":" + std::to_string(device);
+  std::lock_guard<std::mutex> g(g_comm_mu);
+  if (auto h = g_comms[key].lock()) return h;
+  NcclApi& api = sf::nccl();
+  ncclUniqueId id;
+  memcpy(&id, id128, sizeof id);
+  auto h = std::make_shared<NcclHandle>();
+  nccl_check(api.CommInitRank(&h->comm, nranks, id, rank), "ncclCommInitRank");
+  g_comms[key] = h;
+  return h;
 }
+
+Comm::~Comm() = default;
 
 void Comm::allgatherv(const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs, cudaStream_t s) {
   if (fn) {
@@ -295,20 +323,15 @@ sf_status sf_comm_attach(sf_tensor_t h, int nranks, int rank, const void* id128)
     NcclApi& api = nccl();
     if (!api.ok) throw StatusError{SF_ERR_NCCL, api.err};
     SF_CUDA(cudaSetDevice(t->device));
-    ncclUniqueId id;
-    memcpy(&id, id128, sizeof id);
-    ncclComm_t c = nullptr;
-    nccl_check(api.CommInitRank(&c, nranks, id, rank), "ncclCommInitRank");
+    std::shared_ptr<NcclHandle> c = nccl_comm_for(id128, nranks, rank, t->device);
     const sf_status st = sf_set_shard(h, nranks, rank);
-    if (st != SF_OK) {
-      api.CommDestroy(c);
-      return st;
-    }
+    if (st != SF_OK) return st;
     delete t->comm;
     t->comm = new Comm();
     t->comm->nranks = nranks;
     t->comm->rank = rank;
-    t->comm->nccl = c;
+    t->comm->shared = c;
+    t->comm->nccl = c->comm;
     return SF_OK;
   });
 }

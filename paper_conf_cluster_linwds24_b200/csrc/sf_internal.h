@@ -6,6 +6,7 @@
 
 #include <atomic>
 #include <map>
+#include <memory>
 #include <string>
 #include <utility>
 #include <vector>
@@ -114,9 +115,11 @@ struct Plan {
 // Collective transport of a sharded handle (sf_comm.cu): NCCL (sf_comm_attach) or a caller
 // callback (sf_comm_attach_transport).  allgatherv: rank k contributes bytes[k] bytes from
 // `send`; every rank receives them at recv + displs[k] (device memory, stream-ordered).
+struct NcclHandle;  // a shared NCCL communicator (sf_comm.cu; one per (unique id, rank, device))
 struct Comm {
   int nranks = 1, rank = 0;
-  void* nccl = nullptr;  // ncclComm_t
+  void* nccl = nullptr;  // ncclComm_t (owned by `shared`)
+  std::shared_ptr<NcclHandle> shared;
   sf_allgatherv_fn fn = nullptr;
   void* ctx = nullptr;
   void allgatherv(const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs, cudaStream_t s);

@@ -87,15 +87,23 @@ class TorchAllgatherv:
             return 1
 
 
+_NCCL_IDS = {}
+
+
 def attach(T, world, rank, group=None, nccl=None):
     """Shard handle T as rank `rank` of `world` and attach the exchange transport:
     NCCL when the default process group is NCCL (or nccl=True), else TorchAllgatherv."""
     if nccl is None:
         nccl = dist.get_backend(group) == "nccl"
     if nccl:
-        obj = [comm_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0, group=group)
-        T.comm_attach(world, rank, obj[0])
+        # one NCCL unique id per process group: the library shares the communicator between
+        # every handle attached with it (ncclCommInitRank runs once)
+        key = id(group)
+        if key not in _NCCL_IDS:
+            obj = [comm_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0, group=group)
+            _NCCL_IDS[key] = obj[0]
+        T.comm_attach(world, rank, _NCCL_IDS[key])
         return None
     tr = TorchAllgatherv(group)
     T.comm_attach_transport(world, rank, tr.cfn)
