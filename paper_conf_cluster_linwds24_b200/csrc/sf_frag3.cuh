@@ -31,7 +31,7 @@
 #include "sf_frag.cuh"
 
 #ifndef SF_FRAG_U_WIDE
-#define SF_FRAG_U_WIDE 2  // U for N >= 4 at R >= 32 (A/B builds: -DSF_FRAG_U_WIDE=1)
+#define SF_FRAG_U_WIDE 1  // U for N >= 4 at R >= 32: 1 avoids spills (deli-4d +3 %; A/B: -DSF_FRAG_U_WIDE=2)
 #endif
 
 namespace sf {
