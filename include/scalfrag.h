@@ -175,7 +175,8 @@ sf_status sf_shard_rows(sf_tensor_t t, int mode, int rank, uint64_t* row_begin, 
  *   sf_comm_unique_id: rank 0 creates a 128-byte NCCL id (broadcast it, e.g. by torch).
  *   sf_comm_attach:    ncclCommInitRank on this handle's device + sf_set_shard(nranks, rank);
  *                      handles attached with the same (id, nranks, rank, device) share one
- *                      communicator (created once, destroyed with the last such handle).
+ *                      communicator, created once and kept until the process exits (a
+ *                      unique id can initialise only one communicator).
  *   sf_comm_attach_transport: the same exchange over the caller's allgatherv (tests, or a
  *                      non-NCCL fabric); fn returns 0 on success.
  * NCCL is loaded at run time (dlopen libnccl.so.2); SF_ERR_NCCL on any collective error. */

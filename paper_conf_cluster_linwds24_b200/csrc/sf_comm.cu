@@ -84,7 +84,9 @@ static void nccl_check(ncclResult_t r, const char* what) {
 
 // NCCL communicators are shared by every handle attached with the same (unique id, nranks,
 // rank, device): ncclCommInitRank is a collective costing tens to hundreds of ms, and a user
-// (or bench.py's e2e leg) creates a handle per tensor.  Destroyed with the last handle.
+// (or bench.py's e2e leg) creates a handle per tensor.  They live until the process exits: a
+// unique id may initialise a communicator only once, so re-attaching with the same id after
+// the last handle is gone must find the communicator again, not re-initialise it.
 struct NcclHandle {
   ncclComm_t comm = nullptr;
   ~NcclHandle() {
@@ -93,19 +95,21 @@ struct NcclHandle {
 };
 
 static std::mutex g_comm_mu;
-static std::map<std::string, std::weak_ptr<NcclHandle>> g_comms;
+static std::map<std::string, std::shared_ptr<NcclHandle>>* g_comms =
+    new std::map<std::string, std::shared_ptr<NcclHandle>>();  // never destroyed (see above)
 
 static std::shared_ptr<NcclHandle> nccl_comm_for(const void* id128, int nranks, int rank, int device) {
   std::string key(static_cast<const char*>(id128), 128);
   key += ":" + std::to_string(nranks) + ":" + std::to_string(rank) + ":" + std::to_string(device);
   std::lock_guard<std::mutex> g(g_comm_mu);
-  if (auto h = g_comms[key].lock()) return h;
+  auto it = g_comms->find(key);
+  if (it != g_comms->end()) return it->second;
   NcclApi& api = sf::nccl();
   ncclUniqueId id;
   memcpy(&id, id128, sizeof id);
   auto h = std::make_shared<NcclHandle>();
   nccl_check(api.CommInitRank(&h->comm, nranks, id, rank), "ncclCommInitRank");
-  g_comms[key] = h;
+  (*g_comms)[key] = h;
   return h;
 }
 
