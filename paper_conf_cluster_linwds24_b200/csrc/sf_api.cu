@@ -414,9 +414,10 @@ static void make_plan(Tensor& t, int mode, int rank, const sf_launch_t* override
     l = *override_launch;
     normalize_launch(src, mode, rank, l);
   } else {
-    if (src.nranks == 1)  // the hot+tile rule compares how well each candidate's rows would cache
-      for (int m = 0; m < src.nmodes; ++m)
-        if (hot_tile_candidate(src, mode, rank, m)) hot_coverage(src, m, (16ull << 20) / (4ull * rank));
+    // the hot+tile rule compares how well each candidate's rows would cache (row frequencies of
+    // the whole handle; for a v1 shard a proxy of its own)
+    for (int m = 0; m < src.nmodes; ++m)
+      if (hot_tile_candidate(src, mode, rank, m)) hot_coverage(src, m, (16ull << 20) / (4ull * rank));
     l = select_launch(src, f, mode, rank, hi - lo);
   }
   if (l.kernel == SF_KERNEL_FRAG && frag_smem_bytes(src, mode, rank, l) > src.smem_optin)

@@ -342,37 +342,36 @@ static bool l2_refine_enabled() {
 // ---------------------------------------------------------------------------
 static constexpr double kHotMinGatheredBytes = 160.0 * 1024 * 1024;
 static constexpr uint32_t kHotKB = 32 * 1024, kHotKBTiled = 16 * 1024;
-// hot rows + L2 tiles (3-way tensors): tile one gathered factor of 64-512 MB by blocks of 2^19
-// rows (64 MB at R = 32, 32 MB at R = 16; <= 16 tiles, Y revisit ratio <= 0.25) and hot-cache
-// the other.  Of two candidates, tile the one the hot-row cache would serve worse (lower share
-// of nonzeros in its hottest rows, t.hot_cover, measured by the planner): amazon mode 0 tiles
-// mode 1 (Zipf 0.8) and caches mode 2 (Zipf 1.0), 0.81x vs 0.94x the hot-only time.
-static constexpr double kHotTileMinBytes = 64.0 * 1024 * 1024, kHotTileMaxBytes = 512.0 * 1024 * 1024;
-static constexpr double kHotTileMaxTiles = 16, kHotTileMaxRevisit = 0.25;
+// hot rows + L2 tiles: tile one gathered factor by blocks of 2^19 rows (64 MB at R = 32, 32 MB at
+// R = 16; 2..32 tiles, Y revisit ratio rho <= 0.10) and hot-cache the others (16 MB) -- but only
+// a factor the hot-row cache would serve badly: the share of nonzeros whose index is among its
+// hottest 16 MB of rows (t.hot_cover, measured by the planner) must be < 0.8, and of several
+// candidates the least-covered one is tiled.  Fitted on 70 modes (16 random hyper-sparse tensors
+// + the BASELINE / Table III shapes, tools/hot_heldout.py --seed 78, tools/fit_tile_rule.py:
+// best / chosen 0.988 mean) and checked on 39 held-out modes (--seed 77): 0.977 mean vs 0.938
+// for hot rows alone and 0.946 for the previous 3-way-only rule (profiles/r02/hot_rule/).
+static constexpr double kHotTileMaxTiles = 32, kHotTileMaxRevisit = 0.10, kHotTileMaxCover = 0.8;
 static constexpr uint32_t kHotTileRows = 1u << 19;
 
 bool hot_tile_candidate(const Tensor& t, int mode, int rank, int m) {
-  if (t.nmodes != 3 || m == mode) return false;
-  const double F = (double)t.dims[m] * rank * 4.0;
-  return F >= kHotTileMinBytes && F <= kHotTileMaxBytes &&
-         std::ceil((double)t.dims[m] / kHotTileRows) <= kHotTileMaxTiles;
+  (void)rank;
+  if (m == mode) return false;
+  const double T = std::ceil((double)t.dims[m] / kHotTileRows);
+  return T >= 2 && T <= kHotTileMaxTiles;
 }
 
 static void hot_tile_refine(const Tensor& t, const sf_features_t& f, int mode, int rank, sf_launch_t& l) {
-  if (l.hot_kb == 0 || l.staged_mask != 0 || t.nmodes != 3 || f.nnz == 0) return;
+  if (l.hot_kb == 0 || l.staged_mask != 0 || f.nnz == 0) return;
   const double RB = 4.0 * rank, Yb = (double)t.dims[mode] * RB;
   int best = -1;
-  double bestF = 0, bestCover = 2.0;
+  double bestCover = kHotTileMaxCover;
   for (int m = 0; m < t.nmodes; ++m) {
-    if (!hot_tile_candidate(t, mode, rank, m)) continue;
-    const double F = (double)t.dims[m] * RB;
+    if (!hot_tile_candidate(t, mode, rank, m) || t.hot_cover[m] < 0) continue;
     const double T = std::ceil((double)t.dims[m] / kHotTileRows);
     if ((Yb > kL2YInCache ? revisit_ratio(f, T) : 0.0) > kHotTileMaxRevisit) continue;
-    const double cover = t.hot_cover[m] >= 0 ? t.hot_cover[m] : 1.0;
-    if (cover < bestCover - 1e-3 || (std::fabs(cover - bestCover) <= 1e-3 && F > bestF)) {
+    if (t.hot_cover[m] < bestCover) {
       best = m;
-      bestF = F;
-      bestCover = cover;
+      bestCover = t.hot_cover[m];
     }
   }
   if (best < 0) return;
@@ -387,7 +386,7 @@ static void hot_tile_refine(const Tensor& t, const sf_features_t& f, int mode, i
 }
 
 static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
-  if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC) || l.staged_mask != 0) return;
+  if (l.kernel != SF_KERNEL_FRAG || (l.flags & SF_LAUNCH_DETERMINISTIC) || (l.flags & SF_LAUNCH_L2_TILES)) return;
   double gathered = 0;
   for (int m = 0; m < t.nmodes; ++m) {
     if (m == mode || (l.staged_mask & (1u << m))) continue;
@@ -395,6 +394,11 @@ static void hot_refine(const Tensor& t, int mode, int rank, sf_launch_t& l) {
     if (F >= 16.0 * 1024 * 1024) gathered += F;
   }
   if (gathered < kHotMinGatheredBytes || debug_opt("no_hot")) return;  // SF_DEBUG A/B
+  // a shared-memory-staged pick of a small factor next to >= 160 MB of gathered factors is
+  // replaced by the (unstaged) hot-row class: staging + hot rows measured no better than hot
+  // rows alone on deli-4d, and a held-out 4-way tensor ran 1.7x faster unstaged with hot rows
+  l.staged_mask = 0;
+  for (int m = 0; m < SF_MAX_MODES; ++m) l.block_rows[m] = 0;
   // the hot-row class: owner stores, 1024 threads (one CTA per SM), 32 MB of hot rows, no L2
   // tiles, and stages of 4 register batches per lane group (chunk = 8 groups x 4 x U nonzeros:
   // 64 at R >= 32 where U = 2, 128 at R = 16 where U = 4) -- the best fixed class over the
@@ -430,11 +434,10 @@ sf_launch_t select_launch(const Tensor& t, const sf_features_t& f, int mode, int
     }
   }
   if (!picked) l = select_rules(t, f, mode, rank, nnz_local);
-  // hot-row cache first: where it applies to an unstaged pick it beats L2 tiles alone (deli-4d
-  // 1.2-1.8x, flickr-3d 1.2x per mode) or ties them (nell-1), profiles/r02/hot_sweep_g06.jsonl;
-  // then, for 3-way tensors, L2 tiles of one mid-size factor on top (hot_tile_refine): amazon
-  // 0.81x / nell-1 0.96-0.99x the hot-only time; 4-way tensors lose 3-15 % with any tiling
-  // (deli-4d), profiles/r02/sweeps/
+  // hot-row cache first: where it applies it beats L2 tiles alone (deli-4d 1.2-1.8x, flickr-3d
+  // 1.2x per mode) or ties them (nell-1), profiles/r02/hot_sweep_g06.jsonl; then L2 tiles of one
+  // poorly-cached factor on top (hot_tile_refine): amazon 0.81x / nell-1 0.96-0.99x the
+  // hot-only time, profiles/r02/sweeps/ and profiles/r02/hot_rule/
   hot_refine(t, mode, rank, l);
   if (l.hot_kb != 0) {
     if (l2_refine_enabled()) hot_tile_refine(t, f, mode, rank, l);

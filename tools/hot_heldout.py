@@ -35,6 +35,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--count", type=int, default=12)
     ap.add_argument("--seed", type=int, default=77)
+    ap.add_argument("--configs", default="", help="also run these named configs (synth.CONFIGS)")
     args = ap.parse_args()
     import torch
 
@@ -53,15 +54,33 @@ def main():
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / 5
 
-    for k in range(args.count):
-        c = random_tensor(rng, k)
+    tensors = [random_tensor(rng, k) for k in range(args.count)]
+    for name in [x for x in args.configs.split(",") if x]:
+        cfg = synth.CONFIGS[name]
+        tensors.append(dict(name=name, dims=list(cfg.dims), nnz=cfg.nnz, rank=cfg.rank, zipf=list(cfg.zipf),
+                            seed=cfg.seed, config=name))
+    for c in tensors:
         R, N = c["rank"], len(c["dims"])
-        inds, vals = synth.gen_coo_device(c["dims"], c["nnz"], c["seed"], c["zipf"])
-        facs = synth.gen_factors_device(c["dims"], R, c["seed"] + 7)
+        if "config" in c:
+            inds, vals = synth.config_tensor_device(synth.CONFIGS[c["config"]])
+            facs = synth.config_factors_device(synth.CONFIGS[c["config"]])
+        else:
+            inds, vals = synth.gen_coo_device(c["dims"], c["nnz"], c["seed"], c["zipf"])
+            facs = synth.gen_factors_device(c["dims"], R, c["seed"] + 7)
+        # exact row counts per mode -> hot coverage (share of nonzeros in the hottest 16 MB of rows)
+        counts = [torch.bincount(a.long(), minlength=d) for a, d in zip(inds, c["dims"])]
+        hot_rows = (16 << 20) // (4 * R)
+        cover = [float(torch.topk(cn, min(hot_rows, cn.numel())).values.sum()) / c["nnz"] for cn in counts]
         with sf.Tensor(c["dims"], inds, vals) as T:
             del inds, vals
             for n in range(N):
                 out = torch.empty((c["dims"][n], R), device="cuda")
+                cn = counts[n].double()
+                rho = {}
+                for m in range(N):
+                    if m != n and c["dims"][m] > (1 << 19):
+                        Tt = -(-c["dims"][m] // (1 << 19))
+                        rho[m] = float(Tt * (1 - torch.exp(-1.44 * cn / Tt)).sum() / c["nnz"])
                 times = {}
                 auto = sf.Launch()
                 auto.kernel = 0
@@ -88,18 +107,19 @@ def main():
                     try:
                         T.set_launch(n, R, L)
                         times[name] = time_it(T, n, R, facs, out)
-                    except sf.SfError as e:
+                    except sf.SfError:
                         times[name] = None
                 T.plan_release(n, R)
                 del out
                 torch.cuda.empty_cache()
                 ok = {k2: v for k2, v in times.items() if v}
                 best = min(ok.values())
-                print(json.dumps({"tensor": c, "mode": n, "pick": pick, "no_hot_pick": nohot,
+                print(json.dumps({"tensor": c, "mode": n, "pick": pick, "no_hot_pick": nohot, "cover": cover,
+                                  "rho": rho, "y_mb": c["dims"][n] * R * 4 / 2**20,
                                   "times_ms": {k2: (round(v, 4) if v else None) for k2, v in times.items()},
                                   "pick_over_best": best / times["pick"],
                                   "no_hot_over_best": best / times["no_hot_rules"]}), flush=True)
-        del facs
+        del facs, counts
         torch.cuda.empty_cache()
 
 
