@@ -19,6 +19,7 @@
 
 #include <algorithm>
 #include <cub/cub.cuh>
+#include <thrust/iterator/counting_iterator.h>
 #include <vector>
 
 #include "sf_internal.h"
@@ -175,7 +176,7 @@ void dist_build_sub(Tensor& t, int mode) {
       dist_flag_kernel<<<grid_of(n), 256, 0, s>>>(t.ind[mode].as<uint32_t>(), n, gstart.as<uint32_t>(),
                                                   gcnt.as<uint32_t>(), cuts, q, flag.as<uint8_t>());
       size_t tb = 0;
-      cub::CountingInputIterator<uint32_t> it(0);
+      thrust::counting_iterator<uint32_t> it(0);
       SF_CUDA(cub::DeviceSelect::Flagged(nullptr, tb, it, flag.as<uint8_t>(), sel[q].as<uint32_t>(),
                                          nsel.as<uint64_t>(), (int64_t)n, s));
       DevBuf tmp(tb + 16);

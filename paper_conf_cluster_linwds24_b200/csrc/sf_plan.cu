@@ -764,7 +764,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
     rp.fmap[N] = N;  // value word of the raw record
     rp.nfields = 0;
     // hot-row cache: eligible gathered slots are gathered from L2/HBM (not staged in shared
-    // memory, not the L2-tiled mode) and large enough for their rows to be scattered
+    // memory, not the L2-tiled mode; the selector decides whether the plan uses the cache)
     bool hot_q[SF_MAX_MODES] = {};
     std::vector<DevBuf> hcnt(SF_MAX_MODES), hslot(SF_MAX_MODES);
     const uint32_t* hcnt_ptr[SF_MAX_MODES] = {};
