@@ -20,7 +20,7 @@ Contract (one JSON line on rank 0):
   reading R14), max over ranks, CUDA events on the launching stream.
 * e2e: the same metric through the public C ABI from PINNED HOST buffers:
   sf_tensor_create (segmented H2D + validate) + factor H2D + sf_plan (all modes)
-  + sf_mttkrp (all modes) + D2H of every Y, every step.
+  + sf_mttkrp (all modes) + D2H of every Y, every step; the median of --e2e-steps steps.
 * roofline: dominant kernel = frag3_kernel; algorithmic bytes per launch =
   4(N+1)*nnz + 4R*sum_m I_m (SURVEY §8(d) D-3), over its event-timed duration;
   traffic = ncu dram bytes per launch of that config (profiles/ncu_traffic.json).
@@ -235,7 +235,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-trace", action="store_true", help="host time after every call of each e2e step (stderr)")
     ap.add_argument("--cpu-sample", type=int, default=30_000_000)
     ap.add_argument("--ref-sample", type=int, default=1_000_000)
     ap.add_argument("--one-plan", action="store_true", help="plan/time/release one mode at a time")
@@ -452,8 +453,15 @@ def main():
         d2h_s = torch.cuda.Stream(device=dev)
 
         def e2e_step():
+            t_0, marks = time.perf_counter(), []
+
+            def mark(what):
+                if args.e2e_trace:
+                    marks.append((what, round((time.perf_counter() - t_0) * 1e3, 2)))
+
             with (sf.Tensor(cfg.dims, h_inds, h_vals) if world == 1 else
                   sf.Tensor.create_dist(cfg.dims, cfg.nnz, lo, h_inds, h_vals)) as T2:
+                mark("create")
                 if world > 1:
                     sfdist.attach(T2, world, rank)
                 ev_f = {}
@@ -464,6 +472,7 @@ def main():
                         ev_f[m].record(h2d_s)
                 for n in order:
                     plan_mode(T2, n)
+                    mark(f"plan {n}")
                     inf = T2.plan_info(n, R)
                     with torch.cuda.stream(stream):
                         o = torch.empty((inf["out_rows"], R), dtype=torch.float32, device=dev)
@@ -479,16 +488,23 @@ def main():
                         d2h_s.synchronize()
                         T2.plan_release(n, R)
                 torch.cuda.synchronize(dev)
+                mark("synced")
+            mark("closed")
+            if args.e2e_trace:
+                print(json.dumps({"e2e_step_marks_ms": marks}), file=sys.stderr, flush=True)
 
         e2e_step()  # warm-up
-        barrier_sync()
-        s0 = time.perf_counter()
+        step_ms = []
         for _ in range(args.e2e_steps):
+            barrier_sync()
+            s0 = time.perf_counter()
             e2e_step()
-        torch.cuda.synchronize(dev)
-        e2e_ms = (time.perf_counter() - s0) / args.e2e_steps * 1e3
-        if world > 1:
-            e2e_ms = max_over_ranks(e2e_ms)
+            torch.cuda.synchronize(dev)
+            ms = (time.perf_counter() - s0) * 1e3
+            step_ms.append(max_over_ranks(ms) if world > 1 else ms)
+        # the median step: on a fresh box single steps' sf_tensor_create (the pinned upload) ran
+        # up to 3x slower, not reproducibly (profiles/r02/e2e_variance/)
+        e2e_ms = statistics.median(step_ms)
         # the PCIe floor of this step: its H2D bytes at the measured pinned H2D bandwidth
         hb = torch.empty(1 << 28, dtype=torch.float32).pin_memory()
         db = torch.empty_like(hb, device=dev)
@@ -504,7 +520,7 @@ def main():
         e2e = {"value": flops_step / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "ms_per_step": e2e_ms,
                "h2d_gbs": h2d_gbs, "h2d_floor_ms": floor_ms, "over_h2d_floor": e2e_ms / floor_ms,
-               "steps": args.e2e_steps,
+               "steps": args.e2e_steps, "step_ms": [round(x, 2) for x in step_ms], "stat": "median over steps",
                "includes": "sf_tensor_create(pinned host COO, segmented H2D+validate) + factor H2D + "
                            "sf_plan x N + sf_mttkrp x N + D2H of every Y (host wall clock); factor H2D "
                            "overlapped with sf_plan, each Y's D2H with the later modes"}

@@ -330,6 +330,7 @@ static void upload(Tensor& t, const uint32_t* const* inds, const float* vals, in
     ptemp_bytes = presort_temp_bytes(t, seg_len);
     for (auto& b : ptemp) b.alloc(ptemp_bytes + 16);
   }
+  const Ingest ingest = ingest_begin(t);
   try {
     if (pageable) {
       for (int s = 0; s < nstreams; ++s) {
@@ -363,6 +364,7 @@ static void upload(Tensor& t, const uint32_t* const* inds, const float* vals, in
       }
       validate_indices(N, t.dims, len, dseg, d_flag, st[s]);
       if (presort) presort_segment(t, a, len, st[s], ptemp[s].p, ptemp_bytes);
+      ingest_segment(t, ingest, a, len, st[s]);
     }
     for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
     t.pre_alt.release();

@@ -245,6 +245,15 @@ void d2d_copy(void* dst, const void* src, size_t bytes, cudaStream_t s);
 bool presort_begin(Tensor& t, uint64_t seg_len);
 void presort_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t s, void* temp, size_t temp_bytes);
 size_t presort_temp_bytes(const Tensor& t, uint64_t seg_len);
+// Raw-COO work every plan needs, done per segment behind its upload (A8): the AoS record copy
+// (unless the presort builds it) and the whole-handle row counts of modes with >= 2^18 rows
+// (the hot-row cache's input).  Skipped when device memory is short (then built at plan time).
+struct Ingest {
+  bool aos = false;
+  uint32_t cnt_mask = 0;
+};
+Ingest ingest_begin(Tensor& t);
+void ingest_segment(Tensor& t, const Ingest& g, uint64_t a, uint64_t len, cudaStream_t s);
 // keys/pos (optional): receive the matricized order (sorted keys, input positions) when
 // this call had to sort, so build_plan can reuse it instead of sorting again.
 void compute_features(Tensor& t, int mode, sf_features_t* out, DevBuf* keys, DevBuf* pos);

@@ -17,14 +17,13 @@
 #include <cub/cub.cuh>
 
 #include <cub/device/device_merge.cuh>
-#include <thrust/iterator/discard_iterator.h>
-#include <thrust/iterator/transform_iterator.h>
 
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
 #include "sf_internal.h"
+
 
 namespace sf {
 
@@ -37,6 +36,21 @@ static inline int bitlen(uint64_t x) {
 static inline int grid_for(uint64_t n, int threads = 256) {
   return (int)std::max<uint64_t>(1, std::min<uint64_t>((n + threads - 1) / threads, 148ull * 32));
 }
+
+// x / d for a divisor fixed per launch (d < 2^32): the quotient estimate hi64(x * m),
+// m = floor((2^64 - 1) / d), is at most 2 below floor(x / d); two corrections make it exact.
+// (A 64-bit `/` compiles to a ~70-instruction software routine.)
+struct Div64 {
+  uint64_t d, m;
+  explicit Div64(uint64_t d_) : d(d_), m(~0ull / d_) {}
+  __device__ __forceinline__ uint64_t div(uint64_t x) const {
+    uint64_t q = __umul64hi(x, m);
+    uint64_t r = x - q * d;
+    if (r >= d) { ++q; r -= d; }
+    if (r >= d) ++q;
+    return q;
+  }
+};
 
 // ---------------------------------------------------------------------------
 __global__ void key_matricized_kernel(const uint32_t* __restrict__ in, const uint32_t* __restrict__ is,
@@ -88,6 +102,9 @@ bool presort_begin(Tensor& t, uint64_t seg_len) {
   const uint64_t n = t.nnz;
   if (n < 2 || seg_len >= n || n >= (1ull << 30)) return false;
   const int pb = std::max(1, bitlen(n - 1));
+  // Modes whose key and position need more than 64 bits are not presorted: (key, position)
+  // pair runs merged with a pair comparison were measured slower end to end on nell-1 (the
+  // per-segment pair sorts lengthen the upload more than the merge saves)
   int modes = 0;
   for (int m = 0; m < t.nmodes; ++m) modes += (key_bits(t, m) + pb <= 64);
   if (!modes) return false;
@@ -131,6 +148,92 @@ void presort_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t st, void*
                                            t.pre_pb + key_bits(t, m), st));
     count_launch(1 + (uint64_t)((key_bits(t, m) + 7) / 8) * 3);
   }
+  SF_CUDA(cudaGetLastError());
+}
+
+// cnt[x] += #{k < n : ind[perm ? perm[k] : k] == x}, indices >= dim skipped (not yet validated
+// during the upload).  Up to kSmemCountRows rows: a per-block shared-memory histogram flushed
+// once per block; more: warp-aggregated atomics (the lanes holding the same row add once), as
+// skewed (Zipf) rows would otherwise serialise on a few addresses.
+constexpr uint64_t kSmemCountRows = 12288;
+__global__ void row_count_kernel(const uint32_t* __restrict__ ind, const uint32_t* __restrict__ perm, uint64_t n,
+                                 uint64_t dim, uint32_t* __restrict__ cnt) {
+  extern __shared__ uint32_t hist[];
+  const bool small = dim <= kSmemCountRows;
+  if (small) {
+    for (uint64_t i = threadIdx.x; i < dim; i += blockDim.x) hist[i] = 0;
+    __syncthreads();
+  }
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  if (small) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+      const uint32_t x = __ldg(ind + (perm ? __ldg(perm + k) : k));
+      if (x < dim) atomicAdd(hist + x, 1u);
+    }
+  } else {
+    // warp-uniform trip count, so every lane takes part in the match
+    const uint64_t k0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+    for (uint64_t kw = k0; kw < n; kw += stride) {
+      const uint64_t k = kw + (threadIdx.x & 31u);
+      const uint32_t x = (k < n) ? __ldg(ind + (perm ? __ldg(perm + k) : k)) : 0xffffffffu;
+      const unsigned peers = __match_any_sync(0xffffffffu, x);
+      if (x < dim && (threadIdx.x & 31u) == (unsigned)(__ffs(peers) - 1)) atomicAdd(cnt + x, (uint32_t)__popc(peers));
+    }
+  }
+  if (small) {
+    __syncthreads();
+    for (uint64_t i = threadIdx.x; i < dim; i += blockDim.x)
+      if (hist[i]) atomicAdd(cnt + i, hist[i]);
+  }
+}
+
+static void count_rows(const uint32_t* ind, const uint32_t* perm, uint64_t n, uint64_t dim, uint32_t* cnt,
+                       cudaStream_t st) {
+  if (!n) return;
+  const bool small = dim <= kSmemCountRows;
+  row_count_kernel<<<small ? std::min(grid_for(n), 148 * 4) : grid_for(n), 256, small ? dim * 4 : 0, st>>>(
+      ind, perm, n, dim, cnt);
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+Ingest ingest_begin(Tensor& t) {
+  Ingest g;
+  const uint64_t n = t.nnz;
+  if (!n) return g;
+  const int N = t.nmodes;
+  const int WR = (N + 1 <= 4) ? 4 : (N + 1 <= 8 ? 8 : 16);
+  uint64_t need = t.aos.p ? 0 : n * WR * 4;
+  uint32_t mask = 0;
+  for (int m = 0; m < N; ++m)
+    if (t.dims[m] >= (1ull << 18) && t.dims[m] < (1ull << 31) && !t.hot_cnt[m].p) {
+      mask |= 1u << m;
+      need += t.dims[m] * 4;
+    }
+  size_t free_b = 0, total_b = 0;
+  SF_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  if ((double)need > 0.4 * (double)free_b) return g;  // leave it to the first plan
+  if (!t.aos.p) {
+    t.aos.alloc((size_t)n * WR * 4 + 64);
+    t.aos_words = WR;
+    g.aos = true;
+  }
+  for (int m = 0; m < N; ++m)
+    if (mask >> m & 1) {
+      t.hot_cnt[m].alloc(t.dims[m] * 4 + 16);
+      SF_CUDA(cudaMemsetAsync(t.hot_cnt[m].p, 0, t.dims[m] * 4, t.stream));
+    }
+  g.cnt_mask = mask;
+  SF_CUDA(cudaStreamSynchronize(t.stream));  // the segment streams count into zeroed arrays
+  return g;
+}
+
+void ingest_segment(Tensor& t, const Ingest& g, uint64_t a, uint64_t len, cudaStream_t st) {
+  if (g.aos) aos_segment(t, a, len, st);
+  for (int m = 0; m < t.nmodes; ++m)
+    if (g.cnt_mask >> m & 1) {
+      count_rows(t.ind[m].as<uint32_t>() + a, nullptr, len, t.dims[m], t.hot_cnt[m].as<uint32_t>(), st);
+    }
   SF_CUDA(cudaGetLastError());
 }
 
@@ -196,55 +299,143 @@ static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_o
   if (dv.Current() == p0.as<uint32_t>()) pos_out = std::move(p0); else pos_out = std::move(p1);
 }
 
-struct SliceOf {
-  uint64_t Is;
-  __host__ __device__ uint64_t operator()(uint64_t k) const { return k / Is; }
-};
+// First j > k with keys[j] >= target, or n (keys sorted ascending, keys[k] < target):
+// galloping from k, then bisection -- O(log(run length)) reads, mostly cached for short runs.
+__device__ __forceinline__ uint64_t run_end(const uint64_t* __restrict__ keys, uint64_t n, uint64_t k,
+                                            uint64_t target) {
+  uint64_t lo = k, hi = n, step = 1;
+  while (true) {
+    const uint64_t j = lo + step;
+    if (j >= n) break;
+    if (__ldg(keys + j) >= target) {
+      hi = j;
+      break;
+    }
+    lo = j;
+    step <<= 1;
+  }
+  while (hi - lo > 1) {
+    const uint64_t mid = lo + (hi - lo) / 2;
+    if (__ldg(keys + mid) >= target) hi = mid; else lo = mid;
+  }
+  return hi;
+}
 
-// Slice statistics from the run lengths of the slice ids (one thread per slice).
-__global__ void slice_stats_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ nruns,
-                                   FeatAcc* __restrict__ acc) {
+// Slice and fiber statistics of the sorted matricized keys in one pass (
+// reading R4): slices = runs of i_n = key / I_s, fibers = runs of the key.  A warp reads a
+// tile of 32 x RS_ITEMS consecutive keys (RS_ITEMS per lane, coalesced); a run's length is the
+// distance to the next run start -- in the lane, in a later lane (warp suffix-min of each
+// lane's first start), or, for the one run of each kind that leaves the tile, found by
+// galloping in global memory (run_end).
+constexpr int RS_ITEMS = 8;
+__global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restrict__ keys, uint64_t n, Div64 Is,
+                                                        unsigned long long* __restrict__ runs,
+                                                        FeatAcc* __restrict__ acc) {
   __shared__ unsigned long long h[SF_HIST_BINS];
   for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x) h[i] = 0;
   __syncthreads();
-  const uint64_t nr = *nruns;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned long long ms = 0, sq = 0;
-  for (uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nr; r += stride) {
-    const unsigned long long len = cnt[r];
-    ms = max(ms, len);
-    sq += len * len;
-    atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
+  constexpr uint64_t NONE = ~0ull;
+  constexpr uint64_t TILE = 32 * RS_ITEMS;
+  const unsigned full = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x / 32);
+  const uint64_t ntiles = (n + TILE - 1) / TILE;
+  unsigned long long ns = 0, nf = 0, ms = 0, mf = 0, sq = 0;
+  for (uint64_t w = (uint64_t)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32; w < ntiles; w += nwarps) {
+    const uint64_t t0 = w * TILE, t1 = min(n, t0 + TILE);
+    const uint64_t base = t0 + (uint64_t)lane * RS_ITEMS;
+    uint64_t x[RS_ITEMS];
+    if (base + RS_ITEMS <= n) {
+      const ulonglong2* v = reinterpret_cast<const ulonglong2*>(keys + base);
+#pragma unroll
+      for (int q = 0; q < RS_ITEMS / 2; ++q) {
+        const ulonglong2 u = __ldg(v + q);
+        x[2 * q] = u.x;
+        x[2 * q + 1] = u.y;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < RS_ITEMS; ++i) x[i] = (base + i < n) ? __ldg(keys + base + i) : 0;
+    }
+    uint64_t prev = __shfl_up_sync(full, x[RS_ITEMS - 1], 1);
+    if (lane == 0) prev = t0 ? __ldg(keys + t0 - 1) : 0;
+    // start flags (bit i: item i starts a fiber / a slice; items past n start nothing)
+    unsigned fs = 0, ss = 0;
+    uint64_t sprev = Is.div(prev);
+#pragma unroll
+    for (int i = 0; i < RS_ITEMS; ++i) {
+      const uint64_t k = base + i;
+      const uint64_t sl = Is.div(x[i]);
+      if (k < n) {
+        if (k == 0 || x[i] != prev) fs |= 1u << i;
+        if (k == 0 || sl != sprev) ss |= 1u << i;
+      }
+      prev = x[i];
+      sprev = sl;
+    }
+    // the first start at or after the next lane, for either kind; t1 when the tile ends there
+    // with n (the runs end at n), NONE when a run may continue past the tile
+    uint64_t ffirst = fs ? base + (__ffs(fs) - 1) : NONE, sfirst = ss ? base + (__ffs(ss) - 1) : NONE;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const uint64_t a = __shfl_down_sync(full, ffirst, off), b = __shfl_down_sync(full, sfirst, off);
+      if (lane + off < 32) {
+        ffirst = min(ffirst, a);
+        sfirst = min(sfirst, b);
+      }
+    }
+    uint64_t fnext = __shfl_down_sync(full, ffirst, 1), snext = __shfl_down_sync(full, sfirst, 1);
+    if (lane == 31) fnext = snext = NONE;
+    if (t1 == n) {
+      fnext = min(fnext, n);
+      snext = min(snext, n);
+    }
+#pragma unroll
+    for (int i = RS_ITEMS - 1; i >= 0; --i) {
+      const uint64_t k = base + i;
+      if (fs >> i & 1) {
+        const uint64_t e = (fnext != NONE) ? fnext : run_end(keys, n, t1 - 1, x[i] + 1);
+        const unsigned long long len = e - k;
+        ++nf;
+        mf = max(mf, len);
+        fnext = k;
+      }
+      if (ss >> i & 1) {
+        const uint64_t e = (snext != NONE) ? snext : run_end(keys, n, t1 - 1, (Is.div(x[i]) + 1) * Is.d);
+        const unsigned long long len = e - k;
+        ++ns;
+        ms = max(ms, len);
+        sq += len * len;
+        atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
+        snext = k;
+      }
+    }
   }
   typedef cub::BlockReduce<unsigned long long, 256> BR;
   __shared__ typename BR::TempStorage tmp;
-  const unsigned long long a = BR(tmp).Reduce(ms, cub::Max());
+  unsigned long long r[5];
+  r[0] = BR(tmp).Sum(ns);
   __syncthreads();
-  const unsigned long long c = BR(tmp).Sum(sq);
+  r[1] = BR(tmp).Sum(nf);
+  __syncthreads();
+  r[2] = BR(tmp).Reduce(ms, cub::Max());
+  __syncthreads();
+  r[3] = BR(tmp).Reduce(mf, cub::Max());
+  __syncthreads();
+  r[4] = BR(tmp).Sum(sq);
   if (threadIdx.x == 0) {
-    atomicMax(&acc->max_slice, a);
-    atomicAdd(&acc->sum_sq, c);
+    if (r[0]) atomicAdd(runs, r[0]);
+    if (r[1]) atomicAdd(runs + 1, r[1]);
+    atomicMax(&acc->max_slice, r[2]);
+    atomicMax(&acc->max_fiber, r[3]);
+    if (r[4]) atomicAdd(&acc->sum_sq, r[4]);
   }
   __syncthreads();
   for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x)
     if (h[i]) atomicAdd(&acc->hist[i], h[i]);
 }
 
-__global__ void run_max_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ nruns,
-                               unsigned long long* __restrict__ out) {
-  const uint64_t nr = *nruns;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  unsigned long long m = 0;
-  for (uint64_t r = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nr; r += stride)
-    m = max(m, (unsigned long long)cnt[r]);
-  typedef cub::BlockReduce<unsigned long long, 256> BR;
-  __shared__ typename BR::TempStorage tmp;
-  const unsigned long long a = BR(tmp).Reduce(m, cub::Max());
-  if (threadIdx.x == 0) atomicMax(out, a);
-}
-
-// Features (reading R4) of the matricized order: slices = runs of
-// i_n = key / I_s, fibers = runs of the key, each found by one run-length encode.
+// Features (reading R4) of the matricized order.
 static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_features_t* f) {
   const uint64_t n = t.nnz;
   const int s = secondary_mode(t, mode);
@@ -256,32 +447,19 @@ static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_f
   f->mode = mode;
   f->secondary = s;
   if (n > 0) {
-    const uint64_t max_slices = std::min<uint64_t>(n, t.dims[mode]);
-    DevBuf scnt(max_slices * 4 + 16), fcnt(n * 4 + 16), nr(16), accb(sizeof(FeatAcc));
-    SF_CUDA(cudaMemsetAsync(accb.p, 0, sizeof(FeatAcc), t.stream));
-    auto sl = thrust::make_transform_iterator(keys, SliceOf{Is});
-    auto discard = thrust::make_discard_iterator();
-    uint32_t* nrs = nr.as<uint32_t>();
-    size_t t1 = 0, t2 = 0;
-    SF_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, t1, sl, discard, scnt.as<uint32_t>(), nrs, (int64_t)n,
-                                               t.stream));
-    SF_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, t2, keys, discard, fcnt.as<uint32_t>(), nrs + 1, (int64_t)n,
-                                               t.stream));
-    DevBuf tmp(std::max(t1, t2) + 16);
-    SF_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, t1, sl, discard, scnt.as<uint32_t>(), nrs, (int64_t)n,
-                                               t.stream));
-    SF_CUDA(cub::DeviceRunLengthEncode::Encode(tmp.p, t2, keys, discard, fcnt.as<uint32_t>(), nrs + 1, (int64_t)n,
-                                               t.stream));
-    slice_stats_kernel<<<grid_for(max_slices), 256, 0, t.stream>>>(scnt.as<uint32_t>(), nrs, accb.as<FeatAcc>());
-    run_max_kernel<<<grid_for(n), 256, 0, t.stream>>>(fcnt.as<uint32_t>(), nrs + 1, &accb.as<FeatAcc>()->max_fiber);
-    count_launch(6);
+    DevBuf accb(sizeof(FeatAcc) + 16);
+    unsigned long long* runs = reinterpret_cast<unsigned long long*>(accb.as<char>() + sizeof(FeatAcc));
+    SF_CUDA(cudaMemsetAsync(accb.p, 0, sizeof(FeatAcc) + 16, t.stream));
+    run_stats_kernel<<<grid_for((n + RS_ITEMS - 1) / RS_ITEMS), 256, 0, t.stream>>>(keys, n, Div64(Is), runs,
+                                                                                  accb.as<FeatAcc>());
+    count_launch();
     SF_CUDA(cudaGetLastError());
-    uint32_t c[2];
     FeatAcc a;
+    unsigned long long c[2];
     {
-      void* dst[2] = {c, &a};
-      const void* src[2] = {nr.p, accb.p};
-      const size_t nb[2] = {8, sizeof(FeatAcc)};
+      void* dst[2] = {&a, c};
+      const void* src[2] = {accb.p, runs};
+      const size_t nb[2] = {sizeof(FeatAcc), 16};
       d2h_small(t.stream, 2, dst, src, nb);
     }
     f->num_slices = c[0];
@@ -328,11 +506,12 @@ struct TileParams {
 // Single staged mode == the secondary key s: the tile id is (key % I_s) / block_rows, read
 // from the (sequential) matricized keys instead of a random 4-byte gather of i_s.
 __global__ void tile_key_from_keys_kernel(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ pos,
-                                          uint64_t n, uint64_t Is, uint32_t block_rows,
+                                          uint64_t n, Div64 Is, uint32_t block_rows,
                                           uint64_t* __restrict__ tkey, uint32_t* __restrict__ tpos) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    tkey[k] = (keys[k] % Is) / block_rows;
+    const uint64_t key = keys[k];
+    tkey[k] = (uint32_t)(key - Is.div(key) * Is.d) / block_rows;
     tpos[k] = pos[k];
   }
 }
@@ -402,18 +581,6 @@ __global__ void gather_aos_kernel(const uint32_t* __restrict__ aos, const uint32
 
 // ---- hot-row cache (launch.hot_kb; DESIGN.md §5 "hot-row cache") ----
 // cnt[x] = nonzeros of the handle whose mode-m index is x
-__global__ void hot_count_all_kernel(const uint32_t* __restrict__ ind, uint64_t n, uint32_t* __restrict__ cnt) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) atomicAdd(cnt + __ldg(ind + k), 1u);
-}
-
-// cnt[x] = nonzeros of this plan whose gathered index (mode m) is x
-__global__ void hot_count_kernel(const uint32_t* __restrict__ ind, const uint32_t* __restrict__ perm, uint64_t n,
-                                 uint32_t* __restrict__ cnt) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride)
-    atomicAdd(cnt + __ldg(ind + __ldg(perm + k)), 1u);
-}
 
 struct HotCount {
   const uint32_t* cnt[SF_MAX_MODES];
@@ -453,11 +620,20 @@ __global__ void hot_flag_kernel(const uint32_t* __restrict__ cnt, uint64_t dim, 
     flag[x] = __ldg(cnt + x) > tau ? 1u : 0u;
 }
 
-__global__ void hot_rows_kernel(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ slot, uint64_t dim,
-                                uint32_t tau, uint32_t* __restrict__ rows) {
+// rows[slot[x]] = x for every hot row x, and slot[] becomes the record's index map in place:
+// map[x] = slot[x] | bit for hot rows, x for the others (one lookup per field in the gather)
+__global__ void hot_rows_kernel(const uint32_t* __restrict__ cnt, uint32_t* __restrict__ slot, uint64_t dim,
+                                uint32_t tau, uint32_t bit, uint32_t* __restrict__ rows) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < dim; x += stride)
-    if (__ldg(cnt + x) > tau) rows[__ldg(slot + x)] = (uint32_t)x;
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < dim; x += stride) {
+    if (__ldg(cnt + x) > tau) {
+      const uint32_t q = slot[x];
+      rows[q] = (uint32_t)x;
+      slot[x] = q | bit;
+    } else {
+      slot[x] = (uint32_t)x;
+    }
+  }
 }
 
 // The smallest threshold tau with #{rows of every slot in hc with count > tau} <= budget: 32
@@ -503,11 +679,7 @@ static void ensure_hot_counts(Tensor& t, int m) {
   if (t.hot_cnt[m].p) return;
   t.hot_cnt[m].alloc(t.dims[m] * 4 + 16);
   SF_CUDA(cudaMemsetAsync(t.hot_cnt[m].p, 0, t.dims[m] * 4, t.stream));
-  if (t.nnz)
-    hot_count_all_kernel<<<grid_for(t.nnz), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), t.nnz,
-                                                               t.hot_cnt[m].as<uint32_t>());
-  count_launch();
-  SF_CUDA(cudaGetLastError());
+  count_rows(t.ind[m].as<uint32_t>(), nullptr, t.nnz, t.dims[m], t.hot_cnt[m].as<uint32_t>(), t.stream);
 }
 
 void hot_coverage(Tensor& t, int m, uint64_t rows) {
@@ -535,53 +707,77 @@ struct RecParams {
   int fmap[8];
   int nfields;
   uint32_t boff[8];
-  // hot-row cache: field d (a gathered slot) with hcnt[d] != nullptr becomes
-  // hslot[d][x] | hbit[d] when the row x has hcnt[d][x] > htau
-  const uint32_t* hcnt[8];
-  const uint32_t* hslot[8];
-  uint32_t hbit[8];
-  uint32_t htau;
+  // hot-row cache: field d (a gathered slot) with hmap[d] != nullptr becomes hmap[d][x]
+  // (the row's slot in the hot block with the slot's hot bit set, or x itself)
+  const uint32_t* hmap[8];
 };
 
+// Record fields in slot order from a raw AoS record (with the hot-row index map applied).
+template <int WR, int WK>
+__device__ __forceinline__ void rec_fields(const uint32_t (&w)[WR], const RecParams& rp, uint32_t (&o)[WK]) {
+#pragma unroll
+  for (int d = 0; d < WK; ++d) {
+    uint32_t x = 0;
+#pragma unroll
+    for (int q = 0; q < WR; ++q) x = (rp.fmap[d] == q) ? w[q] : x;
+    if (rp.hmap[d]) x = __ldg(rp.hmap[d] + x);
+    o[d] = x;
+  }
+}
+
+template <int WK>
+__device__ __forceinline__ void rec_store(const uint32_t (&o)[WK], const RecParams& rp, uint32_t* __restrict__ rec,
+                                          uint64_t k) {
+  if (WK == 8 && rp.nfields > 0) {  // packed 16-byte record
+    uint32_t o0 = 0, o1 = 0, o2 = 0;
+#pragma unroll
+    for (int f = 0; f < 8; ++f) {
+      if (f >= rp.nfields) break;
+      const uint32_t x = o[f < WK ? f : 0], off = rp.boff[f], wi = off >> 5, sh = off & 31u;
+      const uint32_t lo = x << sh, hi = sh ? (x >> (32u - sh)) : 0u;
+      if (wi == 0) { o0 |= lo; o1 |= hi; } else if (wi == 1) { o1 |= lo; o2 |= hi; } else { o2 |= lo; }
+    }
+    uint32_t val = 0;
+#pragma unroll
+    for (int f = 0; f < WK; ++f) val = (f == rp.nfields) ? o[f] : val;
+    reinterpret_cast<uint4*>(rec)[k] = make_uint4(o0, o1, o2, val);
+    return;
+  }
+  uint4* dst = reinterpret_cast<uint4*>(rec + k * WK);
+#pragma unroll
+  for (int q = 0; q < WK / 4; ++q) dst[q] = make_uint4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+}
+
+// Kernel-order records from the AoS copy: rec[k] = record(aos[perm[k]]).  GR records per
+// thread and iteration (GR = 4 measured slower than 1: fewer resident warps).
+constexpr int GR = 1;
 template <int WR, int WK>
 __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
                                   uint64_t n, RecParams rp, uint32_t* __restrict__ rec) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)perm[k] * WR);
-    uint32_t w[WR];
+  for (uint64_t k0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k0 < n; k0 += GR * stride) {
+    uint32_t w[GR][WR];
 #pragma unroll
-    for (int q = 0; q < WR / 4; ++q) {
-      const uint4 v = __ldg(src + q);
-      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
-    }
-    uint32_t o[WK];
+    for (int j = 0; j < GR; ++j) {
+      const uint64_t k = k0 + j * stride;
+      if (k < n) {
+        const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)__ldg(perm + k) * WR);
 #pragma unroll
-    for (int d = 0; d < WK; ++d) {
-      uint32_t x = 0;
-#pragma unroll
-      for (int q = 0; q < WR; ++q) x = (rp.fmap[d] == q) ? w[q] : x;
-      if (rp.hcnt[d] && __ldg(rp.hcnt[d] + x) > rp.htau) x = __ldg(rp.hslot[d] + x) | rp.hbit[d];
-      o[d] = x;
-    }
-    if (WK == 8 && rp.nfields > 0) {  // packed 16-byte record
-      uint32_t o0 = 0, o1 = 0, o2 = 0;
-#pragma unroll
-      for (int f = 0; f < 8; ++f) {
-        if (f >= rp.nfields) break;
-        const uint32_t x = o[f < WK ? f : 0], off = rp.boff[f], wi = off >> 5, sh = off & 31u;
-        const uint32_t lo = x << sh, hi = sh ? (x >> (32u - sh)) : 0u;
-        if (wi == 0) { o0 |= lo; o1 |= hi; } else if (wi == 1) { o1 |= lo; o2 |= hi; } else { o2 |= lo; }
+        for (int q = 0; q < WR / 4; ++q) {
+          const uint4 v = __ldg(src + q);
+          w[j][4 * q] = v.x; w[j][4 * q + 1] = v.y; w[j][4 * q + 2] = v.z; w[j][4 * q + 3] = v.w;
+        }
       }
-      uint32_t val = 0;
-#pragma unroll
-      for (int f = 0; f < WK; ++f) val = (f == rp.nfields) ? o[f] : val;
-      reinterpret_cast<uint4*>(rec)[k] = make_uint4(o0, o1, o2, val);
-      continue;
     }
-    uint4* dst = reinterpret_cast<uint4*>(rec + k * WK);
+    uint32_t o[GR][WK];
 #pragma unroll
-    for (int q = 0; q < WK / 4; ++q) dst[q] = make_uint4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+    for (int j = 0; j < GR; ++j)
+      if (k0 + j * stride < n) rec_fields<WR, WK>(w[j], rp, o[j]);
+#pragma unroll
+    for (int j = 0; j < GR; ++j) {
+      const uint64_t k = k0 + j * stride;
+      if (k < n) rec_store<WK>(o[j], rp, rec, k);
+    }
   }
 }
 
@@ -704,7 +900,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       DevBuf k0(nl * 8 + 16), k1(nl * 8 + 16), p1(nl * 4 + kPadBytes);
       if (staged_is_secondary)
         tile_key_from_keys_kernel<<<grid_for(nl), 256, 0, t.stream>>>(
-            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, t.dims[s], launch.block_rows[s],
+            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, Div64(t.dims[s]), launch.block_rows[s],
             k0.as<uint64_t>(), perm.as<uint32_t>());
       else
         tile_key_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tp, pos0.as<uint32_t>() + lo, nl, k0.as<uint64_t>(),
@@ -801,9 +997,7 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
         } else {
           cnt->alloc(t.dims[m] * 4 + 16);
           SF_CUDA(cudaMemsetAsync(cnt->p, 0, t.dims[m] * 4, t.stream));
-          hot_count_kernel<<<grid_for(nl), 256, 0, t.stream>>>(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl,
-                                                               cnt->as<uint32_t>());
-          count_launch();
+          count_rows(t.ind[m].as<uint32_t>(), perm.as<uint32_t>(), nl, t.dims[m], cnt->as<uint32_t>(), t.stream);
         }
         hcnt_ptr[q] = cnt->as<uint32_t>();
         hc.cnt[hc.n] = cnt->as<uint32_t>();
@@ -836,18 +1030,15 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
           count_launch(2);
           if (cnt == 0) continue;
           p.hot_rows[q].alloc(cnt * 4 + 16);
-          hot_rows_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt_ptr[q], hslot[q].as<uint32_t>(), I, tau,
-                                                             p.hot_rows[q].as<uint32_t>());
-          count_launch();
           p.hot_bit[q] = packed ? (1u << index_bits(I)) : 0x80000000u;
+          hot_rows_kernel<<<grid_for(I), 256, 0, t.stream>>>(hcnt_ptr[q], hslot[q].as<uint32_t>(), I, tau,
+                                                             p.hot_bit[q], p.hot_rows[q].as<uint32_t>());
+          count_launch();
           p.hot_count[q] = cnt;
           p.hot_off[q] = total;
           total += cnt;
-          rp.hcnt[1 + q] = hcnt_ptr[q];
-          rp.hslot[1 + q] = hslot[q].as<uint32_t>();
-          rp.hbit[1 + q] = p.hot_bit[q];
+          rp.hmap[1 + q] = hslot[q].as<uint32_t>();
         }
-        rp.htau = tau;
         p.hot_total = total;
         trace_mark("build: hot rows");
         if (total) p.hot_cache.alloc(total * rank * 4 + 64);

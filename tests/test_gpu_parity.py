@@ -107,6 +107,46 @@ def test_exact_integers_bitwise(cuda_device):
             assert np.array_equal(Yg[n].astype(np.float64), Y), L.as_dict()
 
 
+def _run_case(kind):
+    """Index sets whose slice / fiber runs start, end and cross the feature kernel's 256-key
+    warp tiles in every way: single nonzero, one run of exactly a tile, runs one past a tile,
+    mixed run lengths, a heavy slice spanning hundreds of tiles."""
+    rng = np.random.default_rng(17)
+    if kind == "one":
+        return (3, 4, 5), [np.array([2], np.uint32), np.array([1], np.uint32), np.array([4], np.uint32)]
+    if kind in ("tile", "tile+1", "tile-1"):
+        n = 256 + {"tile": 0, "tile+1": 1, "tile-1": -1}[kind]
+        return (3, 4, 5), [np.full(n, 1, np.uint32), np.full(n, 2, np.uint32), np.full(n, 3, np.uint32)]
+    if kind == "mixed":
+        lens = [300, 1, 255, 256, 1, 1, 700, 2, 257, 513, 3, 1024]
+        i0 = np.concatenate([np.full(L, k, np.uint32) for k, L in enumerate(lens)])
+        n = len(i0)
+        i1 = (rng.integers(0, 3, n) * (rng.random(n) < 0.9)).astype(np.uint32)  # long fibers too
+        i2 = rng.integers(0, 40, n).astype(np.uint32)
+        perm = rng.permutation(n)
+        return (len(lens), 3, 40), [i0[perm], i1[perm], i2[perm]]
+    # heavy: one slice of mode 0 holds half the nonzeros
+    n = 100003
+    i0 = np.where(rng.random(n) < 0.5, 0, rng.integers(0, 5000, n)).astype(np.uint32)
+    i1 = rng.integers(0, 3, n).astype(np.uint32)
+    i2 = rng.integers(0, 70000, n).astype(np.uint32)
+    return (5000, 3, 70000), [i0, i1, i2]
+
+
+@pytest.mark.parametrize("kind", ["one", "tile", "tile+1", "tile-1", "mixed", "heavy"])
+def test_features_run_edges(cuda_device, kind):
+    dims, inds = _run_case(kind)
+    vals = np.ones(len(inds[0]), np.float32)
+    with sf.Tensor(dims, G.dev_inds(inds), G.dev_f(vals)) as t:
+        for n in range(3):
+            f = t.features(n)
+            of = oplan.features(dims, inds, n)
+            for k in ("num_slices", "num_fibers", "max_nnz_per_slice", "max_nnz_per_fiber",
+                      "sum_sq_nnz_per_slice", "secondary"):
+                assert f[k] == of[k], (kind, n, k)
+            assert f["slice_hist"] == list(of["slice_hist"]), (kind, n)
+
+
 def test_plan_bit_exact_vs_oracle(cuda_device):
     dims = (300, 41, 530)
     inds, vals = synth.gen_coo(dims, 25000, 8, zipf=(1.0, 0.5, 0.8))
@@ -278,6 +318,32 @@ def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
                 t.mttkrp(n, tf, y)
                 torch.cuda.synchronize()
                 G.assert_parity(y.cpu().numpy(), dims, inds, vals, facs, 16, n)
+
+
+@pytest.mark.parametrize("segments", [3, 8])
+def test_presort_wide_keys_bit_exact(cuda_device, segments, monkeypatch):
+    """A handle whose modes mix presorted keys and keys that with the input position need more
+    than 64 bits (those are sorted at their first plan, not during the upload): same matricized
+    order, features and chunks as the full sort (oracle/plan.py ==).  Position bits 19: mode 2
+    (key 1e8 x 1e6, 47 bits) is wide, modes 0 and 1 (1e6 x 2e6, 41 bits) are presorted."""
+    dims = (1_000_000, 2_000_000, 100_000_000)
+    inds, vals = synth.gen_coo(dims, 300_007, 14, zipf=(1.1, 0.5, 1.1))
+    ti = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    tv = torch.from_numpy(vals).pin_memory()
+    for flag in ("", "no_presort"):
+        monkeypatch.setenv("SF_DEBUG", flag)
+        with sf.Tensor(dims, ti, tv, segments=segments, streams=3) as t:
+            for n in range(3):
+                t.set_launch(n, 16, sf.Launch.make(kernel=FRAG, chunk_nnz=100))
+                f = t.features(n)
+                of = oplan.features(dims, inds, n)
+                for k in ("num_slices", "num_fibers", "max_nnz_per_slice", "max_nnz_per_fiber",
+                          "sum_sq_nnz_per_slice"):
+                    assert f[k] == of[k], (flag, n, k)
+                perm, chunks = t.plan_export(n, 16)
+                ref = oplan.plan_order(dims, inds, n, (), {})
+                assert np.array_equal(perm.astype(np.int64), ref), (flag, n)
+                assert np.array_equal(chunks.astype(np.int64), oplan.chunks(np.zeros(len(ref), np.int64), 100))
 
 
 @pytest.mark.parametrize("kind", ["l2tiles", "staged", "hot"])

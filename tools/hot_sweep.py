@@ -58,19 +58,18 @@ def main():
                                    flags=flags, hot_kb=hb * 1024)
                 T.set_launch(n, R, L)
                 info = T.plan_info(n, R)
-                for persist in [False]:
-                    for _ in range(3):
-                        T.mttkrp(n, facs, out, stream=s)
-                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    e0.record(s)
-                    for _ in range(args.reps):
-                        T.mttkrp(n, facs, out, stream=s)
-                    e1.record(s)
-                    torch.cuda.synchronize()
-                    ms = e0.elapsed_time(e1) / args.reps
-                    print(json.dumps({"config": name, "mode": n, "l2tiles": bool(flags & sf.LAUNCH_L2_TILES),
-                                      "hot_mb": hb, "ms": round(ms, 4),
-                                      "plan_ms": round(info["plan_ms"], 2), "selector": base}), flush=True)
+                for _ in range(3):
+                    T.mttkrp(n, facs, out, stream=s)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                for _ in range(args.reps):
+                    T.mttkrp(n, facs, out, stream=s)
+                e1.record(s)
+                torch.cuda.synchronize()
+                ms = e0.elapsed_time(e1) / args.reps
+                print(json.dumps({"config": name, "mode": n, "l2tiles": bool(flags & sf.LAUNCH_L2_TILES),
+                                  "hot_mb": hb, "ms": round(ms, 4),
+                                  "plan_ms": round(info["plan_ms"], 2), "selector": base}), flush=True)
             T.plan_release(n, R)
             del out
             torch.cuda.empty_cache()
