@@ -104,6 +104,13 @@ struct BlockCache {
     *got = b;
     return q;
   }
+  size_t cached_on(int dev) {
+    std::lock_guard<std::mutex> g(mu);
+    size_t b = 0;
+    for (auto it = free_blocks.lower_bound({dev, 0}); it != free_blocks.end() && it->first.first == dev; ++it)
+      b += it->first.second;
+    return b;
+  }
   void put(void* q, size_t b) {
     int dev = 0;
     cudaPointerAttributes a{};
@@ -132,6 +139,14 @@ struct BlockCache {
   }
 };
 static BlockCache g_cache;
+
+size_t device_free_bytes() {
+  size_t free_b = 0, total_b = 0;
+  SF_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  int dev = 0;
+  SF_CUDA(cudaGetDevice(&dev));
+  return free_b + g_cache.cached_on(dev);
+}
 
 // Bytes held by live library buffers (all devices) and their high-water mark (sf_device_bytes).
 static std::atomic<uint64_t> g_in_use{0}, g_peak{0};

@@ -242,6 +242,8 @@ void d2d_copy(void* dst, const void* src, size_t bytes, cudaStream_t s);
 // upload || presort: decide and allocate (returns false: no mode qualifies / disabled by
 // SF_PRESORT=0 / not enough memory), per-segment work on the upload stream, CUB temp bytes
 // one segment's sort needs.
+// Free device memory of the current device: the driver's plus the library's cached blocks.
+size_t device_free_bytes();
 bool presort_begin(Tensor& t, uint64_t seg_len);
 void presort_segment(Tensor& t, uint64_t a, uint64_t len, cudaStream_t s, void* temp, size_t temp_bytes);
 size_t presort_temp_bytes(const Tensor& t, uint64_t seg_len);

@@ -108,8 +108,7 @@ bool presort_begin(Tensor& t, uint64_t seg_len) {
   int modes = 0;
   for (int m = 0; m < t.nmodes; ++m) modes += (key_bits(t, m) + pb <= 64);
   if (!modes) return false;
-  size_t free_b = 0, total_b = 0;
-  SF_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  const size_t free_b = device_free_bytes();
   // pre keys + the segment staging buffer now, and a merge buffer + split keys/positions later
   if ((double)n * 8.0 * (modes + 4) > 0.6 * (double)free_b) return false;
   t.pre_pb = pb;
@@ -210,8 +209,7 @@ Ingest ingest_begin(Tensor& t) {
       mask |= 1u << m;
       need += t.dims[m] * 4;
     }
-  size_t free_b = 0, total_b = 0;
-  SF_CUDA(cudaMemGetInfo(&free_b, &total_b));
+  const size_t free_b = device_free_bytes();
   if ((double)need > 0.4 * (double)free_b) return g;  // leave it to the first plan
   if (!t.aos.p) {
     t.aos.alloc((size_t)n * WR * 4 + 64);
@@ -341,6 +339,10 @@ __global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restri
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x / 32);
   const uint64_t ntiles = (n + TILE - 1) / TILE;
   unsigned long long ns = 0, nf = 0, ms = 0, mf = 0, sq = 0;
+  // slices of < 2^RS_LOW_BINS nonzeros (nearly all in hyper-sparse modes) are binned in
+  // registers: shared-memory atomics on a handful of bins would serialise
+  constexpr int RS_LOW_BINS = 6;
+  unsigned hlow[RS_LOW_BINS] = {};
   for (uint64_t w = (uint64_t)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32; w < ntiles; w += nwarps) {
     const uint64_t t0 = w * TILE, t1 = min(n, t0 + TILE);
     const uint64_t base = t0 + (uint64_t)lane * RS_ITEMS;
@@ -406,10 +408,21 @@ __global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restri
         ++ns;
         ms = max(ms, len);
         sq += len * len;
-        atomicAdd(&h[63 - __clzll((long long)len)], 1ull);
+        const int bin = 63 - __clzll((long long)len);
+        if (bin < RS_LOW_BINS) {
+#pragma unroll
+          for (int b = 0; b < RS_LOW_BINS; ++b) hlow[b] += (b == bin);
+        } else {
+          atomicAdd(&h[bin], 1ull);
+        }
         snext = k;
       }
     }
+  }
+#pragma unroll
+  for (int b = 0; b < RS_LOW_BINS; ++b) {
+    const unsigned v = __reduce_add_sync(full, hlow[b]);
+    if (lane == 0 && v) atomicAdd(&h[b], (unsigned long long)v);
   }
   typedef cub::BlockReduce<unsigned long long, 256> BR;
   __shared__ typename BR::TempStorage tmp;

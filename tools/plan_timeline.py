@@ -24,6 +24,7 @@ def main():
     ap.add_argument("config", nargs="?", default="nell2")
     ap.add_argument("--out", default=None, help="also write the chrome trace here")
     ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--release", action="store_true", help="release each plan after building it (amazon)")
     args = ap.parse_args()
     import torch
     from torch.profiler import ProfilerActivity, profile
@@ -46,6 +47,8 @@ def main():
             T.plan(n, R)
             torch.cuda.synchronize()
             marks.append((f"plan {n}", time.perf_counter() - t0))
+            if args.release:
+                T.plan_release(n, R)
         T.close()
 
     one([], time.perf_counter())  # warm-up (module load, allocator)
