@@ -186,6 +186,12 @@ sf_status sf_comm_unique_id(void* id128);
 sf_status sf_comm_attach(sf_tensor_t t, int nranks, int rank, const void* id128);
 sf_status sf_comm_attach_transport(sf_tensor_t t, int nranks, int rank, sf_allgatherv_fn fn, void* ctx);
 sf_status sf_comm_detach(sf_tensor_t t);
+/* Diagnostic (collective: every rank of the attached comm calls it): a rank-stamped
+ * allgatherv (rank k sends k + 1 words) and alltoallv (rank r sends (r + q) % 3 + 1 words to
+ * rank q) of device buffers through the attached transport on `stream`, checked word by word
+ * on the host.  SF_OK, SF_ERR_NCCL on a wrong word or a failed collective, SF_ERR_INVALID_ARG
+ * without a comm.  Synchronizes. */
+sf_status sf_comm_check(sf_tensor_t t, void* stream);
 /* Replicated Y from the row-sharded local blocks after sf_mttkrp (optional):
  * full (device, I_mode x rank) receives every rank's owned rows, zeros elsewhere. */
 sf_status sf_allgather_rows(sf_tensor_t t, int mode, int rank, const float* local, float* full, void* stream);

@@ -104,7 +104,7 @@ EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
             "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
             "sf_trim_cache", "sf_shard_rows", "sf_comm_unique_id", "sf_comm_attach",
-            "sf_comm_attach_transport", "sf_comm_detach", "sf_allgather_rows", "sf_exchange_map",
+            "sf_comm_attach_transport", "sf_comm_detach", "sf_comm_check", "sf_allgather_rows", "sf_exchange_map",
             "sf_tensor_create_dist", "sf_device_bytes"]
 
 # int fn(void* ctx, const void* send, void* recv, const uint64_t* bytes, const uint64_t* displs,
@@ -149,6 +149,7 @@ def lib(build_if_missing: bool = True):
             L.sf_comm_attach.argtypes = [P, I, I, P]
             L.sf_comm_attach_transport.argtypes = [P, I, I, ALLGATHERV_FN, P]
             L.sf_comm_detach.argtypes = [P]
+            L.sf_comm_check.argtypes = [P, P]
             L.sf_allgather_rows.argtypes = [P, I, I, P, P, P]
             L.sf_exchange_map.argtypes = [I, P, P, P]
             L.sf_device_bytes.argtypes = [ctypes.POINTER(U64), ctypes.POINTER(U64), I]
@@ -325,6 +326,10 @@ class Tensor:
 
     def comm_detach(self):
         _check(lib().sf_comm_detach(self._h))
+
+    def comm_check(self, stream=None):
+        """Collective self-test of the attached transport (sf_comm_check)."""
+        _check(lib().sf_comm_check(self._h, _stream_handle(stream)))
 
     def allgather_rows(self, mode, local, full, stream=None):
         """Replicated Y (full, I_mode x R on every rank) from the row-sharded local blocks."""

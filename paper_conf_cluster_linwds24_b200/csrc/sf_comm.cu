@@ -370,6 +370,64 @@ sf_status sf_comm_detach(sf_tensor_t h) {
   });
 }
 
+sf_status sf_comm_check(sf_tensor_t h, void* stream) {
+  return comm_guard([&]() -> sf_status {
+    if (!h) throw StatusError{SF_ERR_INVALID_ARG, "NULL handle"};
+    Tensor* t = reinterpret_cast<Tensor*>(h);
+    if (!t->comm) throw StatusError{SF_ERR_INVALID_ARG, "no comm attached"};
+    SF_CUDA(cudaSetDevice(t->device));
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    Comm& c = *t->comm;
+    const int P = c.nranks, r = c.rank;
+    // allgatherv: rank k contributes k + 1 words k * 1000 + i
+    std::vector<uint64_t> bytes(P), displs(P);
+    uint64_t tot = 0;
+    for (int k = 0; k < P; ++k) {
+      bytes[k] = 4ull * (k + 1);
+      displs[k] = tot;
+      tot += bytes[k];
+    }
+    std::vector<uint32_t> mine(r + 1), got(tot / 4);
+    for (int i = 0; i <= r; ++i) mine[i] = (uint32_t)(r * 1000 + i);
+    DevBuf sb(bytes[r] + 16), rb(tot + 16);
+    SF_CUDA(cudaMemcpyAsync(sb.p, mine.data(), bytes[r], cudaMemcpyHostToDevice, s));
+    SF_CUDA(cudaMemsetAsync(rb.p, 0xff, tot, s));
+    c.allgatherv(sb.p, rb.p, bytes.data(), displs.data(), s);
+    SF_CUDA(cudaMemcpyAsync(got.data(), rb.p, tot, cudaMemcpyDeviceToHost, s));
+    SF_CUDA(cudaStreamSynchronize(s));
+    for (int k = 0; k < P; ++k)
+      for (int i = 0; i <= k; ++i)
+        if (got[displs[k] / 4 + i] != (uint32_t)(k * 1000 + i))
+          throw StatusError{SF_ERR_NCCL, "comm check: allgatherv delivered a wrong word"};
+    // alltoallv: rank a sends (a + b) % 3 + 1 words a * 1000000 + b * 1000 + i to rank b
+    auto nw = [](int a, int b) { return (uint64_t)((a + b) % 3 + 1); };
+    std::vector<uint64_t> sbytes(P), sdispl(P), rbytes(P), rdispl(P);
+    uint64_t st = 0, rt = 0;
+    for (int q = 0; q < P; ++q) {
+      sbytes[q] = 4 * nw(r, q);
+      sdispl[q] = st;
+      st += sbytes[q];
+      rbytes[q] = 4 * nw(q, r);
+      rdispl[q] = rt;
+      rt += rbytes[q];
+    }
+    std::vector<uint32_t> out(st / 4), in(rt / 4);
+    for (int q = 0; q < P; ++q)
+      for (uint64_t i = 0; i < nw(r, q); ++i) out[sdispl[q] / 4 + i] = (uint32_t)(r * 1000000 + q * 1000 + i);
+    DevBuf sa(st + 16), ra(rt + 16);
+    SF_CUDA(cudaMemcpyAsync(sa.p, out.data(), st, cudaMemcpyHostToDevice, s));
+    SF_CUDA(cudaMemsetAsync(ra.p, 0xff, rt, s));
+    c.alltoallv(sa.p, sbytes.data(), sdispl.data(), ra.p, rbytes.data(), rdispl.data(), s);
+    SF_CUDA(cudaMemcpyAsync(in.data(), ra.p, rt, cudaMemcpyDeviceToHost, s));
+    SF_CUDA(cudaStreamSynchronize(s));
+    for (int k = 0; k < P; ++k)
+      for (uint64_t i = 0; i < nw(k, r); ++i)
+        if (in[rdispl[k] / 4 + i] != (uint32_t)(k * 1000000 + r * 1000 + i))
+          throw StatusError{SF_ERR_NCCL, "comm check: alltoallv delivered a wrong word"};
+    return SF_OK;
+  });
+}
+
 // Host-only: the exchange map for given row ranges (tests pin it against the rule by hand).
 // send_first[k] = 1 iff rank k sends its first row; owner[k] = the rank receiving it (-1: empty).
 sf_status sf_exchange_map(int nranks, const uint64_t* ranges, int32_t* send_first, int32_t* owner) {

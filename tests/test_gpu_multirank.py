@@ -50,3 +50,35 @@ def test_nccl_ranks_exchange_matches_single(cuda_device):
     r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900, cwd=ROOT)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     assert "MULTIRANK OK" in r.stdout, r.stdout[-3000:]
+
+
+def test_nccl_one_rank_data_plane(cuda_device):
+    """The NCCL transport on the one GPU gpurun gives: a 1-rank communicator (dlopen'ed
+    libnccl.so.2, ncclGetUniqueId, ncclCommInitRank, grouped ncclBroadcast = allgatherv, grouped
+    ncclSend / ncclRecv to self = alltoallv) delivers every word (sf_comm_check), and the
+    attached handle's MTTKRP and sf_allgather_rows equal the unattached result bitwise."""
+    import numpy as np
+    import torch
+
+    import synth
+    import paper_conf_cluster_linwds24_b200 as sf
+    dims, R = (300, 200, 250), 32
+    inds, vals = synth.gen_coo(dims, 30011, 5, zipf=(1.0, 0.7, 0.9), val_kind="int")
+    facs = [torch.from_numpy(f).cuda() for f in synth.gen_factors(dims, R, 6, "int")]
+    ti = [torch.from_numpy(a.view(np.int32)).cuda() for a in inds]
+    tv = torch.from_numpy(vals).cuda()
+    for n in range(3):
+        ref = torch.empty((dims[n], R), device="cuda")
+        with sf.Tensor(dims, ti, tv) as T0:
+            T0.plan(n, R)
+            T0.mttkrp(n, facs, ref)
+        with sf.Tensor(dims, ti, tv) as T:
+            T.comm_attach(1, 0, sf.comm_unique_id())
+            T.comm_check()
+            T.plan(n, R)
+            y = torch.empty((T.plan_info(n, R)["out_rows"], R), device="cuda")
+            T.mttkrp(n, facs, y)
+            full = torch.empty((dims[n], R), device="cuda")
+            T.allgather_rows(n, y, full)
+            torch.cuda.synchronize()
+            assert torch.equal(y, ref) and torch.equal(full, ref)

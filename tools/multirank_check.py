@@ -37,6 +37,8 @@ def main():
             T1.mttkrp(n, facs, full)
         with sf.Tensor(dims, inds, vals) as T:
             sfdist.attach(T, world, rank)
+            if n == 0:
+                T.comm_check()  # the transport's allgatherv / alltoallv deliver every word
             T.plan(n, R)
             info = T.plan_info(n, R)
             y = torch.full((info["out_rows"], R), float("nan"), device=dev)
