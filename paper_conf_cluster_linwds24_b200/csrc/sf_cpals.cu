@@ -150,7 +150,8 @@ __global__ void __launch_bounds__(256) rowmat_rt_kernel(const float* __restrict_
 }
 
 // Alg. 1 line 5 and the Gram refresh fused (R in {16, 32, 64}): per tile of TR = 4096 / R
-// rows, M is read once into shared memory, A = M Vinv is formed in registers (4 rows x 4
+// rows, M is read once into shared memory (cp.async, the next tile in flight while this one
+// is computed: the synchronous load left every tile's DRAM latency exposed), A = M Vinv is formed in registers (4 rows x 4
 // columns per thread, rows strided by NRB so a quarter-warp's LDS.128 hit distinct banks),
 // written back through shared memory with coalesced stores, and G_n += A^T A (fp32 per
 // tile, fp64 across tiles) plus, for the fit, <M, A> are taken from the same tile: M is
@@ -163,8 +164,8 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
   constexpr int NCB = R / 4, NRB = 256 / NCB, TR = 4 * NRB, LD = R + 4;  // padded row stride
   constexpr int TPG = NCB * NCB, NG = 256 / TPG;
   extern __shared__ __align__(16) float sm[];
-  float* Ms = sm;                 // TR x LD
-  float* As = Ms + TR * LD;       // TR x LD
+  float* Mbuf = sm;               // 2 x TR x LD: the M tile being used and the next one in flight
+  float* As = Mbuf + 2 * TR * LD; // TR x LD
   float* Vs = As + TR * LD;       // R x R
   const int tid = threadIdx.x;
   for (int e = tid; e < R * R; e += 256) Vs[e] = Vinv[e];
@@ -175,17 +176,34 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
   for (int q = 0; q < 16; ++q) gacc[q] = 0.0;
   double dacc = 0.0;
   const uint64_t ntiles = (I + TR - 1) / TR;
-  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+  // M tile tb -> buffer b with cp.async (16 B per copy, rows past I zero-filled): the next
+  // tile's copies are in flight while this one is computed
+  auto prefetch = [&](uint64_t tb, int b) {
+    if (tb < ntiles) {
+      const uint64_t r0 = tb * TR;
+      const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
+      const float4* src = reinterpret_cast<const float4*>(M + r0 * R);
+      float* dstb = Mbuf + b * TR * LD;
+      for (int e = tid; e < TR * NCB; e += 256) {
+        const int r = e / NCB, c = e % NCB;
+        const uint32_t d = (uint32_t)__cvta_generic_to_shared(dstb + r * LD + 4 * c);
+        const bool ok = r < rows;
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(ok ? src + e : src),
+                     "r"(ok ? 16 : 0) : "memory");
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int buf = 0;
+  prefetch(blockIdx.x, 0);
+  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, buf ^= 1) {
     const uint64_t r0 = tb * TR;
     const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
-    __syncthreads();  // previous tile's Gram reads of As are done
-    const float4* src = reinterpret_cast<const float4*>(M + r0 * R);
-    for (int e = tid; e < TR * NCB; e += 256) {
-      const int r = e / NCB, c = e % NCB;
-      const float4 v = (r < rows) ? __ldg(src + e) : make_float4(0.f, 0.f, 0.f, 0.f);
-      *reinterpret_cast<float4*>(Ms + r * LD + 4 * c) = v;
-    }
-    __syncthreads();
+    __syncthreads();  // the previous tile's reads of the other buffer and of As are done
+    prefetch(tb + gridDim.x, buf ^ 1);
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
+    __syncthreads();  // every thread's copies of this tile have landed
+    const float* Ms = Mbuf + buf * TR * LD;
     float a[4][4];
 #pragma unroll
     for (int x = 0; x < 4; ++x)
@@ -243,6 +261,7 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
     for (int q = 0; q < 16; ++q) gacc[q] += (double)s4[q];
   }
   // reduce the NG row groups' Gram partials (shared memory reused) and the fit dot
+  asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   double* red = reinterpret_cast<double*>(sm);
   if constexpr (NG > 1) {
@@ -268,7 +287,7 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
 template <int R>
 static size_t update_rt_smem() {
   constexpr int NCB = R / 4, NRB = 256 / NCB, TR = 4 * NRB, LD = R + 4;
-  return (size_t)(2 * TR * LD + R * R) * sizeof(float);
+  return (size_t)(3 * TR * LD + R * R) * sizeof(float);
 }
 
 // Vinv = (Hadamard_{m != n} G_m)^†, one CTA, fp64 Gauss-Jordan on [V | I].

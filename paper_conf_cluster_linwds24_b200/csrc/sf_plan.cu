@@ -761,36 +761,23 @@ __device__ __forceinline__ void rec_store(const uint32_t (&o)[WK], const RecPara
   for (int q = 0; q < WK / 4; ++q) dst[q] = make_uint4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
 }
 
-// Kernel-order records from the AoS copy: rec[k] = record(aos[perm[k]]).  GR records per
-// thread and iteration (GR = 4 measured slower than 1: fewer resident warps).
-constexpr int GR = 1;
+// Kernel-order records from the AoS copy: rec[k] = record(aos[perm[k]]).  (Four independent
+// gathers per thread were measured 10-20 % slower: fewer resident warps.)
 template <int WR, int WK>
 __global__ void gather_rec_kernel(const uint32_t* __restrict__ aos, const uint32_t* __restrict__ perm,
                                   uint64_t n, RecParams rp, uint32_t* __restrict__ rec) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t k0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k0 < n; k0 += GR * stride) {
-    uint32_t w[GR][WR];
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)__ldg(perm + k) * WR);
+    uint32_t w[WR];
 #pragma unroll
-    for (int j = 0; j < GR; ++j) {
-      const uint64_t k = k0 + j * stride;
-      if (k < n) {
-        const uint4* src = reinterpret_cast<const uint4*>(aos + (uint64_t)__ldg(perm + k) * WR);
-#pragma unroll
-        for (int q = 0; q < WR / 4; ++q) {
-          const uint4 v = __ldg(src + q);
-          w[j][4 * q] = v.x; w[j][4 * q + 1] = v.y; w[j][4 * q + 2] = v.z; w[j][4 * q + 3] = v.w;
-        }
-      }
+    for (int q = 0; q < WR / 4; ++q) {
+      const uint4 v = __ldg(src + q);
+      w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
     }
-    uint32_t o[GR][WK];
-#pragma unroll
-    for (int j = 0; j < GR; ++j)
-      if (k0 + j * stride < n) rec_fields<WR, WK>(w[j], rp, o[j]);
-#pragma unroll
-    for (int j = 0; j < GR; ++j) {
-      const uint64_t k = k0 + j * stride;
-      if (k < n) rec_store<WK>(o[j], rp, rec, k);
-    }
+    uint32_t o[WK];
+    rec_fields<WR, WK>(w, rp, o);
+    rec_store<WK>(o, rp, rec, k);
   }
 }
 

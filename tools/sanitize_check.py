@@ -75,6 +75,29 @@ def main():
                 A = [f.clone() for f in tf]
                 fits = T.cp_als(A, iters=2)
                 assert all(np.isfinite(fits))
+    # host inputs: segmented upload with presort, the upload-time AoS copy and row counts of a
+    # >= 2^18-row mode (warp-aggregated atomics), the smem-histogram counts of small modes,
+    # one-pass run statistics, hot-row plans
+    dims, R = (300_000, 50, 400), 16
+    inds, vals = synth.gen_coo(dims, 100_003, 7, zipf=(1.2, 0.7, 0.9), val_kind="signed")
+    facs = synth.gen_factors(dims, R, 8, "signed")
+    tf = [torch.from_numpy(f).cuda() for f in facs]
+    hi = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    hv = torch.from_numpy(vals).pin_memory()
+    with sf.Tensor(dims, hi, hv, segments=5, streams=3) as T:
+        for n in range(3):
+            for L in (None, sf.Launch.make(kernel=FRAG, chunk_nnz=64, block_threads=1024, hot_kb=64)):
+                if L is None:
+                    T.plan(n, R)
+                else:
+                    T.set_launch(n, R, L)
+                y = torch.full((dims[n], R), float("nan"), device="cuda")
+                T.mttkrp(n, tf, y)
+                torch.cuda.synchronize()
+                Y, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
+                rel, zv = oracle.max_rel_err(y.cpu().numpy(), Y, S)
+                assert rel <= 1e-4 and zv == 0, ("host input", n, rel)
+                worst = max(worst, rel)
     print(f"SANITIZE WORKLOAD OK (worst rel err {worst:.2e}, {sf.kernel_launches()} kernels)")
 
 
