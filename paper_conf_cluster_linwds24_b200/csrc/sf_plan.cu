@@ -5,13 +5,15 @@
 // launch parameters based on the sparsity features of the matrixed tensor after
 // chunking."  Here, per (mode n, rank):
 //   1. matricized order: stable LSD radix sort of the key i_n * I_s + i_s with the
-//      input position as payload (s = smallest gathered mode; reading R10);
-//   2. features from run lengths of that order;
+//      input position as payload (s = smallest gathered mode; reading R10), or
+//      the merge of the segment runs sorted during the upload (presort);
+//   2. features from run lengths of that order (run_stats_kernel);
 //   3. shard cut [floor(p*nnz/P), floor((p+1)*nnz/P)) of that order (§8(e));
 //   4. tiles ("tensor blocks ... based on the resource constraints of hardware",
 //      PAPER.md L34): a second stable sort by tile id -> order (tile, i_n, i_s, pos);
-//   5. gather the kernel-order SoA arrays;
-//   6. chunks ("segments"): a new chunk at every tile start and every
+//   5. the hot-row cache: row counts, one global threshold, slots and the index map;
+//   6. gather the kernel-order records from the AoS copy (COO-kernel plans: SoA arrays);
+//   7. chunks ("segments"): a new chunk at every tile start and every
 //      C nonzeros inside a tile.
 // All of it is integer work; tests compare it == against oracle/plan.py.
 #include <cub/cub.cuh>
