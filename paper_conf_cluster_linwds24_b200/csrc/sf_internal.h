@@ -149,6 +149,9 @@ struct Tensor {
   // the mode merges the sorted runs instead of sorting all nonzeros.
   DevBuf pre[SF_MAX_MODES];
   bool have_pre[SF_MAX_MODES] = {};
+  // the last matricized sort of mode m carried the other mode's (i_o >> 17) above bit
+  // carry_kb[m] of its keys (0 = plain keys; sf_plan.cu key_matricized_kernel)
+  int carry_kb[SF_MAX_MODES] = {};
   DevBuf pre_alt;              // composed keys of a segment before its sort (upload only)
   DevBuf hot_cnt[SF_MAX_MODES];  // hot-row cache: nonzeros per row of mode m (whole handle), lazily
   double hot_cover[SF_MAX_MODES] = {-1, -1, -1, -1, -1, -1, -1, -1};  // share of nonzeros in the

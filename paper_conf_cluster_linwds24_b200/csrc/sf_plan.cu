@@ -55,12 +55,19 @@ struct Div64 {
 };
 
 // ---------------------------------------------------------------------------
+// key = i_n * I_s + i_s; with `io`, the bits of (i_o >> kCarryShift) ride above bit kb (the
+// sort covers bits [0, kb) only, so they travel with the key unsorted: tile ids of the other
+// gathered mode without a random gather later, tile_key_from_carry_kernel)
+constexpr int kCarryShift = 17;
 __global__ void key_matricized_kernel(const uint32_t* __restrict__ in, const uint32_t* __restrict__ is,
                                       uint64_t Is, uint64_t n, uint64_t* __restrict__ key,
-                                      uint32_t* __restrict__ pos) {
+                                      uint32_t* __restrict__ pos, const uint32_t* __restrict__ io = nullptr,
+                                      int kb = 0) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
-    key[e] = (uint64_t)in[e] * Is + (uint64_t)is[e];
+    uint64_t k = (uint64_t)in[e] * Is + (uint64_t)is[e];
+    if (io) k |= (uint64_t)(io[e] >> kCarryShift) << kb;
+    key[e] = k;
     pos[e] = (uint32_t)e;
   }
 }
@@ -277,17 +284,28 @@ static void presort_finish(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_ou
 
 // Matricized sort of the whole tensor for `mode`. Returns sorted keys + positions.
 static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_out) {
+  t.carry_kb[mode] = 0;
   if (t.have_pre[mode]) return presort_finish(t, mode, keys_out, pos_out);
   const uint64_t n = t.nnz;
   const int s = secondary_mode(t, mode);
   const uint64_t Is = t.dims[s];
+  const int end_bit = std::max(1, bitlen(t.dims[mode] * Is - 1));
+  // 3-way: carry the other gathered mode's coarse index when it fits above the key bits
+  const uint32_t* io = nullptr;
+  if (t.nmodes == 3) {
+    const int o = 3 - mode - s;
+    const int cb = bitlen((t.dims[o] - 1) >> kCarryShift);
+    if (cb > 0 && end_bit + cb <= 64) {
+      io = t.ind[o].as<uint32_t>();
+      t.carry_kb[mode] = end_bit;
+    }
+  }
   DevBuf k0(n * 8 + 16), k1(n * 8 + 16), p0(n * 4 + 16), p1(n * 4 + 16);
   key_matricized_kernel<<<grid_for(n), 256, 0, t.stream>>>(t.ind[mode].as<uint32_t>(),
                                                          t.ind[s].as<uint32_t>(), Is, n,
-                                                         k0.as<uint64_t>(), p0.as<uint32_t>());
+                                                         k0.as<uint64_t>(), p0.as<uint32_t>(), io, end_bit);
   count_launch();
   SF_CUDA(cudaGetLastError());
-  const int end_bit = std::max(1, bitlen(t.dims[mode] * Is - 1));
   cub::DoubleBuffer<uint64_t> dk(k0.as<uint64_t>(), k1.as<uint64_t>());
   cub::DoubleBuffer<uint32_t> dv(p0.as<uint32_t>(), p1.as<uint32_t>());
   size_t temp = 0;
@@ -302,12 +320,12 @@ static void matricized_sort(Tensor& t, int mode, DevBuf& keys_out, DevBuf& pos_o
 // First j > k with keys[j] >= target, or n (keys sorted ascending, keys[k] < target):
 // galloping from k, then bisection -- O(log(run length)) reads, mostly cached for short runs.
 __device__ __forceinline__ uint64_t run_end(const uint64_t* __restrict__ keys, uint64_t n, uint64_t k,
-                                            uint64_t target) {
+                                            uint64_t target, uint64_t kmask) {
   uint64_t lo = k, hi = n, step = 1;
   while (true) {
     const uint64_t j = lo + step;
     if (j >= n) break;
-    if (__ldg(keys + j) >= target) {
+    if ((__ldg(keys + j) & kmask) >= target) {
       hi = j;
       break;
     }
@@ -316,7 +334,7 @@ __device__ __forceinline__ uint64_t run_end(const uint64_t* __restrict__ keys, u
   }
   while (hi - lo > 1) {
     const uint64_t mid = lo + (hi - lo) / 2;
-    if (__ldg(keys + mid) >= target) hi = mid; else lo = mid;
+    if ((__ldg(keys + mid) & kmask) >= target) hi = mid; else lo = mid;
   }
   return hi;
 }
@@ -329,7 +347,7 @@ __device__ __forceinline__ uint64_t run_end(const uint64_t* __restrict__ keys, u
 // galloping in global memory (run_end).
 constexpr int RS_ITEMS = 8;
 __global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restrict__ keys, uint64_t n, Div64 Is,
-                                                        unsigned long long* __restrict__ runs,
+                                                        uint64_t kmask, unsigned long long* __restrict__ runs,
                                                         FeatAcc* __restrict__ acc) {
   __shared__ unsigned long long h[SF_HIST_BINS];
   for (int i = threadIdx.x; i < SF_HIST_BINS; i += blockDim.x) h[i] = 0;
@@ -354,15 +372,15 @@ __global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restri
 #pragma unroll
       for (int q = 0; q < RS_ITEMS / 2; ++q) {
         const ulonglong2 u = __ldg(v + q);
-        x[2 * q] = u.x;
-        x[2 * q + 1] = u.y;
+        x[2 * q] = u.x & kmask;
+        x[2 * q + 1] = u.y & kmask;
       }
     } else {
 #pragma unroll
-      for (int i = 0; i < RS_ITEMS; ++i) x[i] = (base + i < n) ? __ldg(keys + base + i) : 0;
+      for (int i = 0; i < RS_ITEMS; ++i) x[i] = (base + i < n) ? (__ldg(keys + base + i) & kmask) : 0;
     }
     uint64_t prev = __shfl_up_sync(full, x[RS_ITEMS - 1], 1);
-    if (lane == 0) prev = t0 ? __ldg(keys + t0 - 1) : 0;
+    if (lane == 0) prev = t0 ? (__ldg(keys + t0 - 1) & kmask) : 0;
     // start flags (bit i: item i starts a fiber / a slice; items past n start nothing)
     unsigned fs = 0, ss = 0;
     uint64_t sprev = Is.div(prev);
@@ -398,14 +416,14 @@ __global__ void __launch_bounds__(256) run_stats_kernel(const uint64_t* __restri
     for (int i = RS_ITEMS - 1; i >= 0; --i) {
       const uint64_t k = base + i;
       if (fs >> i & 1) {
-        const uint64_t e = (fnext != NONE) ? fnext : run_end(keys, n, t1 - 1, x[i] + 1);
+        const uint64_t e = (fnext != NONE) ? fnext : run_end(keys, n, t1 - 1, x[i] + 1, kmask);
         const unsigned long long len = e - k;
         ++nf;
         mf = max(mf, len);
         fnext = k;
       }
       if (ss >> i & 1) {
-        const uint64_t e = (snext != NONE) ? snext : run_end(keys, n, t1 - 1, (Is.div(x[i]) + 1) * Is.d);
+        const uint64_t e = (snext != NONE) ? snext : run_end(keys, n, t1 - 1, (Is.div(x[i]) + 1) * Is.d, kmask);
         const unsigned long long len = e - k;
         ++ns;
         ms = max(ms, len);
@@ -465,7 +483,8 @@ static void features_from_sorted(Tensor& t, int mode, const uint64_t* keys, sf_f
     DevBuf accb(sizeof(FeatAcc) + 16);
     unsigned long long* runs = reinterpret_cast<unsigned long long*>(accb.as<char>() + sizeof(FeatAcc));
     SF_CUDA(cudaMemsetAsync(accb.p, 0, sizeof(FeatAcc) + 16, t.stream));
-    run_stats_kernel<<<grid_for((n + RS_ITEMS - 1) / RS_ITEMS), 256, 0, t.stream>>>(keys, n, Div64(Is), runs,
+    const uint64_t kmask = t.carry_kb[mode] ? (1ull << t.carry_kb[mode]) - 1 : ~0ull;
+    run_stats_kernel<<<grid_for((n + RS_ITEMS - 1) / RS_ITEMS), 256, 0, t.stream>>>(keys, n, Div64(Is), kmask, runs,
                                                                                   accb.as<FeatAcc>());
     count_launch();
     SF_CUDA(cudaGetLastError());
@@ -521,12 +540,24 @@ struct TileParams {
 // Single staged mode == the secondary key s: the tile id is (key % I_s) / block_rows, read
 // from the (sequential) matricized keys instead of a random 4-byte gather of i_s.
 __global__ void tile_key_from_keys_kernel(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ pos,
-                                          uint64_t n, Div64 Is, uint32_t block_rows,
+                                          uint64_t n, Div64 Is, uint64_t kmask, uint32_t block_rows,
                                           uint64_t* __restrict__ tkey, uint32_t* __restrict__ tpos) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
-    const uint64_t key = keys[k];
+    const uint64_t key = keys[k] & kmask;
     tkey[k] = (uint32_t)(key - Is.div(key) * Is.d) / block_rows;
+    tpos[k] = pos[k];
+  }
+}
+
+// Single staged mode == the carried other mode o (3-way): tile id = i_o / block_rows =
+// (i_o >> 17) / (block_rows >> 17) for block_rows a multiple of 2^17, from the key's high bits.
+__global__ void tile_key_from_carry_kernel(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ pos,
+                                           uint64_t n, int kb, uint32_t coarse_rows, uint64_t* __restrict__ tkey,
+                                           uint32_t* __restrict__ tpos) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    tkey[k] = (uint32_t)(keys[k] >> kb) / coarse_rows;
     tpos[k] = pos[k];
   }
 }
@@ -872,15 +903,21 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       const size_t nb[2] = {8, 8};
       d2h_small(t.stream, 2, dst, src, nb);
     }
-    p.row_begin = kb / t.dims[s];
-    p.row_end = ke / t.dims[s] + 1;
+    const uint64_t kmask = t.carry_kb[mode] ? (1ull << t.carry_kb[mode]) - 1 : ~0ull;
+    p.row_begin = (kb & kmask) / t.dims[s];
+    p.row_end = (ke & kmask) / t.dims[s] + 1;
   }
   // the caller's out block: whole Y unsharded, the touched rows of a shard
   p.out_row0 = t.nranks > 1 ? p.row_begin : 0;
   p.out_rows = t.nranks > 1 ? p.row_end - p.row_begin : t.dims[mode];
   trace_mark("build: shard range");
   const bool staged_is_secondary = launch.kernel == SF_KERNEL_FRAG && launch.staged_mask == (1u << s);
-  if (!staged_is_secondary) keys.release();  // else kept for the tile keys
+  // tiles of the other mode of a 3-way tensor from the bits its sort carried
+  const int o = N == 3 ? 3 - mode - s : -1;
+  const bool staged_is_carry = launch.kernel == SF_KERNEL_FRAG && o >= 0 && t.carry_kb[mode] &&
+                               launch.staged_mask == (1u << o) &&
+                               launch.block_rows[o] % (1u << kCarryShift) == 0;
+  if (!staged_is_secondary && !staged_is_carry) keys.release();  // else kept for the tile keys
 
   // Kernel order (positions into the raw COO).
   const bool staged = (launch.kernel == SF_KERNEL_FRAG) && launch.staged_mask != 0;
@@ -900,10 +937,15 @@ void build_plan(Tensor& t, Plan& p, int mode, int rank, const sf_launch_t& launc
       tp.staged_mask = launch.staged_mask;
       tp.nmodes = N;
       DevBuf k0(nl * 8 + 16), k1(nl * 8 + 16), p1(nl * 4 + kPadBytes);
+      const uint64_t kmask = t.carry_kb[mode] ? (1ull << t.carry_kb[mode]) - 1 : ~0ull;
       if (staged_is_secondary)
         tile_key_from_keys_kernel<<<grid_for(nl), 256, 0, t.stream>>>(
-            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, Div64(t.dims[s]), launch.block_rows[s],
+            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, Div64(t.dims[s]), kmask, launch.block_rows[s],
             k0.as<uint64_t>(), perm.as<uint32_t>());
+      else if (staged_is_carry)
+        tile_key_from_carry_kernel<<<grid_for(nl), 256, 0, t.stream>>>(
+            keys.as<uint64_t>() + lo, pos0.as<uint32_t>() + lo, nl, t.carry_kb[mode],
+            launch.block_rows[o] >> kCarryShift, k0.as<uint64_t>(), perm.as<uint32_t>());
       else
         tile_key_kernel<<<grid_for(nl), 256, 0, t.stream>>>(tp, pos0.as<uint32_t>() + lo, nl, k0.as<uint64_t>(),
                                                            perm.as<uint32_t>());

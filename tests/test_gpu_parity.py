@@ -320,6 +320,40 @@ def test_presort_upload_bit_exact(cuda_device, segments, streams, monkeypatch):
                 G.assert_parity(y.cpu().numpy(), dims, inds, vals, facs, 16, n)
 
 
+@pytest.mark.parametrize("block_rows", [1 << 17, 3 << 17, 100_000])
+def test_l2_tiles_of_the_other_mode_bit_exact(cuda_device, block_rows):
+    """3-way L2-tiled plans that tile the non-secondary gathered mode o: its coarse index rides
+    above the sort key (tile ids without a random gather) when block_rows is a multiple of
+    2^17, else the gathered tile keys; same order, chunks, features and Y as the oracle."""
+    dims, R = (50_000, 300, 600_000), 16
+    inds, vals = synth.gen_coo(dims, 200_003, 21, zipf=(0.9, 0.6, 1.0), val_kind="int")
+    facs = synth.gen_factors(dims, R, 22, "int")
+    tf = [G.dev_f(f) for f in facs]
+    for host in (False, True):
+        ti = ([torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds] if host else G.dev_inds(inds))
+        tv = torch.from_numpy(vals).pin_memory() if host else G.dev_f(vals)
+        with sf.Tensor(dims, ti, tv) as t:
+            for n in (0, 1):
+                f = t.features(n)
+                of = oplan.features(dims, inds, n)
+                for k in ("num_slices", "num_fibers", "max_nnz_per_slice", "max_nnz_per_fiber",
+                          "sum_sq_nnz_per_slice"):
+                    assert f[k] == of[k], (n, k)
+                assert f["slice_hist"] == list(of["slice_hist"])
+                L = sf.Launch.make(kernel=FRAG, chunk_nnz=64, staged={2: block_rows}, flags=sf.LAUNCH_L2_TILES)
+                t.set_launch(n, R, L)
+                perm, chunks = t.plan_export(n, R)
+                ref = oplan.plan_order(dims, inds, n, (2,), {2: block_rows})
+                assert np.array_equal(perm.astype(np.int64), ref), (host, n, block_rows)
+                tiles = oplan.tile_ids(dims, inds, (2,), {2: block_rows}, sel=ref)
+                assert np.array_equal(chunks.astype(np.int64), oplan.chunks(tiles, 64))
+                y = torch.empty((dims[n], R), device="cuda:0")
+                t.mttkrp(n, tf, y)
+                torch.cuda.synchronize()
+                Y, _ = oracle.mttkrp(dims, inds, vals, facs, R, n)
+                assert np.array_equal(y.cpu().numpy().astype(np.float64), Y), (host, n)
+
+
 @pytest.mark.parametrize("segments", [3, 8])
 def test_presort_wide_keys_bit_exact(cuda_device, segments, monkeypatch):
     """A handle whose modes mix presorted keys and keys that with the input position need more
