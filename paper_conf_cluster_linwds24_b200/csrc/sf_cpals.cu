@@ -64,21 +64,40 @@ __global__ void gram_kernel(const float* __restrict__ A, uint64_t I, int R, doub
 template <int R>
 __global__ void __launch_bounds__(256) gram_rt_kernel(const float* __restrict__ A, uint64_t I,
                                                       double* __restrict__ G) {
-  constexpr int TR = 128, NB = R / 4, TPG = NB * NB, NG = 256 / TPG;
-  __shared__ __align__(16) float tile[TR * R];
-  __shared__ double red[NG > 1 ? NG * 16 * TPG : 1];  // row-group partials (48 KB static at R = 32)
+  constexpr int TR = 4096 / R, NB = R / 4, TPG = NB * NB, NG = 256 / TPG;
+  // two 16 KB tiles (the next one streams in with cp.async while this one is used), then
+  // reused for the row-group partials (NG * 16 * TPG doubles <= 32 KB)
+  __shared__ __align__(16) unsigned char sbuf[2 * TR * R * 4];
+  static_assert(NG * 16 * TPG * 8 <= 2 * TR * R * 4, "partials must fit the tile buffers");
+  float* const tiles = reinterpret_cast<float*>(sbuf);
   const int tid = threadIdx.x, g = tid / TPG, l = tid % TPG, bi = l / NB, bj = l % NB;
   double acc[16];
 #pragma unroll
   for (int q = 0; q < 16; ++q) acc[q] = 0.0;
   const uint64_t ntiles = (I + TR - 1) / TR;
-  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
-    const uint64_t r0 = tb * TR;
-    const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
-    const float4* src = reinterpret_cast<const float4*>(A + r0 * R);
-    float4* dst = reinterpret_cast<float4*>(tile);
-    for (int e = tid; e < TR * R / 4; e += 256) dst[e] = (e < rows * R / 4) ? __ldg(src + e) : make_float4(0, 0, 0, 0);
+  auto prefetch = [&](uint64_t tb, int b) {  // rows past I are zero-filled
+    if (tb < ntiles) {
+      const uint64_t r0 = tb * TR;
+      const int rows = (I - r0 < (uint64_t)TR) ? (int)(I - r0) : TR;
+      const float4* src = reinterpret_cast<const float4*>(A + r0 * R);
+      float* dst = tiles + b * TR * R;
+      for (int e = tid; e < TR * R / 4; e += 256) {
+        const bool ok = e < rows * R / 4;
+        const uint32_t d = (uint32_t)__cvta_generic_to_shared(dst + 4 * e);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(ok ? src + e : src),
+                     "r"(ok ? 16 : 0) : "memory");
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int buf = 0;
+  prefetch(blockIdx.x, 0);
+  for (uint64_t tb = blockIdx.x; tb < ntiles; tb += gridDim.x, buf ^= 1) {
+    __syncthreads();  // everyone is done with the other buffer
+    prefetch(tb + gridDim.x, buf ^ 1);
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncthreads();
+    const float* tile = tiles + buf * TR * R;
     float s[16];
 #pragma unroll
     for (int q = 0; q < 16; ++q) s[q] = 0.f;
@@ -93,8 +112,10 @@ __global__ void __launch_bounds__(256) gram_rt_kernel(const float* __restrict__ 
     }
 #pragma unroll
     for (int q = 0; q < 16; ++q) acc[q] += (double)s[q];
-    __syncthreads();
   }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  double* red = reinterpret_cast<double*>(sbuf);
   if constexpr (NG > 1) {
 #pragma unroll
     for (int q = 0; q < 16; ++q) red[(g * 16 + q) * TPG + l] = acc[q];
@@ -421,7 +442,7 @@ static int grid_of(uint64_t n, int threads) {
 
 static void gram(const float* A, uint64_t I, int R, double* G, cudaStream_t s) {
   SF_CUDA(cudaMemsetAsync(G, 0, sizeof(double) * R * R, s));
-  const int rt_grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((I + 127) / 128, 148ull * 4));
+  const int rt_grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((I + 4096 / R - 1) / (4096 / R), 148ull * 4));
   switch (R) {  // register-tiled kernels; the scalar one for other ranks
     case 16: gram_rt_kernel<16><<<rt_grid, 256, 0, s>>>(A, I, G); break;
     case 32: gram_rt_kernel<32><<<rt_grid, 256, 0, s>>>(A, I, G); break;
