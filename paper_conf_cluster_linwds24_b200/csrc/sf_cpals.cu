@@ -183,7 +183,9 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
                                                            const float* __restrict__ Vinv, float* __restrict__ A,
                                                            double* __restrict__ G, double* __restrict__ dot) {
   constexpr int NCB = R / 4, NRB = 256 / NCB, TR = 4 * NRB, LD = R + 4;  // padded row stride
-  constexpr int TPG = NCB * NCB, NG = 256 / TPG;
+  // Gram: only the upper-triangular 4 x 4 blocks (G is symmetric), one per thread of a row
+  // group; NG row groups split each tile's rows (threads past NG * TPG skip the Gram)
+  constexpr int TPG = NCB * (NCB + 1) / 2, NG = 256 / TPG;
   extern __shared__ __align__(16) float sm[];
   float* Mbuf = sm;               // 2 x TR x LD: the M tile being used and the next one in flight
   float* As = Mbuf + 2 * TR * LD; // TR x LD
@@ -191,7 +193,13 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
   const int tid = threadIdx.x;
   for (int e = tid; e < R * R; e += 256) Vs[e] = Vinv[e];
   const int rs = tid % NRB, cb = tid / NRB;            // A-block: rows rs + NRB*x, cols 4cb..4cb+3
-  const int g = tid / TPG, l = tid % TPG, bi = l / NCB, bj = l % NCB;  // Gram block
+  const int g = tid / TPG, l = tid % TPG;  // Gram block (bi <= bj) number l of row group g
+  int bi = 0, rem = l;
+  while (rem >= NCB - bi) {
+    rem -= NCB - bi;
+    ++bi;
+  }
+  const int bj = bi + rem;
   double gacc[16];
 #pragma unroll
   for (int q = 0; q < 16; ++q) gacc[q] = 0.0;
@@ -269,7 +277,7 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
     float s4[16];
 #pragma unroll
     for (int q = 0; q < 16; ++q) s4[q] = 0.f;
-    for (int rr = g; rr < rows; rr += NG) {
+    for (int rr = g; g < NG && rr < rows; rr += NG) {
       const float4 x4 = *reinterpret_cast<const float4*>(As + rr * LD + 4 * bi);
       const float4 y4 = *reinterpret_cast<const float4*>(As + rr * LD + 4 * bj);
       const float av[4] = {x4.x, x4.y, x4.z, x4.w}, bv[4] = {y4.x, y4.y, y4.z, y4.w};
@@ -285,9 +293,12 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
   asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   double* red = reinterpret_cast<double*>(sm);
+  static_assert((size_t)NG * 16 * TPG * 8 <= (size_t)3 * TR * LD * 4, "Gram partials must fit the tile buffers");
   if constexpr (NG > 1) {
+    if (g < NG) {
 #pragma unroll
-    for (int q = 0; q < 16; ++q) red[(g * 16 + q) * TPG + l] = gacc[q];
+      for (int q = 0; q < 16; ++q) red[(g * 16 + q) * TPG + l] = gacc[q];
+    }
   }
   __syncthreads();
   if (g == 0) {
@@ -296,7 +307,9 @@ __global__ void __launch_bounds__(256, 2) update_rt_kernel(const float* __restri
       double v = gacc[q];
       if constexpr (NG > 1)
         for (int h = 1; h < NG; ++h) v += red[(h * 16 + q) * TPG + l];
-      atomicAdd(&G[(4 * bi + q / 4) * R + 4 * bj + q % 4], v);
+      const int x = q / 4, y = q % 4;
+      atomicAdd(&G[(4 * bi + x) * R + 4 * bj + y], v);
+      if (bi != bj) atomicAdd(&G[(4 * bj + y) * R + 4 * bi + x], v);
     }
   }
   if (dot) {
