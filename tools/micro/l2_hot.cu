@@ -7,6 +7,10 @@
 //   1  hot rows: L2::cache_hint evict_last, cold rows: evict_first
 //   2  hot rows: evict_last, cold rows: plain (evict_normal)
 //   3  hot rows: evict_unchanged... (fraction policy 1.0 evict_last on hot only, cold evict_unchanged)
+//   4  hot rows copied into a dense block (records point into it), plain loads
+//   5  every row renumbered by frequency (no scatter)
+//   6  dense hot block + evict_last on hot rows, evict_first on cold rows
+//   7  dense hot block + evict_last on hot rows, plain cold rows
 // hot = Zipf rank below k_A / k_B with k chosen so the hot rows of both factors take H bytes and
 // have equal expected counts at the cut (the optimal static cache for independent references).
 //
@@ -80,8 +84,10 @@ __global__ void __launch_bounds__(512) gather(const uint4* __restrict__ rec, uin
   uint32_t cur = 0xFFFFFFFFu;
   auto load = [&](const float* base, const float* hbase, uint32_t idx, float4& a, float4& b) {
     const bool hot = idx >> 31;
-    const float* p = (V == 4 && hot ? hbase : base) + (size_t)(idx & 0x7FFFFFFFu) * 32 + 8 * lig;
+    const float* p = ((V == 4 || V >= 6) && hot ? hbase : base) + (size_t)(idx & 0x7FFFFFFFu) * 32 + 8 * lig;
     if (V == 0 || V == 4) ld_na(p, a, b);
+    else if (V == 6) { if (hot) ld_pol(p, a, b, p_last); else ld_pol(p, a, b, p_first); }
+    else if (V == 7) { if (hot) ld_pol(p, a, b, p_last); else ld_na(p, a, b); }
     else if (V == 1) { if (hot) ld_pol(p, a, b, p_last); else ld_pol(p, a, b, p_first); }
     else if (V == 2) { if (hot) ld_pol(p, a, b, p_last); else ld_na(p, a, b); }
     else { if (hot) ld_pol(p, a, b, p_last); else ld_pol(p, a, b, p_unch); }
@@ -143,10 +149,10 @@ int main(int argc, char** argv) {
   for (double HMB : {0.0, 32.0, 64.0, 96.0, 128.0}) {
     const double rows = HMB * 1048576.0 / 128.0;
     const uint32_t kA = (uint32_t)(rows / (1.0 + ratio)), kB = (uint32_t)(rows - kA);
-    for (int V = 0; V < 6; ++V) {
-      if (HMB == 0.0 && V > 0 && V < 5) continue;
+    for (int V = 0; V < 8; ++V) {
+      if (HMB == 0.0 && V > 0 && V != 5) continue;
       if (HMB > 0.0 && V == 5) continue;
-      if (V == 0 || V == 4 || V == 5) {
+      if (V == 0 || V == 4 || V == 5) {  // V 6, 7 reuse V 4's dense-hot records
         gen<<<sms * 8, 256>>>(rec, nnz, IA, IB, s, kA, kB, V == 4 ? 1 : (V == 5 ? 2 : 0));
         CK(cudaDeviceSynchronize());
       }
@@ -157,6 +163,8 @@ int main(int argc, char** argv) {
           case 2: gather<2><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
           case 3: gather<3><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
           case 4: gather<4><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
+          case 6: gather<6><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
+          case 7: gather<7><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
           default: gather<0><<<sms * 2, 512>>>(rec, nnz, A, B, Y, HA, HB); break;
         }
       };
