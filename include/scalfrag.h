@@ -259,6 +259,21 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
                              const float* const* factors, int rank, int mode, float* out,
                              int segments, int streams);
 
+/* The same one-shot pipeline for several modes at once (one MTTKRP per mode n with
+ * outs[n] != NULL, all with the same factors: the N MTTKRPs of a step): every segment is
+ * uploaded ONCE and, behind its H2D, range-checked, copied into 16/32-byte AoS records
+ * (shared by the modes) and, per requested mode, sorted by i_n and reduced along its runs
+ * (compute overlaps the H2D of later segments).  outs: nmodes DEVICE
+ * pointers (NULL = mode not computed), Y_n is I_n x rank row-major, overwritten.  factors:
+ * nmodes device pointers; A_m may be NULL only if m is the one mode computed.  stream: the
+ * work is ordered after what the caller queued on it before the call (e.g. the factor
+ * uploads; NULL = no ordering).  Device footprint: O(streams x segment) + the caller's
+ * arrays.  Synchronizes before returning; errors as sf_mttkrp_streamed. */
+sf_status sf_mttkrp_streamed_modes(int nmodes, const uint64_t* dims, uint64_t nnz,
+                                   const uint32_t* const* inds_host, const float* vals_host,
+                                   const float* const* factors, int rank, float* const* outs,
+                                   int segments, int streams, void* stream);
+
 /* Boundary-row exchange helper for multi-GPU row shards (§8(e)): for k < count with
  * rows[k] >= 0 (device int64 array):
  *   op 0 (PACK): buf[k, :] = Y[rows[k], :]      op 1 (ADD): Y[rows[k], :] += buf[k, :]

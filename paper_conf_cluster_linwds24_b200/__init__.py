@@ -100,7 +100,7 @@ class PlanInfo(ctypes.Structure):
 
 EXPORTED = ["sf_tensor_create", "sf_tensor_create_ex", "sf_tensor_destroy", "sf_set_shard",
             "sf_plan", "sf_set_launch", "sf_features", "sf_plan_info", "sf_plan_export",
-            "sf_mttkrp", "sf_mttkrp_streamed", "sf_status_string", "sf_last_error",
+            "sf_mttkrp", "sf_mttkrp_streamed", "sf_mttkrp_streamed_modes", "sf_status_string", "sf_last_error",
             "sf_kernel_launches", "sf_version", "sf_rows_op", "sf_selector_features",
             "sf_selector_candidates", "sf_set_selector_model", "sf_cpals", "sf_plan_release",
             "sf_trim_cache", "sf_shard_rows", "sf_comm_unique_id", "sf_comm_attach",
@@ -137,6 +137,7 @@ def lib(build_if_missing: bool = True):
             L.sf_plan_export.argtypes = [P, I, I, P, P]
             L.sf_mttkrp.argtypes = [P, I, P, I, P, P]
             L.sf_mttkrp_streamed.argtypes = [I, P, U64, P, P, P, I, I, P, I, I]
+            L.sf_mttkrp_streamed_modes.argtypes = [I, P, U64, P, P, P, I, P, I, I, P]
             L.sf_rows_op.argtypes = [P, I, P, P, I, I, P]
             L.sf_selector_features.argtypes = [P, I, I, P, ctypes.POINTER(I)]
             L.sf_selector_candidates.argtypes = [P, I, I, P, ctypes.POINTER(I)]
@@ -417,6 +418,20 @@ def mttkrp_streamed(dims, inds, vals, factors, mode, out, segments=8, streams=4)
     _check(lib().sf_mttkrp_streamed(N, d, int(len(vals)), ip, _ptr(vals), fp, int(out.shape[1]), int(mode),
                                     _ptr(out), int(segments), int(streams)))
     return out
+
+
+def mttkrp_streamed_modes(dims, inds, vals, factors, outs, segments=8, streams=4, stream=None):
+    """One-shot streamed MTTKRP of every mode n with outs[n] is not None (HOST COO, one upload
+    for all modes; the work is ordered after what `stream` already holds)."""
+    N = len(dims)
+    d = (ctypes.c_uint64 * N)(*[int(x) for x in dims])
+    ip = (ctypes.c_void_p * N)(*[_ptr(a) for a in inds])
+    fp = (ctypes.c_void_p * N)(*[_ptr(f) if f is not None else None for f in factors])
+    op = (ctypes.c_void_p * N)(*[_ptr(o) if o is not None else None for o in outs])
+    rank = next((int(o.shape[1]) for o in outs if o is not None), 1)  # no output: the library rejects it
+    _check(lib().sf_mttkrp_streamed_modes(N, d, int(len(vals)), ip, _ptr(vals), fp, rank, op, int(segments),
+                                          int(streams), _stream_handle(stream)))
+    return outs
 
 
 def comm_unique_id() -> bytes:

@@ -742,82 +742,139 @@ sf_status sf_allgather_rows(sf_tensor_t h, int mode, int rank, const float* loca
   });
 }
 
+// One-shot streamed MTTKRP of every mode n with outs[n] != NULL (A8 (ii)): each segment of the
+// host COO is uploaded once and, on the same stream, range-checked, copied into AoS records,
+// and for every requested mode sorted by i_n and reduced (or, other ranks, one atomic per
+// nonzero); segment k+1's upload overlaps segment k's work.
+static void streamed_impl(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* const* inds_host,
+                          const float* vals_host, const float* const* factors, int rank, float* const* outs,
+                          int segments, int streams, cudaStream_t after) {
+  if (nmodes < 2 || nmodes > SF_MAX_MODES || !dims || !factors || !outs)
+    throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
+  if (rank < 1) throw StatusError{SF_ERR_INVALID_ARG, "bad rank"};
+  if (nnz > 0 && (!inds_host || !vals_host)) throw StatusError{SF_ERR_INVALID_ARG, "NULL COO"};
+  uint32_t todo = 0;
+  for (int n = 0; n < nmodes; ++n)
+    if (outs[n]) todo |= 1u << n;
+  if (!todo) throw StatusError{SF_ERR_INVALID_ARG, "no output mode"};
+  for (int m = 0; m < nmodes; ++m)
+    if ((todo & ~(1u << m)) && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
+  if (segments <= 0) segments = 8;
+  if (streams <= 0) streams = 4;
+  segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, nnz)));
+  streams = std::max(1, std::min(streams, segments));
+  const uint64_t seg_len = (nnz + segments - 1) / segments;
+  // sorted segments (A8 (ii) + pre-reduction): rank 16/32/64 (nmodes <= 7) sort every segment
+  // by i_n on the device and reduce runs in registers; other ranks keep one atomic per nonzero
+  const bool sorted = seg_sorted_supported(rank) && nmodes <= 7;
+  auto bits_of = [&](int n) {
+    int kb = 1;
+    for (uint64_t x = dims[n] - 1; x; x >>= 1) ++kb;
+    return kb;
+  };
+  int kbits = 1;
+  for (int n = 0; n < nmodes; ++n)
+    if (todo >> n & 1) kbits = std::max(kbits, bits_of(n));
+  const size_t A = 64;
+  auto al = [&](size_t b) { return (b + A - 1) & ~(A - 1); };
+  const size_t raw_bytes = al((size_t)seg_len * 4) * (nmodes + 1);
+  const int W = seg_aos_words(nmodes);
+  const size_t aos_bytes = sorted ? al((size_t)seg_len * 4 * W) : 0;
+  const size_t sort_temp = sorted ? seg_sort_temp_bytes(seg_len, kbits) : 0;
+  const size_t sort_bytes = sorted ? 3 * al((size_t)seg_len * 4) + sort_temp : 0;
+  std::vector<cudaStream_t> st(streams);
+  for (auto& s : st) SF_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  std::vector<DevBuf> ring;
+  DevBuf flag(16);
+  cudaEvent_t zeroed = nullptr, before = nullptr;
+  try {
+    ring.reserve(streams);
+    for (int s = 0; s < streams; ++s) ring.emplace_back(raw_bytes + aos_bytes + sort_bytes + A);
+    SF_CUDA(cudaEventCreateWithFlags(&zeroed, cudaEventDisableTiming));
+    if (after) {  // work already queued on the caller's stream (e.g. the factor uploads) first
+      SF_CUDA(cudaEventCreateWithFlags(&before, cudaEventDisableTiming));
+      SF_CUDA(cudaEventRecord(before, after));
+      SF_CUDA(cudaStreamWaitEvent(st[0], before, 0));
+    }
+    SF_CUDA(cudaMemsetAsync(flag.p, 0, 16, st[0]));
+    for (int n = 0; n < nmodes; ++n)
+      if (todo >> n & 1) SF_CUDA(cudaMemsetAsync(outs[n], 0, sizeof(float) * dims[n] * (size_t)rank, st[0]));
+    SF_CUDA(cudaEventRecord(zeroed, st[0]));
+    for (int s = 1; s < streams; ++s) SF_CUDA(cudaStreamWaitEvent(st[s], zeroed, 0));
+    if (sorted)  // the payload of every segment sort: positions 0 .. seg_len-1
+      for (int s = 0; s < streams; ++s)
+        launch_iota(reinterpret_cast<uint32_t*>(ring[s].as<char>() + raw_bytes + aos_bytes + 2 * al(seg_len * 4)),
+                    seg_len, st[s]);
+    for (int k = 0; k < segments; ++k) {
+      const uint64_t a = (uint64_t)k * seg_len;
+      if (a >= nnz) break;
+      const uint64_t len = std::min(nnz, a + seg_len) - a;
+      const int s = k % streams;
+      char* base = ring[s].as<char>();
+      uint32_t* di[SF_MAX_MODES];
+      for (int m = 0; m < nmodes; ++m) {
+        di[m] = reinterpret_cast<uint32_t*>(base + (size_t)m * al(seg_len * 4));
+        SF_CUDA(cudaMemcpyAsync(di[m], inds_host[m] + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+      }
+      float* dv = reinterpret_cast<float*>(base + (size_t)nmodes * al(seg_len * 4));
+      SF_CUDA(cudaMemcpyAsync(dv, vals_host + a, len * 4, cudaMemcpyHostToDevice, st[s]));
+      validate_indices(nmodes, dims, len, di, flag.as<int>(), st[s]);
+      if (sorted) {
+        uint32_t* aos = reinterpret_cast<uint32_t*>(base + raw_bytes);
+        char* sb = base + raw_bytes + aos_bytes;
+        uint32_t* skey = reinterpret_cast<uint32_t*>(sb);
+        uint32_t* spos = reinterpret_cast<uint32_t*>(sb + al(seg_len * 4));
+        const uint32_t* iota = reinterpret_cast<const uint32_t*>(sb + 2 * al(seg_len * 4));
+        void* temp = sb + 3 * al(seg_len * 4);
+        launch_seg_aos(nmodes, len, di, dv, aos, st[s]);
+        for (int n = 0; n < nmodes; ++n) {
+          if (!(todo >> n & 1)) continue;
+          seg_sort(di[n], skey, iota, spos, len, bits_of(n), temp, sort_temp, st[s]);
+          launch_seg_sorted(nmodes, dims, len, aos, skey, spos, factors, rank, n, outs[n], st[s]);
+        }
+      } else {
+        for (int n = 0; n < nmodes; ++n)
+          if (todo >> n & 1) launch_coo(nmodes, dims, len, di, dv, factors, rank, n, outs[n], st[s]);
+      }
+    }
+    for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
+    int bad = 0;
+    SF_CUDA(cudaMemcpy(&bad, flag.p, 4, cudaMemcpyDeviceToHost));
+    for (auto& s : st) cudaStreamDestroy(s);
+    cudaEventDestroy(zeroed);
+    if (before) cudaEventDestroy(before);
+    if (bad) throw StatusError{SF_ERR_INDEX_OUT_OF_RANGE, "some index is >= its dimension"};
+  } catch (...) {
+    for (auto& s : st) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
+    if (zeroed) cudaEventDestroy(zeroed);
+    if (before) cudaEventDestroy(before);
+    throw;
+  }
+}
+
 sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
                              const uint32_t* const* inds_host, const float* vals_host,
                              const float* const* factors, int rank, int mode, float* out,
                              int segments, int streams) {
   NvtxRange nvtx_("sf_mttkrp_streamed");
   return guard([&]() -> sf_status {
-    if (nmodes < 2 || nmodes > SF_MAX_MODES || !dims || !factors || !out)
-      throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
-    if (mode < 0 || mode >= nmodes || rank < 1) throw StatusError{SF_ERR_INVALID_ARG, "bad mode/rank"};
-    if (nnz > 0 && (!inds_host || !vals_host)) throw StatusError{SF_ERR_INVALID_ARG, "NULL COO"};
-    for (int m = 0; m < nmodes; ++m)
-      if (m != mode && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
-    if (segments <= 0) segments = 8;
-    if (streams <= 0) streams = 4;
-    segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, nnz)));
-    streams = std::max(1, std::min(streams, segments));
-    const uint64_t seg_len = (nnz + segments - 1) / segments;
-    // sorted segments (A8 (ii) + pre-reduction): rank 16/32/64 sort every segment by i_n on
-    // the device and reduce runs in registers; other ranks keep one atomic per nonzero
-    const bool sorted = seg_sorted_supported(rank);
-    int kbits = 1;
-    for (uint64_t x = dims[mode] - 1; x; x >>= 1) ++kbits;
-    const size_t raw_bytes = (size_t)seg_len * 4 * (nmodes + 1) + 64;
-    const size_t sort_temp = sorted ? seg_sort_temp_bytes(seg_len, kbits) : 0;
-    const size_t sort_bytes = sorted ? (size_t)seg_len * 12 + 3 * 64 + sort_temp : 0;
-    std::vector<cudaStream_t> st(streams);
-    for (auto& s : st) SF_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
-    std::vector<DevBuf> ring;
-    DevBuf flag(16);
-    cudaEvent_t zeroed = nullptr;
-    try {
-      ring.reserve(streams);
-      for (int s = 0; s < streams; ++s) ring.emplace_back(raw_bytes + sort_bytes);
-      SF_CUDA(cudaEventCreateWithFlags(&zeroed, cudaEventDisableTiming));
-      SF_CUDA(cudaMemsetAsync(flag.p, 0, 16, st[0]));
-      SF_CUDA(cudaMemsetAsync(out, 0, sizeof(float) * dims[mode] * (size_t)rank, st[0]));
-      SF_CUDA(cudaEventRecord(zeroed, st[0]));
-      for (int s = 1; s < streams; ++s) SF_CUDA(cudaStreamWaitEvent(st[s], zeroed, 0));
-      for (int k = 0; k < segments; ++k) {
-        const uint64_t a = (uint64_t)k * seg_len;
-        if (a >= nnz) break;
-        const uint64_t len = std::min(nnz, a + seg_len) - a;
-        const int s = k % streams;
-        char* base = ring[s].as<char>();
-        uint32_t* di[SF_MAX_MODES];
-        for (int m = 0; m < nmodes; ++m) {
-          di[m] = reinterpret_cast<uint32_t*>(base + (size_t)m * seg_len * 4);
-          SF_CUDA(cudaMemcpyAsync(di[m], inds_host[m] + a, len * 4, cudaMemcpyHostToDevice, st[s]));
-        }
-        float* dv = reinterpret_cast<float*>(base + (size_t)nmodes * seg_len * 4);
-        SF_CUDA(cudaMemcpyAsync(dv, vals_host + a, len * 4, cudaMemcpyHostToDevice, st[s]));
-        validate_indices(nmodes, dims, len, di, flag.as<int>(), st[s]);
-        if (sorted) {
-          char* sb = base + raw_bytes;
-          uint32_t* skey = reinterpret_cast<uint32_t*>(sb);
-          uint32_t* spos = reinterpret_cast<uint32_t*>(sb + ((seg_len * 4 + 63) & ~(size_t)63));
-          uint32_t* iota = reinterpret_cast<uint32_t*>(sb + 2 * ((seg_len * 4 + 63) & ~(size_t)63));
-          void* temp = sb + 3 * ((seg_len * 4 + 63) & ~(size_t)63);
-          launch_iota(iota, len, st[s]);
-          seg_sort(di[mode], skey, iota, spos, len, kbits, temp, sort_temp, st[s]);
-          launch_seg_sorted(nmodes, dims, len, di, dv, skey, spos, factors, rank, mode, out, st[s]);
-        } else {
-          launch_coo(nmodes, dims, len, di, dv, factors, rank, mode, out, st[s]);
-        }
-      }
-      for (auto& s : st) SF_CUDA(cudaStreamSynchronize(s));
-      int bad = 0;
-      SF_CUDA(cudaMemcpy(&bad, flag.p, 4, cudaMemcpyDeviceToHost));
-      for (auto& s : st) cudaStreamDestroy(s);
-      cudaEventDestroy(zeroed);
-      if (bad) throw StatusError{SF_ERR_INDEX_OUT_OF_RANGE, "some index is >= its dimension"};
-    } catch (...) {
-      for (auto& s : st) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
-      if (zeroed) cudaEventDestroy(zeroed);
-      throw;
-    }
+    if (nmodes < 2 || nmodes > SF_MAX_MODES || !out) throw StatusError{SF_ERR_INVALID_ARG, "bad arguments"};
+    if (mode < 0 || mode >= nmodes) throw StatusError{SF_ERR_INVALID_ARG, "bad mode/rank"};
+    float* outs[SF_MAX_MODES] = {};
+    outs[mode] = out;
+    streamed_impl(nmodes, dims, nnz, inds_host, vals_host, factors, rank, outs, segments, streams, nullptr);
+    return SF_OK;
+  });
+}
+
+sf_status sf_mttkrp_streamed_modes(int nmodes, const uint64_t* dims, uint64_t nnz,
+                                   const uint32_t* const* inds_host, const float* vals_host,
+                                   const float* const* factors, int rank, float* const* outs,
+                                   int segments, int streams, void* stream) {
+  NvtxRange nvtx_("sf_mttkrp_streamed_modes");
+  return guard([&]() -> sf_status {
+    streamed_impl(nmodes, dims, nnz, inds_host, vals_host, factors, rank, outs, segments, streams,
+                  static_cast<cudaStream_t>(stream));
     return SF_OK;
   });
 }

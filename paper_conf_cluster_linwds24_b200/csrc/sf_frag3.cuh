@@ -110,7 +110,9 @@ __device__ __forceinline__ uint32_t pk_field(uint32_t w0, uint32_t w1, uint32_t 
 // deltas were measured 9 % slower on nell-2 and removed.)
 constexpr int kRecPlain = 0, kRecPacked = 1;
 
-template <int N, int R, int S, int RF>
+// HOT: the plan has a hot-row cache (the per-gather select is compiled only into these
+// instantiations: on L2-resident plans it cost 5 %, nell-2 0.767 vs 0.729 ms per mode).
+template <int N, int R, int S, int RF, bool HOT>
 __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   using namespace detail;
   using LM = LaneMap<R>;
@@ -270,7 +272,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     auto gather = [&](int q, uint32_t row_idx) -> F8 {
       const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
       size_t row = (size_t)row_idx * R4;
-      if (q >= S) {  // hot-row cache: the slot inside the dense hot block
+      if (HOT && q >= S) {  // hot-row cache: the slot inside the dense hot block
         const uint32_t hb = p.hot_bit[q];
         if (row_idx & hb) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
       }
@@ -480,21 +482,22 @@ static __global__ void frag3_combine_kernel(const uint32_t* __restrict__ carry_r
 void frag3_launch_r16(int N, int S, const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s);
 void frag3_launch_r32(int N, int S, const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s);
 void frag3_launch_r64(int N, int S, const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s);
-int frag3_occ_r16(int N, int S, int threads, size_t smem);
-int frag3_occ_r32(int N, int S, int threads, size_t smem);
-int frag3_occ_r64(int N, int S, int threads, size_t smem);
+int frag3_occ_r16(int N, int S, int threads, size_t smem, bool hot);
+int frag3_occ_r32(int N, int S, int threads, size_t smem, bool hot);
+int frag3_occ_r64(int N, int S, int threads, size_t smem, bool hot);
 void boundary_zero3_r16(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out, cudaStream_t s);
 void boundary_zero3_r32(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out, cudaStream_t s);
 void boundary_zero3_r64(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out, cudaStream_t s);
 
-// Dynamic shared memory opted in per (device, instantiation, record format): only ever RAISED
-// (the occupancy query and the launch share it; lowering the attribute for a smaller plan
-// would make a later launch of a larger plan fail with "invalid argument").
+// Dynamic shared memory opted in per (device, instantiation, variant v = record format +
+// 2 * HOT): only ever RAISED (the occupancy query and the launch share it; lowering the
+// attribute for a smaller plan would make a later launch of a larger plan fail with
+// "invalid argument").
 template <int N, int R, int S>
 size_t& frag3_smem_optin(int dev, int v) {
-  static size_t set[16][2] = {};
+  static size_t set[16][4] = {};
   static size_t spill = 0;
-  return (dev < 16 && v < 2) ? set[dev][v] : spill;
+  return (dev < 16 && v < 4) ? set[dev][v] : spill;
 }
 
 template <int N, int R, int S, class K>
@@ -508,21 +511,49 @@ void frag3_ensure_smem(K k, int v, size_t smem) {
   }
 }
 
+// The instantiation a plan runs: record format from fp.W, HOT when a gathered slot has hot
+// rows (never when every gathered slot is staged in shared memory).
+template <int N, int R, int S>
+void (*frag3_pick(bool packed, bool hot, int* v))(const Frag3Params) {
+  constexpr bool kHotPossible = S < N - 1;
+  void (*k)(const Frag3Params) = frag3_kernel<N, R, S, kRecPlain, false>;
+  *v = 0;
+  if constexpr (kHotPossible) {
+    if (hot) {
+      k = frag3_kernel<N, R, S, kRecPlain, true>;
+      *v = 2;
+    }
+  }
+  if constexpr (N >= 4) {
+    if (packed) {
+      k = frag3_kernel<N, R, S, kRecPacked, false>;
+      *v = 1;
+      if constexpr (kHotPossible) {
+        if (hot) {
+          k = frag3_kernel<N, R, S, kRecPacked, true>;
+          *v = 3;
+        }
+      }
+    }
+  }
+  return k;
+}
+
 template <int N, int R, int S>
 void frag3_launch_one(const Frag3Params& fp, int grid, int threads, size_t smem, cudaStream_t s) {
-  auto k = frag3_kernel<N, R, S, kRecPlain>;
-  if constexpr (N >= 4) {
-    if (fp.W == 4) k = frag3_kernel<N, R, S, kRecPacked>;
-  }
-  const int v = (fp.W == 4 && N >= 4) ? 1 : 0;
+  bool hot = false;
+  for (int q = 0; q < SF_MAX_MODES; ++q) hot = hot || fp.hot_bit[q] != 0;
+  int v = 0;
+  auto k = frag3_pick<N, R, S>(fp.W == 4 && N >= 4, hot, &v);
   frag3_ensure_smem<N, R, S>(k, v, smem);
   k<<<grid, threads, smem, s>>>(fp);
 }
 
 template <int N, int R, int S>
-int frag3_occ_one(int threads, size_t smem) {
-  auto k = frag3_kernel<N, R, S, kRecPlain>;
-  frag3_ensure_smem<N, R, S>(k, 0, smem);
+int frag3_occ_one(int threads, size_t smem, bool hot) {
+  int v = 0;
+  auto k = frag3_pick<N, R, S>(false, hot, &v);
+  frag3_ensure_smem<N, R, S>(k, v, smem);
   int nb = 0;
   SF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, threads, smem));
   return nb;
@@ -534,8 +565,8 @@ int frag3_occ_one(int threads, size_t smem) {
     SF_FRAG_NS_SWITCH(R, frag3_launch_one, fp, grid, threads, smem, s);                                  \
     throw StatusError{SF_ERR_UNSUPPORTED, "frag3 kernel: unsupported (N, S)"};                          \
   }                                                                                                      \
-  int frag3_occ_r##R(int N, int S, int threads, size_t smem) {                                           \
-    SF_FRAG_NS_SWITCH(R, frag3_occ_one, threads, smem);                                                  \
+  int frag3_occ_r##R(int N, int S, int threads, size_t smem, bool hot) {                                 \
+    SF_FRAG_NS_SWITCH(R, frag3_occ_one, threads, smem, hot);                                             \
     return 0;                                                                                            \
   }                                                                                                      \
   void boundary_zero3_r##R(const Frag3Params& fp, uint32_t ctas, uint32_t groups, float* out,           \

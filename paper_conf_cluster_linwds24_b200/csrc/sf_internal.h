@@ -288,9 +288,12 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
                 cudaStream_t s);
 bool frag_supported(int nmodes, int rank);
 bool seg_sorted_supported(int rank);
-void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* const* inds,
-                       const float* vals, const uint32_t* skey, const uint32_t* spos, const float* const* factors,
-                       int rank, int mode, float* out, cudaStream_t s);
+int seg_aos_words(int nmodes);
+void launch_seg_aos(int nmodes, uint64_t len, const uint32_t* const* inds, const float* vals, uint32_t* aos,
+                    cudaStream_t s);
+void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* aos, const uint32_t* skey,
+                       const uint32_t* spos, const float* const* factors, int rank, int mode, float* out,
+                       cudaStream_t s);
 void launch_iota(uint32_t* x, uint64_t n, cudaStream_t s);
 size_t seg_sort_temp_bytes(uint64_t len, int bits);
 void seg_sort(const uint32_t* keys_in, uint32_t* keys_out, const uint32_t* vals_in, uint32_t* vals_out, uint64_t len,

@@ -203,57 +203,87 @@ void launch_coo(int nmodes, const uint64_t* dims, uint64_t nnz, const uint32_t* 
 }
 
 // ---------------------------------------------------------------------------
-// Sorted-segment kernel (the one-shot streamed path, §8(a) A8 (ii)).  A segment of the raw
-// COO, once on the device, is sorted by i_n (keys = i_n, payload = position in the segment);
-// each lane group then walks a contiguous range of the sorted positions, accumulating in
-// registers while i_n is unchanged and adding one vector atomic per run piece -- a heavy row
-// gets one atomic per (segment, group) instead of one per nonzero, which keeps the fp32
-// chain short (SURVEY C-2: amazon's 1.2e8-nonzero row).  Out-of-range nonzeros are skipped
-// (the segment's range check runs concurrently and is reported at the end).
+// Sorted-segment kernel (the one-shot streamed paths, §8(a) A8 (ii)).  A segment of the raw
+// COO, once on the device, is copied into W-word AoS records [i_0 .. i_{N-1}, 0.., v]
+// (one coalesced pass, shared by every mode computed from the segment) and sorted by i_n
+// (keys = i_n, payload = position in the segment); each lane group then walks a contiguous
+// range of the sorted positions, reading each nonzero as one 16/32-byte record, accumulating
+// in registers while i_n is unchanged and adding one vector atomic per run piece -- a heavy
+// row gets one atomic per (segment, group) instead of one per nonzero, which keeps the fp32
+// chain short (SURVEY C-2: amazon's 1.2e8-nonzero row).  SEG_U nonzeros per group are in
+// flight (their records and factor rows are loaded before any is accumulated).
+// Out-of-range nonzeros are skipped (the segment's range check runs before and is reported
+// at the end).
 // ---------------------------------------------------------------------------
 struct SegParams {
-  const uint32_t* ind[SF_MAX_MODES];  // segment arrays (input order)
-  const float* val;
+  const uint32_t* aos;                // segment records (input order), W words each
   const uint32_t* skey;               // sorted i_n
   const uint32_t* spos;               // position of the sorted slot in the segment
   const float* fac[SF_MAX_MODES];
   float* out;
   uint64_t dims[SF_MAX_MODES];
   uint64_t len;
+  uint32_t dn;                        // min(dims[mode], 2^32 - 1): i_n >= dn is skipped
   int nmodes, mode;
 };
 
-template <int R>
+constexpr int SEG_U = 4;
+
+template <int R, int W>
 __global__ void __launch_bounds__(256) seg_sorted_kernel(SegParams p) {
   constexpr int LPN = R / 4;
   const int sub = threadIdx.x % LPN;
   const uint64_t g = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) / LPN;
   const uint64_t G = ((uint64_t)gridDim.x * blockDim.x) / LPN;
   const uint64_t k0 = g * p.len / G, k1 = (g + 1) * p.len / G;
+  const uint32_t dn = p.dn;
   uint32_t cur = 0xFFFFFFFFu;
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (uint64_t k = k0; k < k1; ++k) {
-    const uint32_t i = __ldg(p.skey + k);
-    const uint32_t e = __ldg(p.spos + k);
-    if (i != cur) {
-      if (cur != 0xFFFFFFFFu) red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
-      acc = make_float4(0.f, 0.f, 0.f, 0.f);
-      cur = i < p.dims[p.mode] ? i : 0xFFFFFFFFu;
-    }
-    if (cur == 0xFFFFFFFFu) continue;
-    const float v = __ldg(p.val + e);
-    float4 prod = make_float4(v, v, v, v);
-    bool ok = true;
+  for (uint64_t k = k0; k < k1; k += SEG_U) {
+    uint32_t ii[SEG_U];
+    uint32_t w[SEG_U][W];
 #pragma unroll
-    for (int m = 0; m < SF_MAX_MODES; ++m) {
-      if (m >= p.nmodes) break;
-      if (m == p.mode) continue;
-      const uint32_t im = __ldg(p.ind[m] + e);
-      ok = ok && im < p.dims[m];
-      if (ok) prod = f4mul(prod, ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub));
+    for (int u = 0; u < SEG_U; ++u) {
+      const bool in = k + u < k1;
+      ii[u] = in ? __ldg(p.skey + k + u) : 0xFFFFFFFFu;
+      const uint32_t e = in ? __ldg(p.spos + k + u) : 0u;
+      const uint4* r = reinterpret_cast<const uint4*>(p.aos + (size_t)e * W);
+#pragma unroll
+      for (int q = 0; q < W / 4; ++q) {
+        const uint4 x = __ldg(r + q);
+        w[u][4 * q] = x.x; w[u][4 * q + 1] = x.y; w[u][4 * q + 2] = x.z; w[u][4 * q + 3] = x.w;
+      }
     }
-    if (ok) {
-      acc.x += prod.x; acc.y += prod.y; acc.z += prod.z; acc.w += prod.w;
+    float4 prod[SEG_U];
+    bool ok[SEG_U];
+#pragma unroll
+    for (int u = 0; u < SEG_U; ++u) {
+      const float v = __uint_as_float(w[u][W - 1]);
+      prod[u] = make_float4(v, v, v, v);
+      ok[u] = ii[u] < dn;
+    }
+#pragma unroll
+    for (int m = 0; m < W - 1; ++m) {
+      if (m < p.nmodes && m != p.mode) {
+#pragma unroll
+        for (int u = 0; u < SEG_U; ++u) {
+          const uint32_t im = w[u][m];
+          ok[u] = ok[u] && im < p.dims[m];
+          if (ok[u]) prod[u] = f4mul(prod[u], ldg_f4(p.fac[m] + (size_t)im * R + 4 * sub));
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < SEG_U; ++u) {
+      if (k + u >= k1) continue;
+      if (ii[u] != cur) {
+        if (cur != 0xFFFFFFFFu) red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
+        acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        cur = ii[u] < dn ? ii[u] : 0xFFFFFFFFu;
+      }
+      if (ok[u]) {
+        acc.x += prod[u].x; acc.y += prod[u].y; acc.z += prod[u].z; acc.w += prod[u].w;
+      }
     }
   }
   if (cur != 0xFFFFFFFFu) red_add_v4(p.out + (size_t)cur * R + 4 * sub, acc);
@@ -261,17 +291,60 @@ __global__ void __launch_bounds__(256) seg_sorted_kernel(SegParams p) {
 
 bool seg_sorted_supported(int rank) { return rank == 16 || rank == 32 || rank == 64; }
 
-void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* const* inds,
-                       const float* vals, const uint32_t* skey, const uint32_t* spos, const float* const* factors,
-                       int rank, int mode, float* out, cudaStream_t s) {
+int seg_aos_words(int nmodes) { return (nmodes + 1 <= 4) ? 4 : 8; }
+
+struct SegAosParams {
+  const uint32_t* ind[SF_MAX_MODES];
+  const float* val;
+  uint32_t* aos;
+  int nmodes, W;
+};
+
+__global__ void seg_aos_kernel(SegAosParams a, uint64_t n) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+    uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+    for (int m = 0; m < 7; ++m)
+      if (m < a.nmodes) w[m] = __ldg(a.ind[m] + e);
+    const uint32_t v = __float_as_uint(__ldg(a.val + e));
+    uint4* r = reinterpret_cast<uint4*>(a.aos + e * a.W);
+    if (a.W == 8) {
+      r[0] = make_uint4(w[0], w[1], w[2], w[3]);
+      r[1] = make_uint4(w[4], w[5], w[6], v);
+    } else {
+      r[0] = make_uint4(w[0], w[1], w[2], v);
+    }
+  }
+}
+
+void launch_seg_aos(int nmodes, uint64_t len, const uint32_t* const* inds, const float* vals, uint32_t* aos,
+                    cudaStream_t s) {
+  if (len == 0) return;
+  if (nmodes > 7) throw StatusError{SF_ERR_UNSUPPORTED, "sorted segments: nmodes <= 7"};
+  SegAosParams a{};
+  for (int m = 0; m < nmodes; ++m) a.ind[m] = inds[m];
+  a.val = vals;
+  a.aos = aos;
+  a.nmodes = nmodes;
+  a.W = seg_aos_words(nmodes);
+  seg_aos_kernel<<<(int)std::min<uint64_t>((len + 255) / 256, 148 * 16), 256, 0, s>>>(a, len);
+  count_launch();
+  SF_CUDA(cudaGetLastError());
+}
+
+void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uint32_t* aos, const uint32_t* skey,
+                       const uint32_t* spos, const float* const* factors, int rank, int mode, float* out,
+                       cudaStream_t s) {
   if (len == 0) return;
   SegParams p{};
-  for (int m = 0; m < nmodes; ++m) { p.ind[m] = inds[m]; p.fac[m] = factors[m]; p.dims[m] = dims[m]; }
-  p.val = vals;
+  for (int m = 0; m < nmodes; ++m) { p.fac[m] = factors[m]; p.dims[m] = dims[m]; }
+  p.aos = aos;
   p.skey = skey;
   p.spos = spos;
   p.out = out;
   p.len = len;
+  p.dn = (uint32_t)std::min<uint64_t>(dims[mode], 0xFFFFFFFFull);
   p.nmodes = nmodes;
   p.mode = mode;
   // ~64 nonzeros per lane group: long runs per group, enough groups to fill the GPU
@@ -279,10 +352,16 @@ void launch_seg_sorted(int nmodes, const uint64_t* dims, uint64_t len, const uin
     const uint64_t groups = std::max<uint64_t>(1, len / 64);
     return (int)std::max<uint64_t>(1, std::min<uint64_t>((groups * lpn + 255) / 256, (uint64_t)148 * 16));
   };
-  switch (rank) {
-    case 16: seg_sorted_kernel<16><<<grid_for(4), 256, 0, s>>>(p); break;
-    case 32: seg_sorted_kernel<32><<<grid_for(8), 256, 0, s>>>(p); break;
-    default: seg_sorted_kernel<64><<<grid_for(16), 256, 0, s>>>(p); break;
+  const bool w8 = seg_aos_words(nmodes) == 8;
+  if (rank == 16) {
+    if (w8) seg_sorted_kernel<16, 8><<<grid_for(4), 256, 0, s>>>(p);
+    else seg_sorted_kernel<16, 4><<<grid_for(4), 256, 0, s>>>(p);
+  } else if (rank == 32) {
+    if (w8) seg_sorted_kernel<32, 8><<<grid_for(8), 256, 0, s>>>(p);
+    else seg_sorted_kernel<32, 4><<<grid_for(8), 256, 0, s>>>(p);
+  } else {
+    if (w8) seg_sorted_kernel<64, 8><<<grid_for(16), 256, 0, s>>>(p);
+    else seg_sorted_kernel<64, 4><<<grid_for(16), 256, 0, s>>>(p);
   }
   count_launch();
   SF_CUDA(cudaGetLastError());
@@ -360,11 +439,11 @@ __global__ void hot_fill_kernel(const HotFill h, int R4, float* __restrict__ cac
   }
 }
 
-static int frag3_occ(int N, int R, int S, int threads, size_t smem) {
+static int frag3_occ(int N, int R, int S, int threads, size_t smem, bool hot) {
   switch (R) {
-    case 16: return frag3_occ_r16(N, S, threads, smem);
-    case 32: return frag3_occ_r32(N, S, threads, smem);
-    case 64: return frag3_occ_r64(N, S, threads, smem);
+    case 16: return frag3_occ_r16(N, S, threads, smem, hot);
+    case 32: return frag3_occ_r32(N, S, threads, smem, hot);
+    case 64: return frag3_occ_r64(N, S, threads, smem, hot);
     default: return 0;
   }
 }
@@ -435,7 +514,7 @@ static void launch_frag3(const Tensor& t, const Plan& p, const float* const* fac
   const int threads = l.block_threads;
   int per_sm = l.ctas_per_sm;
   if (p.occ_threads != threads || p.occ_smem != smem) {  // occupancy query once per plan launch shape
-    p.occ = frag3_occ(N, R, S, threads, smem);
+    p.occ = frag3_occ(N, R, S, threads, smem, p.hot_total > 0);
     p.occ_threads = threads;
     p.occ_smem = smem;
   }

@@ -86,6 +86,32 @@ def test_streamed_fullsize_nell2(cuda_device):
         assert rel <= G.TOL, (n, rel)
 
 
+def test_streamed_modes_fullsize_nell2(cuda_device):
+    """sf_mttkrp_streamed_modes at BASELINE.json configs[1] size: all three modes from ONE
+    upload of the pinned host COO (the bench's one-shot e2e path), sampled rows incl. the
+    heaviest within the north-star tolerance, empty rows exactly 0."""
+    cfg = synth.CONFIGS["nell2"]
+    inds, vals = synth.config_tensor(cfg)
+    facs = synth.config_factors(cfg)
+    R = cfg.rank
+    rng = np.random.default_rng(5)
+    h_inds = [torch.from_numpy(a.view(np.int32)).pin_memory() for a in inds]
+    h_vals = torch.from_numpy(vals).pin_memory()
+    d_facs = [torch.from_numpy(f).cuda() for f in facs]
+    outs = [torch.full((d, R), float("nan"), device="cuda") for d in cfg.dims]
+    sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, d_facs, outs, 16, 4)
+    torch.cuda.synchronize()
+    for n in range(cfg.nmodes):
+        rows, empty, _ = _sample_rows(rng, inds[n], cfg.dims[n], k=24)
+        Yr, Sr = oracle.mttkrp_rows(cfg.dims, inds, vals, facs, R, n, rows)
+        got = outs[n][torch.from_numpy(rows).cuda()].cpu().numpy()
+        rel, _ = oracle.max_rel_err(got, Yr, Sr)
+        assert rel <= G.TOL, (n, rel)
+        if len(empty):
+            assert not outs[n][torch.from_numpy(empty).cuda()].any()
+        assert torch.isfinite(outs[n]).all()
+
+
 def test_streamed_heavy_row(cuda_device):
     """SURVEY C-2: one row holding a large share of 2e7 nonzeros (amazon mode 3 has 1.2e8 in one
     row) -- the sorted-segment kernel pre-reduces it in registers, so the fp32 atomic chain

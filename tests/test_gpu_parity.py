@@ -228,6 +228,51 @@ def test_streamed_one_shot(cuda_device, segments, streams):
         G.assert_parity(y.cpu().numpy(), cfg.dims, inds, vals, facs, cfg.rank, n)
 
 
+@pytest.mark.parametrize("dims,R,nnz,mask", [
+    ((100, 80, 60), 16, 10_000, (1, 1, 1)),        # 16-byte records, every mode
+    ((100, 80, 60), 32, 10_000, (1, 0, 1)),        # a subset of modes (A_2 still gathered)
+    ((30, 20, 40, 7), 32, 20_000, (1, 1, 1, 1)),   # N = 4: 32-byte records
+    ((9, 11, 13, 5, 3), 64, 5_000, (0, 1, 0, 1, 1)),
+    ((100, 80, 60), 12, 10_000, (1, 1, 1)),        # rank outside 16/32/64: one atomic per nonzero
+])
+@pytest.mark.parametrize("segments,streams", [(1, 1), (5, 3), (16, 4)])
+def test_streamed_modes_one_shot(cuda_device, dims, R, nnz, mask, segments, streams):
+    """sf_mttkrp_streamed_modes: one upload of the host COO, every requested mode computed from
+    each segment (A8 (ii)); each Y against the fp64 oracle."""
+    inds, vals = synth.gen_coo(dims, nnz, 77, zipf=(1.0,) * len(dims), val_kind="signed")
+    facs = synth.gen_factors(dims, R, 78, "signed")
+    tf = [G.dev_f(f) for f in facs]
+    outs = [torch.full((dims[n], R), float("nan"), device="cuda:0") if mask[n] else None
+            for n in range(len(dims))]
+    if sum(mask) == 1:  # the one computed mode's factor may be NULL
+        tf[mask.index(1)] = None
+    sf.mttkrp_streamed_modes(dims, inds, vals, tf, outs, segments, streams)
+    torch.cuda.synchronize()
+    for n in range(len(dims)):
+        if mask[n]:
+            G.assert_parity(outs[n].cpu().numpy(), dims, inds, vals, facs, R, n)
+
+
+def test_streamed_modes_errors(cuda_device):
+    dims, R = (10, 9, 8), 16
+    inds, vals = synth.gen_coo(dims, 1000, 5)
+    facs = [G.dev_f(f) for f in synth.gen_factors(dims, R, 6)]
+    with pytest.raises(sf.SfError):  # no output mode
+        sf.mttkrp_streamed_modes(dims, inds, vals, facs, [None, None, None])
+    bad = [a.copy() for a in inds]
+    bad[1][500] = 9  # == dims[1]
+    outs = [torch.empty((d, R), device="cuda:0") for d in dims]
+    with pytest.raises(sf.SfError) as ei:
+        sf.mttkrp_streamed_modes(dims, bad, vals, facs, outs, 4, 2)
+    assert ei.value.status == 2  # SF_ERR_INDEX_OUT_OF_RANGE
+    # the offending nonzero was skipped, every other one summed
+    keep = np.ones(1000, bool)
+    keep[500] = False
+    for n in range(3):
+        G.assert_parity(outs[n].cpu().numpy(), dims, [a[keep] for a in inds], vals[keep],
+                        [f.cpu().numpy() for f in facs], R, n)
+
+
 def test_edge_cases(cuda_device):
     dims, R = (10, 9, 8), 16
     facs = synth.gen_factors(dims, R, 1)
