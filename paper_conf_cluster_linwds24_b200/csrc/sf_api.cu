@@ -841,8 +841,11 @@ static void streamed_impl(int nmodes, const uint64_t* dims, uint64_t nnz, const 
     int bad = 0;
     SF_CUDA(cudaMemcpy(&bad, flag.p, 4, cudaMemcpyDeviceToHost));
     for (auto& s : st) cudaStreamDestroy(s);
+    st.clear();  // (the handler below must not destroy them again)
     cudaEventDestroy(zeroed);
+    zeroed = nullptr;
     if (before) cudaEventDestroy(before);
+    before = nullptr;
     if (bad) throw StatusError{SF_ERR_INDEX_OUT_OF_RANGE, "some index is >= its dimension"};
   } catch (...) {
     for (auto& s : st) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }

@@ -2,7 +2,8 @@
 nnz = 1,741,809,018, R = 16) at full size on ONE B200: each mode planned by the selector,
 run, checked on sampled rows against the oracle, then released (one plan resident at a
 time keeps the footprint < 180 GB).  The oracle streams the tensor in 100M-nonzero chunks
-(device generator -> host -> oracle.mttkrp_rows, fp64 sums over chunks)."""
+(device generator -> host -> oracle.mttkrp_rows, fp64 sums over chunks).  The same rows are
+then checked for the one-shot streamed path from pinned host memory."""
 import numpy as np
 import pytest
 import torch
@@ -66,4 +67,21 @@ def test_amazon_fullsize_sampled_rows(cuda_device):
         del y
         T.plan_release(n, R)
     T.close()
+    sf.trim_cache()
+    # the one-shot path (sf_mttkrp_streamed_modes: every mode from one upload of the pinned host
+    # COO, 16 segments) against the same oracle rows -- the heavy rows' fp32 chains stay short
+    inds, vals = synth.config_tensor_device(cfg)
+    h_inds = [a.cpu().pin_memory() for a in inds]
+    h_vals = vals.cpu().pin_memory()
+    del inds, vals
+    torch.cuda.empty_cache()
+    outs = [torch.full((d, R), float("nan"), device="cuda") for d in cfg.dims]
+    sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, facs, outs, 16, 4)
+    torch.cuda.synchronize()
+    for n in range(cfg.nmodes):
+        assert torch.isfinite(outs[n]).all()
+        got = outs[n][torch.from_numpy(rows[n]).cuda()].cpu().numpy()
+        rel, zv = oracle.max_rel_err(got, Yr[n], Sr[n])
+        assert rel <= G.TOL, ("one-shot", n, rel)
+        assert zv == 0.0
     sf.trim_cache()

@@ -2,7 +2,8 @@
 """Small workload for compute-sanitizer (memcheck / racecheck / synccheck):
 every kernel family of libscalfrag on a skewed tiny tensor and a heavy-row tensor --
 frag3 in owner / memset+atomics / shared-memory-staged / L2-tiled / hot-row / deterministic
-launches, 3-way and 4-way (packed records), the sorted-segment streamed path, shards,
+launches, 3-way and 4-way (packed records), the sorted-segment streamed paths (one mode /
+all modes from one upload), shards,
 CP-ALS.  Checks every result against the oracle so a silent corruption also fails.
 
   compute-sanitizer --tool memcheck  python tools/sanitize_check.py
@@ -70,6 +71,13 @@ def main():
             sf.mttkrp_streamed(dims, inds, vals, tf, n, y, 3, 2)
             rel, zv = oracle.max_rel_err(y.cpu().numpy(), Y, S)
             assert rel <= 1e-4 and zv == 0, ("streamed", dims, n, rel)
+        # every mode from one upload (sf_mttkrp_streamed_modes, 16/32-byte segment records)
+        outs = [torch.full((d, R), float("nan"), device="cuda") for d in dims]
+        sf.mttkrp_streamed_modes(dims, inds, vals, tf, outs, 5, 3)
+        for n in range(N):
+            Y, S = oracle.mttkrp(dims, inds, vals, facs, R, n)
+            rel, zv = oracle.max_rel_err(outs[n].cpu().numpy(), Y, S)
+            assert rel <= 1e-4 and zv == 0, ("streamed_modes", dims, n, rel)
         if N == 3 and R <= 64:
             with sf.Tensor(dims, ti, tv) as T:
                 A = [f.clone() for f in tf]
