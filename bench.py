@@ -237,7 +237,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-oneshot", action="store_true", help="e2e: resident path only")
-    ap.add_argument("--oneshot-segments", type=int, default=16)
+    ap.add_argument("--oneshot-segments", type=int, default=0,
+                    help="0: 16, or 32 above 5e8 nonzeros (profiles/r02/s3/stream_study_all_modes.jsonl)")
     ap.add_argument("--e2e-trace", action="store_true", help="host time after every call of each e2e step (stderr)")
     ap.add_argument("--cpu-sample", type=int, default=30_000_000)
     ap.add_argument("--ref-sample", type=int, default=1_000_000)
@@ -255,6 +256,8 @@ def main():
         sys.exit(2)
     cfg = synth.CONFIGS[args.config]
 
+    if args.oneshot_segments <= 0:
+        args.oneshot_segments = 32 if cfg.nnz > 500_000_000 else 16
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return

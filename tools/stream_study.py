@@ -3,7 +3,8 @@
 L201-229, Fig. 11 "fix the number of segments to 4 ... fix the number of CUDA
 streams to 4"), on B200 with synthetic tensors shaped like the paper's workloads.
 
-For a host-resident (pinned) COO tensor and one mode:
+For a host-resident (pinned) COO tensor and one mode (and, under "all_modes_one_upload", every
+mode from one upload with sf_mttkrp_streamed_modes):
   T_h2d      the COO upload alone (cudaMemcpy of the N+1 arrays)
   T_(1,1)    sf_mttkrp_streamed with 1 segment on 1 stream (no overlap)
   T_compute  = T_(1,1) - T_h2d
@@ -75,6 +76,25 @@ def main():
         t_comp = max(t11 - t_h2d, 1e-6)
         ov = {k: (t_h2d + t_comp - v) / min(t_h2d, t_comp) for k, v in grid.items()}
 
+        # every mode from one upload (sf_mttkrp_streamed_modes): the N MTTKRPs of a step
+        ys = [torch.empty((d, R), device="cuda") for d in cfg.dims]
+        reps_all = 2 if cfg.nnz > 5e8 else 5
+        grid_all = {}
+        for S in (1, 4, 8, 16, 32):
+            for K in (1, 2, 4):
+                if K > S:
+                    continue
+                grid_all[f"{S}x{K}"] = wall(lambda: sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, facs, ys, S, K),
+                                            reps=reps_all)
+        t11a = grid_all["1x1"]
+        t_comp_all = max(t11a - t_h2d, 1e-6)
+        ov_all = {k: (t_h2d + t_comp_all - v) / min(t_h2d, t_comp_all) for k, v in grid_all.items()}
+        best_all = min(grid_all, key=grid_all.get)
+        all_modes = {"t_streamed_ms": grid_all, "t_compute_ms": t_comp_all, "overlap_ratio": ov_all,
+                     "best": best_all, "best_over_h2d": grid_all[best_all] / t_h2d,
+                     "speedup_best_vs_1x1": t11a / grid_all[best_all]}
+        del ys
+
         def resident():
             with sf.Tensor(cfg.dims, h_inds, h_vals, segments=8, streams=4) as T:
                 T.plan(n, R)
@@ -96,7 +116,8 @@ def main():
                      "breakdown_ms": {"h2d": t_h2d, "kernel": t_comp, "d2h": t_d2h,
                                       "serial_sum": t_h2d + t_comp + t_d2h,
                                       "streamed_best_plus_d2h": grid[best] + t_d2h},
-                     "streamed_peak_device_bytes_32seg": int(peak_streamed)}
+                     "streamed_peak_device_bytes_32seg": int(peak_streamed),
+                     "all_modes_one_upload": all_modes}
         print(json.dumps({name: out[name]}), flush=True)
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     path = os.path.join(ROOT, "gpurun_out", "stream_study.json")
