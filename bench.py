@@ -591,7 +591,11 @@ def main():
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": achieved / peaks["hbm_gbs"], "traffic": traffic, "traffic_src": traffic_src,
                          "kernel": "frag3_kernel", "peak_src": peaks["src"],
-                         "bytes_per_launch": bytes_launch, "launch_ms": mean_launch_ms},
+                         "bytes_per_launch": bytes_launch, "launch_ms": mean_launch_ms,
+                         # the DRAM bytes ncu measured for this config's
+                         # launches moved in the launch time, against the same peak
+                         "dram_gbs": None if not traffic else traffic / (mean_launch_ms * 1e-3) / 1e9,
+                         "dram_frac": None if not traffic else traffic / (mean_launch_ms * 1e-3) / 1e9 / peaks["hbm_gbs"]},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches),

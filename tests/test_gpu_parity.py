@@ -253,6 +253,31 @@ def test_streamed_modes_one_shot(cuda_device, dims, R, nnz, mask, segments, stre
             G.assert_parity(outs[n].cpu().numpy(), dims, inds, vals, facs, R, n)
 
 
+def test_streamed_modes_edge(cuda_device):
+    """Empty tensor (every Y exactly 0), N = 8 (beyond the record widths: one atomic per
+    nonzero), and a single nonzero on a 2-way tensor with more segments than nonzeros."""
+    dims, R = (10, 9, 8), 16
+    facs = [G.dev_f(f) for f in synth.gen_factors(dims, R, 6)]
+    outs = [torch.full((d, R), 7.0, device="cuda:0") for d in dims]
+    e = [np.zeros(0, np.uint32)] * 3
+    sf.mttkrp_streamed_modes(dims, e, np.zeros(0, np.float32), facs, outs, 4, 2)
+    assert all(not o.any() for o in outs)
+    dims8 = (3, 4, 5, 3, 4, 5, 3, 4)
+    inds, vals = synth.gen_coo(dims8, 3000, 9, val_kind="signed")
+    facs8 = synth.gen_factors(dims8, R, 10, "signed")
+    outs = [torch.full((d, R), float("nan"), device="cuda:0") for d in dims8]
+    sf.mttkrp_streamed_modes(dims8, inds, vals, [G.dev_f(f) for f in facs8], outs, 3, 2)
+    for n in range(8):
+        G.assert_parity(outs[n].cpu().numpy(), dims8, inds, vals, facs8, R, n)
+    dims2 = (5, 6)
+    one = [np.array([4], np.uint32), np.array([2], np.uint32)]
+    f2 = synth.gen_factors(dims2, 32, 11)
+    outs = [torch.full((d, 32), float("nan"), device="cuda:0") for d in dims2]
+    sf.mttkrp_streamed_modes(dims2, one, np.array([0.5], np.float32), [G.dev_f(f) for f in f2], outs, 8, 4)
+    for n in range(2):
+        G.assert_parity(outs[n].cpu().numpy(), dims2, one, np.array([0.5], np.float32), f2, 32, n)
+
+
 def test_streamed_modes_errors(cuda_device):
     dims, R = (10, 9, 8), 16
     inds, vals = synth.gen_coo(dims, 1000, 5)
