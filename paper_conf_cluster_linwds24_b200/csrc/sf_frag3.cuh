@@ -239,7 +239,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           const uint32_t first = s0, cnt = min(K, ge - s0);
           const uint32_t bytes = cnt * (uint32_t)(W * 4);
           mbar_expect_tx_only(&wbar[st], bytes);
-          bulk_g2s(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
+          bulk_g2s_stream(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
         }
       }
       __syncwarp();
@@ -303,17 +303,17 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
         red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
         if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
       } else {
-        if constexpr (VEC == 8) st256(out0 + (size_t)cur * R, acc0, acc1);
-        else st128(out0 + (size_t)cur * R, acc0);
+        if constexpr (VEC == 8) st256_stream(out0 + (size_t)cur * R, acc0, acc1);
+        else st128_stream(out0 + (size_t)cur * R, acc0);
       }
       acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
       acc1 = acc0;
     };
     auto zero_rows = [&](uint32_t r0, uint32_t r1) {  // rows (r0, r1) exclusive
       for (uint32_t r = r0 + 1; r < r1; ++r) {
-        if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
-                                      make_float4(0.f, 0.f, 0.f, 0.f));
-        else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
+        if constexpr (VEC == 8) st256_stream(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
+                                             make_float4(0.f, 0.f, 0.f, 0.f));
+        else st128_stream(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
       }
     };
     auto advance = [&](uint32_t i) {  // run edge inside the sub-range: close `cur`, open i
