@@ -44,6 +44,13 @@ __device__ __forceinline__ void ldg256_na(const float4* p, float4& a, float4& b)
       : "l"(p));
 }
 
+// 256-bit gather with an L2 cache-hint policy (createpolicy), A/B experiments on hot / cold rows
+__device__ __forceinline__ void ldg256_na_pol(const float4* p, float4& a, float4& b, uint64_t pol) {
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+      : "l"(p), "l"(pol));
+}
+
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count));
 }

@@ -30,6 +30,10 @@
 
 #include "sf_frag.cuh"
 
+#ifndef SF_HOT_POLICY
+#define SF_HOT_POLICY 0  // A/B: L2 evict_last on hot-row gathers, evict_first on cold ones
+#endif
+
 #ifndef SF_FRAG_U_WIDE
 #define SF_FRAG_U_WIDE 1  // U for N >= 4 at R >= 32: 1 avoids spills (deli-4d +3 %; A/B: -DSF_FRAG_U_WIDE=2)
 #endif
@@ -181,6 +185,11 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   const float4* gbase[G - S > 0 ? G - S : 1];
 #pragma unroll
   for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]);
+#if SF_HOT_POLICY
+  uint64_t pol_last, pol_first;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_first));
+#endif
   uint32_t fac_phase = 0;
   uint32_t it = 0;  // stages this warp has consumed (stage = it % 2, parity = (it / 2) & 1)
   float* const out0 = p.out + 4 * c0;
@@ -272,12 +281,21 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     auto gather = [&](int q, uint32_t row_idx) -> F8 {
       const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
       size_t row = (size_t)row_idx * R4;
+      bool is_hot = false;
       if (HOT && q >= S) {  // hot-row cache: the slot inside the dense hot block
         const uint32_t hb = p.hot_bit[q];
-        if (row_idx & hb) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
+        is_hot = (row_idx & hb) != 0;
+        if (is_hot) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
       }
+      (void)is_hot;
       F8 r;
       if constexpr (VEC == 8) {
+#if SF_HOT_POLICY
+        if (HOT && q >= S) {  // A/B: hot rows evict_last, cold rows evict_first in L2
+          ldg256_na_pol(base + row + c0, r.a, r.b, is_hot ? pol_last : pol_first);
+          return r;
+        }
+#endif
         if (q < S) {
           const float4 x = base[row + c0 + par];
           const float4 y = base[row + c0 + 1 - par];
