@@ -500,16 +500,36 @@ def main():
 
         # The one-shot path (sf_mttkrp_streamed_modes): the factors go up
         # first, then every segment of the COO is uploaded once and all modes are computed from
-        # it behind the later segments' H2D; then the D2H of every Y.  No plans; at N = 1 only.
+        # it behind the later segments' H2D; then the D2H of every Y.  No plans.  At N > 1 each
+        # rank streams its own nonzero range, its partial Ys are combined by a reduce-scatter
+        # (NCCL over NVLink, BJ:north_star (5)) and each rank reads back its block
+        # of rows.
+        pad_rows = [-(-cfg.dims[n] // world) * world for n in range(N)]
+        blk_rows = [pr // world for pr in pad_rows]
+        h_blk = [torch.empty((blk_rows[n], R), dtype=torch.float32).pin_memory() for n in range(N)] \
+            if world > 1 else h_out
+
         def oneshot_step():
             with torch.cuda.stream(stream):
                 for m in up_order:
                     df[m].copy_(h_facs[m], non_blocking=True)
-                outs1 = [torch.empty((cfg.dims[n], R), dtype=torch.float32, device=dev) for n in range(N)]
-                sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, df, outs1, args.oneshot_segments, 4,
-                                         stream=stream)
+                outs1 = [torch.empty((pad_rows[n], R), dtype=torch.float32, device=dev) for n in range(N)]
+                for n in range(N):
+                    outs1[n][cfg.dims[n]:].zero_()
+                sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, df, [o[:cfg.dims[n]] for n, o in enumerate(outs1)],
+                                         args.oneshot_segments, 4, stream=stream)
                 for n in order:
-                    h_out[n].copy_(outs1[n], non_blocking=True)
+                    if world == 1:
+                        h_out[n].copy_(outs1[n], non_blocking=True)
+                        continue
+                    if same_gpu:  # gloo (tests on one GPU): a host-staged all-reduce
+                        t_ = outs1[n].cpu()
+                        dist.all_reduce(t_)
+                        blk = t_[rank * blk_rows[n]:(rank + 1) * blk_rows[n]]
+                    else:
+                        blk = torch.empty((blk_rows[n], R), dtype=torch.float32, device=dev)
+                        dist.reduce_scatter_tensor(blk, outs1[n])
+                    h_blk[n].copy_(blk, non_blocking=True)
             torch.cuda.synchronize(dev)
 
         def time_steps(fn):
@@ -530,7 +550,7 @@ def main():
         # up to 3x slower, not reproducibly (profiles/r02/e2e_variance/)
         paths = {"resident": statistics.median(step_ms)}
         oneshot_ms = None
-        if world == 1 and not args.no_oneshot:
+        if not args.no_oneshot:
             oneshot_ms = time_steps(oneshot_step)
             paths["one_shot"] = statistics.median(oneshot_ms)
         path = min(paths, key=paths.get)
@@ -564,9 +584,13 @@ def main():
                        "value": flops_step / (paths["one_shot"] * 1e-3) / 1e9,
                        "step_ms": [round(x, 2) for x in oneshot_ms],
                        "segments": args.oneshot_segments, "streams": 4,
+                       "d2h_bytes_per_step": int(sum(b.numel() * 4 for b in h_blk)),
+                       "combine": None if world == 1 else "reduce-scatter of the partial Ys (NCCL)",
                        "includes": "factor H2D + sf_mttkrp_streamed_modes(pinned host COO: per segment "
                                    "H2D + validate + AoS + per mode sort and reduce, overlapped with the "
-                                   "next segments' H2D) + D2H of every Y (host wall clock)"}})},
+                                   "next segments' H2D) + D2H of every Y (at N > 1: each rank streams "
+                                   "its nonzero range, reduce-scatter of the partial Ys, D2H of its row "
+                                   "block; host wall clock, max over ranks)"}})},
                "includes": "the faster of the two public host-input paths (paths.*), same step, same "
                            "factors, same H2D/D2H bytes"}
     elif not args.no_e2e and e2e_skip:

@@ -35,6 +35,10 @@ def test_bench_two_ranks_same_gpu(cuda_device):
     line = [l for l in r.stdout.splitlines() if l.startswith("{")][-1]
     d = json.loads(line)
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["parallelism"] == "nnz-shard2"
+    # both host-input paths at N = 2: resident shards, and the one-shot path on each rank's
+    # nonzero range with the partial Ys combined across ranks
+    assert set(d["e2e"]["paths"]) == {"resident", "one_shot"}, d["e2e"]
+    assert all(v["ms_per_step"] > 0 for v in d["e2e"]["paths"].values())
 
 
 def test_nccl_ranks_exchange_matches_single(cuda_device):

@@ -4,7 +4,8 @@ the boundary exchange inside libscalfrag), and
   * the row-sharded local blocks must equal the single-rank result bit-exactly on the rows
     each rank owns and be 0 elsewhere (integer data), every row owned at most once;
   * sf_allgather_rows must rebuild the full single-rank Y on every rank;
-  * sf_cpals on the shards must give the same fits and factors as on one rank."""
+  * sf_cpals on the shards must give the same fits and factors as on one rank;
+  * the one-shot path on each rank's nonzero range, summed over ranks, must equal one rank's Y."""
 import os
 import sys
 
@@ -106,6 +107,25 @@ def main():
             if not torch.equal(y1, y2):
                 ok = False
                 msgs.append(f"dist v2 mode {n} rank {rank}: auto-planned Y differs from v1")
+    # the one-shot path at N ranks (bench.py's e2e leg): each rank streams its nonzero range from
+    # host memory into partial Ys of every mode; their sum over ranks (all-reduce) must equal the
+    # single-rank Y bit for bit (integer data)
+    h_i = [a[lo:hi].cpu().pin_memory() for a in inds]
+    h_v = vals[lo:hi].cpu().pin_memory()
+    parts = [torch.empty((d, R), device=dev) for d in dims]
+    sf.mttkrp_streamed_modes(dims, h_i, h_v, facs, parts, 4, 2)
+    torch.cuda.synchronize()
+    for n in range(3):
+        with sf.Tensor(dims, inds, vals) as T1:
+            T1.plan(n, R)
+            full = torch.empty((dims[n], R), device=dev)
+            T1.mttkrp(n, facs, full)
+        torch.cuda.synchronize()
+        tot = parts[n].cpu() if os.environ.get("SF_SAME_GPU") == "1" else parts[n]
+        dist.all_reduce(tot)
+        if not torch.equal(tot.to(dev), full):
+            ok = False
+            msgs.append(f"one-shot mode {n} rank {rank}: sum of the partial Ys differs from one rank")
     # CP-ALS on the shards == CP-ALS on one rank (same initial factors) up to fp32 summation
     # order (the shards sum M and the Grams in a different order): the bar of
     # tests/test_gpu_cpals.py against the fp64 oracle (fits 2e-4 over 3 sweeps, factors 2e-3
