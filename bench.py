@@ -235,7 +235,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-steps", type=int, default=7)
     ap.add_argument("--no-oneshot", action="store_true", help="e2e: resident path only")
     ap.add_argument("--oneshot-segments", type=int, default=0,
                     help="0: 16, or 32 above 5e8 nonzeros (profiles/r02/s3/stream_study_all_modes.jsonl)")
