@@ -64,3 +64,28 @@ def test_no_oracle_in_product_path():
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "oracle.c" not in txt and "liboracle" not in txt, f
+
+
+def test_streamed_modes_argument_errors_without_gpu():
+    """sf_mttkrp_streamed_modes rejects bad arguments before touching the device (the checks a
+    C caller relies on: no output mode, a NULL factor a requested mode gathers, bad rank)."""
+    import numpy as np
+    import pytest
+    dims = (4, 3, 2)
+    inds = [np.zeros(5, np.uint32) for _ in dims]
+    vals = np.ones(5, np.float32)
+    facs = [np.ones((d, 16), np.float32) for d in dims]
+    with pytest.raises(sf.SfError) as ei:
+        sf.mttkrp_streamed_modes(dims, inds, vals, facs, [None, None, None], stream=0)
+    assert ei.value.status == 1  # SF_ERR_INVALID_ARG
+    out = np.zeros((4, 16), np.float32)
+    with pytest.raises(sf.SfError) as ei:  # mode 0 gathers A_1: it must not be NULL
+        sf.mttkrp_streamed_modes(dims, inds, vals, [facs[0], None, facs[2]], [out, None, None], stream=0)
+    assert ei.value.status == 1
+    L = sf.lib()
+    d = (ctypes.c_uint64 * 3)(*dims)
+    op = (ctypes.c_void_p * 3)(out.ctypes.data, None, None)
+    fp = (ctypes.c_void_p * 3)(*[f.ctypes.data for f in facs])
+    ip = (ctypes.c_void_p * 3)(*[a.ctypes.data for a in inds])
+    assert L.sf_mttkrp_streamed_modes(3, d, 5, ip, vals.ctypes.data, fp, 0, op, 4, 2, None) == 1  # rank 0
+    assert L.sf_mttkrp_streamed_modes(1, d, 5, ip, vals.ctypes.data, fp, 16, op, 4, 2, None) == 1  # nmodes 1

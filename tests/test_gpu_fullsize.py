@@ -86,11 +86,12 @@ def test_streamed_fullsize_nell2(cuda_device):
         assert rel <= G.TOL, (n, rel)
 
 
-def test_streamed_modes_fullsize_nell2(cuda_device):
-    """sf_mttkrp_streamed_modes at BASELINE.json configs[1] size: all three modes from ONE
-    upload of the pinned host COO (the bench's one-shot e2e path), sampled rows incl. the
-    heaviest within the north-star tolerance, empty rows exactly 0."""
-    cfg = synth.CONFIGS["nell2"]
+@pytest.mark.parametrize("name", ["nell2", "deli4d"])
+def test_streamed_modes_fullsize(cuda_device, name):
+    """sf_mttkrp_streamed_modes at BASELINE.json configs[1] / configs[2] size: every mode from ONE
+    upload of the pinned host COO (the bench's one-shot e2e path; 16- and 32-byte segment
+    records), sampled rows incl. the heaviest within the north-star tolerance, empty rows exactly 0."""
+    cfg = synth.CONFIGS[name]
     inds, vals = synth.config_tensor(cfg)
     facs = synth.config_factors(cfg)
     R = cfg.rank
