@@ -36,10 +36,39 @@ __device__ __forceinline__ uint32_t su32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-__device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
+#ifndef SF_VEC4_PF
+#define SF_VEC4_PF 0
+#endif
+#define SF_STR_(x) #x
+#define SF_STR(x) SF_STR_(x)
+#ifndef SF_VEC4_NA
+#define SF_VEC4_NA 0  // 1: 128-bit gathers (R = 16) bypass L1 allocation (A/B: amazon 1.4-1.7x slower)
+#endif
+__device__ __forceinline__ float4 ldg128(const float4* p) {
+#if SF_VEC4_NA
+  float4 a;
+  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
+  return a;
+#elif SF_VEC4_PF
+  float4 a;  // L1-allocating, with an explicit L2 prefetch size (A/B: -DSF_VEC4_PF=64 / 128 / 256)
+  asm("ld.global.nc.L2::" SF_STR(SF_VEC4_PF) "B.v4.f32 {%0,%1,%2,%3}, [%4];"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
+  return a;
+#else
+  return __ldg(p);
+#endif
+}
 
 __device__ __forceinline__ void ldg256_na(const float4* p, float4& a, float4& b) {
   asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+      : "l"(p));
+}
+// L1-allocating 256-bit gather: the hot-row plans' gathers (session 3 A/B: deli-4d +2.3 %,
+// nell-1 unchanged; on the L2-resident nell-2 plans allocation cost 1.5 %, so those keep
+// ldg256_na)
+__device__ __forceinline__ void ldg256_l1(const float4* p, float4& a, float4& b) {
+  asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
       : "l"(p));
 }

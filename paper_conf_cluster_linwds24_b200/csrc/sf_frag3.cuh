@@ -302,7 +302,8 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           r.a = par ? y : x;
           r.b = par ? x : y;
         } else {
-          ldg256_na(base + row + c0, r.a, r.b);
+          if constexpr (HOT) ldg256_l1(base + row + c0, r.a, r.b);
+          else ldg256_na(base + row + c0, r.a, r.b);
         }
       } else {
         r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
