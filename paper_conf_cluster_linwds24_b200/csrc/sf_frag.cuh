@@ -36,6 +36,11 @@ __device__ __forceinline__ uint32_t su32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+__device__ __forceinline__ float4 ldg128_na(const float4* p) {
+  float4 a;
+  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
+  return a;
+}
 #ifndef SF_VEC4_PF
 #define SF_VEC4_PF 0
 #endif

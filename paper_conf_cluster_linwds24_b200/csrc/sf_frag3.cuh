@@ -30,6 +30,10 @@
 
 #include "sf_frag.cuh"
 
+#ifndef SF_SPLIT_L1
+#define SF_SPLIT_L1 0  // A/B: L1 allocation only for hot-row gathers
+#endif
+
 #ifndef SF_HOT_POLICY
 #define SF_HOT_POLICY 0  // A/B: L2 evict_last on hot-row gathers, evict_first on cold ones
 #endif
@@ -302,11 +306,23 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           r.a = par ? y : x;
           r.b = par ? x : y;
         } else {
+#if SF_SPLIT_L1
+          // A/B: only the hot rows allocate in L1, cold rows bypass it
+          if (HOT && is_hot) ldg256_l1(base + row + c0, r.a, r.b);
+          else ldg256_na(base + row + c0, r.a, r.b);
+#else
           if constexpr (HOT) ldg256_l1(base + row + c0, r.a, r.b);
           else ldg256_na(base + row + c0, r.a, r.b);
+#endif
         }
       } else {
+#if SF_SPLIT_L1
+        if (q < S) r.a = base[row + c0];
+        else if (!HOT || is_hot) r.a = ldg128(base + row + c0);
+        else r.a = ldg128_na(base + row + c0);
+#else
         r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
+#endif
       }
       return r;
     };
