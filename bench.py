@@ -238,7 +238,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=7)
     ap.add_argument("--no-oneshot", action="store_true", help="e2e: resident path only")
     ap.add_argument("--oneshot-segments", type=int, default=0,
-                    help="0: 16, or 32 above 5e8 nonzeros (profiles/r02/s3/stream_study_all_modes.jsonl)")
+                    help="0: the library's choice (about 5 M nonzeros per segment, 2..32)")
     ap.add_argument("--e2e-trace", action="store_true", help="host time after every call of each e2e step (stderr)")
     ap.add_argument("--cpu-sample", type=int, default=30_000_000)
     ap.add_argument("--ref-sample", type=int, default=1_000_000)
@@ -256,8 +256,6 @@ def main():
         sys.exit(2)
     cfg = synth.CONFIGS[args.config]
 
-    if args.oneshot_segments <= 0:
-        args.oneshot_segments = 32 if cfg.nnz > 500_000_000 else 16
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return
@@ -517,7 +515,7 @@ def main():
                 for n in range(N):
                     outs1[n][cfg.dims[n]:].zero_()
                 sf.mttkrp_streamed_modes(cfg.dims, h_inds, h_vals, df, [o[:cfg.dims[n]] for n, o in enumerate(outs1)],
-                                         args.oneshot_segments, 4, stream=stream)
+                                         args.oneshot_segments, 0, stream=stream)
                 for n in order:
                     if world == 1:
                         h_out[n].copy_(outs1[n], non_blocking=True)
@@ -583,7 +581,7 @@ def main():
                        "ms_per_step": paths["one_shot"],
                        "value": flops_step / (paths["one_shot"] * 1e-3) / 1e9,
                        "step_ms": [round(x, 2) for x in oneshot_ms],
-                       "segments": args.oneshot_segments, "streams": 4,
+                       "segments": args.oneshot_segments or "auto (about 5 M nonzeros each, 2..32)",
                        "d2h_bytes_per_step": int(sum(b.numel() * 4 for b in h_blk)),
                        "combine": None if world == 1 else "reduce-scatter of the partial Ys (NCCL)",
                        "includes": "factor H2D + sf_mttkrp_streamed_modes(pinned host COO: per segment "

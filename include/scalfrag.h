@@ -268,7 +268,9 @@ sf_status sf_mttkrp_streamed(int nmodes, const uint64_t* dims, uint64_t nnz,
  * nmodes device pointers; A_m may be NULL only if m is the one mode computed.  stream: the
  * work is ordered after what the caller queued on it before the call (e.g. the factor
  * uploads; NULL = no ordering).  Device footprint: O(streams x segment) + the caller's
- * arrays.  Synchronizes before returning; errors as sf_mttkrp_streamed. */
+ * arrays.  segments / streams <= 0: chosen by the library (about 5 M nonzeros per segment,
+ * 2..32; 4 streams, 2 for <= 2 segments).  Synchronizes before returning; errors as
+ * sf_mttkrp_streamed. */
 sf_status sf_mttkrp_streamed_modes(int nmodes, const uint64_t* dims, uint64_t nnz,
                                    const uint32_t* const* inds_host, const float* vals_host,
                                    const float* const* factors, int rank, float* const* outs,

@@ -759,8 +759,10 @@ static void streamed_impl(int nmodes, const uint64_t* dims, uint64_t nnz, const 
   if (!todo) throw StatusError{SF_ERR_INVALID_ARG, "no output mode"};
   for (int m = 0; m < nmodes; ++m)
     if ((todo & ~(1u << m)) && !factors[m]) throw StatusError{SF_ERR_INVALID_ARG, "factors[m] is NULL"};
-  if (segments <= 0) segments = 8;
-  if (streams <= 0) streams = 4;
+  // segments <= 0: about 5 M nonzeros per segment, 2..32 (every segment costs ~5 + 4 x modes
+  // launches, which dominate below ~10 M nonzeros; profiles/r02/s3/stream_study_all_modes.jsonl)
+  if (segments <= 0) segments = (int)std::min<uint64_t>(32, std::max<uint64_t>(2, (nnz + 2500000) / 5000000));
+  if (streams <= 0) streams = segments <= 2 ? 2 : 4;
   segments = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)segments, std::max<uint64_t>(1, nnz)));
   streams = std::max(1, std::min(streams, segments));
   const uint64_t seg_len = (nnz + segments - 1) / segments;
