@@ -36,33 +36,9 @@ __device__ __forceinline__ uint32_t su32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
-__device__ __forceinline__ float4 ldg128_na(const float4* p) {
-  float4 a;
-  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
-  return a;
-}
-#ifndef SF_VEC4_PF
-#define SF_VEC4_PF 0
-#endif
-#define SF_STR_(x) #x
-#define SF_STR(x) SF_STR_(x)
-#ifndef SF_VEC4_NA
-#define SF_VEC4_NA 0  // 1: 128-bit gathers (R = 16) bypass L1 allocation (A/B: amazon 1.4-1.7x slower)
-#endif
-__device__ __forceinline__ float4 ldg128(const float4* p) {
-#if SF_VEC4_NA
-  float4 a;
-  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
-  return a;
-#elif SF_VEC4_PF
-  float4 a;  // L1-allocating, with an explicit L2 prefetch size (A/B: -DSF_VEC4_PF=64 / 128 / 256)
-  asm("ld.global.nc.L2::" SF_STR(SF_VEC4_PF) "B.v4.f32 {%0,%1,%2,%3}, [%4];"
-      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w) : "l"(p));
-  return a;
-#else
-  return __ldg(p);
-#endif
-}
+// 128-bit gathers (R = 16) allocate in L1: bypassing it made amazon 1.4-1.7x slower
+// (session 3) -- its hot 64-byte rows hit there
+__device__ __forceinline__ float4 ldg128(const float4* p) { return __ldg(p); }
 
 __device__ __forceinline__ void ldg256_na(const float4* p, float4& a, float4& b) {
   asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
@@ -76,13 +52,6 @@ __device__ __forceinline__ void ldg256_l1(const float4* p, float4& a, float4& b)
   asm("ld.global.nc.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
       : "l"(p));
-}
-
-// 256-bit gather with an L2 cache-hint policy (createpolicy), A/B experiments on hot / cold rows
-__device__ __forceinline__ void ldg256_na_pol(const float4* p, float4& a, float4& b, uint64_t pol) {
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
-      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
-      : "l"(p), "l"(pol));
 }
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -101,44 +70,6 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(su32(dst)),
       "l"(src), "r"(bytes), "r"(su32(bar))
       : "memory");
-}
-#ifndef SF_STREAM_EVICT_FIRST
-#define SF_STREAM_EVICT_FIRST 0  // A/B: records and Y stores marked L2 evict_first
-#endif
-// The record stream (read once per launch): a 1-D bulk copy, optionally with an L2
-// evict_first policy so the streamed records do not displace gathered factor rows.
-__device__ __forceinline__ void bulk_g2s_stream(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-#if SF_STREAM_EVICT_FIRST
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
-          su32(dst)),
-      "l"(src), "r"(bytes), "r"(su32(bar)), "l"(pol)
-      : "memory");
-#else
-  bulk_g2s(dst, src, bytes, bar);
-#endif
-}
-__device__ __forceinline__ void st256_stream(float* p, const float4& a, const float4& b) {
-#if SF_STREAM_EVICT_FIRST
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  asm volatile("st.global.L2::cache_hint.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;" ::"l"(p), "f"(a.x), "f"(a.y),
-               "f"(a.z), "f"(a.w), "f"(b.x), "f"(b.y), "f"(b.z), "f"(b.w), "l"(pol));
-#else
-  st256(p, a, b);
-#endif
-}
-__device__ __forceinline__ void st128_stream(float* p, const float4& a) {
-#if SF_STREAM_EVICT_FIRST
-  uint64_t pol;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-  asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1,%2,%3,%4}, %5;" ::"l"(p), "f"(a.x), "f"(a.y), "f"(a.z),
-               "f"(a.w), "l"(pol));
-#else
-  st128(p, a);
-#endif
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t done = 0;

@@ -30,14 +30,6 @@
 
 #include "sf_frag.cuh"
 
-#ifndef SF_SPLIT_L1
-#define SF_SPLIT_L1 0  // A/B: L1 allocation only for hot-row gathers
-#endif
-
-#ifndef SF_HOT_POLICY
-#define SF_HOT_POLICY 0  // A/B: L2 evict_last on hot-row gathers, evict_first on cold ones
-#endif
-
 #ifndef SF_FRAG_U_WIDE
 #define SF_FRAG_U_WIDE 1  // U for N >= 4 at R >= 32: 1 avoids spills (deli-4d +3 %; A/B: -DSF_FRAG_U_WIDE=2)
 #endif
@@ -189,11 +181,6 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
   const float4* gbase[G - S > 0 ? G - S : 1];
 #pragma unroll
   for (int q = S; q < G; ++q) gbase[q - S] = reinterpret_cast<const float4*>(p.fac[p.slot_mode[q]]);
-#if SF_HOT_POLICY
-  uint64_t pol_last, pol_first;
-  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_first));
-#endif
   uint32_t fac_phase = 0;
   uint32_t it = 0;  // stages this warp has consumed (stage = it % 2, parity = (it / 2) & 1)
   float* const out0 = p.out + 4 * c0;
@@ -252,7 +239,7 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
           const uint32_t first = s0, cnt = min(K, ge - s0);
           const uint32_t bytes = cnt * (uint32_t)(W * 4);
           mbar_expect_tx_only(&wbar[st], bytes);
-          bulk_g2s_stream(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
+          bulk_g2s(my_region0 + (size_t)st * GPW * RS, p.rec + (size_t)first * W, bytes, &wbar[st]);
         }
       }
       __syncwarp();
@@ -285,44 +272,23 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
     auto gather = [&](int q, uint32_t row_idx) -> F8 {
       const float4* base = (q < S) ? sbase[q < S ? q : 0] : gbase[q >= S ? q - S : 0];
       size_t row = (size_t)row_idx * R4;
-      bool is_hot = false;
       if (HOT && q >= S) {  // hot-row cache: the slot inside the dense hot block
         const uint32_t hb = p.hot_bit[q];
-        is_hot = (row_idx & hb) != 0;
-        if (is_hot) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
+        if (row_idx & hb) row = (size_t)((int64_t)(row_idx & ~hb) * R4 + p.hot_delta[q]);
       }
-      (void)is_hot;
       F8 r;
       if constexpr (VEC == 8) {
-#if SF_HOT_POLICY
-        if (HOT && q >= S) {  // A/B: hot rows evict_last, cold rows evict_first in L2
-          ldg256_na_pol(base + row + c0, r.a, r.b, is_hot ? pol_last : pol_first);
-          return r;
-        }
-#endif
         if (q < S) {
           const float4 x = base[row + c0 + par];
           const float4 y = base[row + c0 + 1 - par];
           r.a = par ? y : x;
           r.b = par ? x : y;
         } else {
-#if SF_SPLIT_L1
-          // A/B: only the hot rows allocate in L1, cold rows bypass it
-          if (HOT && is_hot) ldg256_l1(base + row + c0, r.a, r.b);
-          else ldg256_na(base + row + c0, r.a, r.b);
-#else
           if constexpr (HOT) ldg256_l1(base + row + c0, r.a, r.b);
           else ldg256_na(base + row + c0, r.a, r.b);
-#endif
         }
       } else {
-#if SF_SPLIT_L1
-        if (q < S) r.a = base[row + c0];
-        else if (!HOT || is_hot) r.a = ldg128(base + row + c0);
-        else r.a = ldg128_na(base + row + c0);
-#else
         r.a = (q < S) ? base[row + c0] : ldg128(base + row + c0);
-#endif
       }
       return r;
     };
@@ -338,17 +304,17 @@ __global__ void __launch_bounds__(1024) frag3_kernel(const Frag3Params p) {
         red_add_v4_nomem(out0 + (size_t)cur * R, acc0);
         if constexpr (VEC == 8) red_add_v4_nomem(out1 + (size_t)cur * R, acc1);
       } else {
-        if constexpr (VEC == 8) st256_stream(out0 + (size_t)cur * R, acc0, acc1);
-        else st128_stream(out0 + (size_t)cur * R, acc0);
+        if constexpr (VEC == 8) st256(out0 + (size_t)cur * R, acc0, acc1);
+        else st128(out0 + (size_t)cur * R, acc0);
       }
       acc0 = make_float4(0.f, 0.f, 0.f, 0.f);
       acc1 = acc0;
     };
     auto zero_rows = [&](uint32_t r0, uint32_t r1) {  // rows (r0, r1) exclusive
       for (uint32_t r = r0 + 1; r < r1; ++r) {
-        if constexpr (VEC == 8) st256_stream(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
+        if constexpr (VEC == 8) st256(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f),
                                              make_float4(0.f, 0.f, 0.f, 0.f));
-        else st128_stream(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
+        else st128(out0 + (size_t)r * R, make_float4(0.f, 0.f, 0.f, 0.f));
       }
     };
     auto advance = [&](uint32_t i) {  // run edge inside the sub-range: close `cur`, open i
