@@ -278,6 +278,27 @@ def test_streamed_modes_edge(cuda_device):
         G.assert_parity(outs[n].cpu().numpy(), dims2, one, np.array([0.5], np.float32), f2, 32, n)
 
 
+def test_streamed_modes_orders_after_the_callers_stream(cuda_device):
+    """`stream` orders the one-shot work after what the caller queued on it: factors written on
+    that stream behind a long-running kernel must be the ones the MTTKRPs read."""
+    dims, R = (60, 50, 40), 16
+    inds, vals = synth.gen_coo(dims, 20_000, 31, val_kind="signed")
+    facs = synth.gen_factors(dims, R, 32, "signed")
+    s = torch.cuda.Stream()
+    tf = [torch.zeros((d, R), device="cuda:0") for d in dims]
+    src = [G.dev_f(f) for f in facs]
+    torch.cuda.synchronize()
+    with torch.cuda.stream(s):
+        torch.cuda._sleep(50_000_000)  # ~25 ms of spinning before the factors land
+        for t_, f_ in zip(tf, src):
+            t_.copy_(f_, non_blocking=True)
+    outs = [torch.full((d, R), float("nan"), device="cuda:0") for d in dims]
+    sf.mttkrp_streamed_modes(dims, inds, vals, tf, outs, 3, 2, stream=s)
+    torch.cuda.synchronize()
+    for n in range(3):
+        G.assert_parity(outs[n].cpu().numpy(), dims, inds, vals, facs, R, n)
+
+
 def test_streamed_modes_errors(cuda_device):
     dims, R = (10, 9, 8), 16
     inds, vals = synth.gen_coo(dims, 1000, 5)
