@@ -21,6 +21,19 @@ def main():
     import torch
 
     import paper_conf_cluster_linwds24_b200 as sf
+    torch.cuda.init()
+    l2f = os.environ.get("L2FETCH")  # experiment: cudaLimitMaxL2FetchGranularity (bytes)
+    if l2f is not None:
+        import ctypes
+        import glob
+        so = glob.glob(os.path.join(os.path.dirname(torch.__file__), "..", "nvidia", "cuda_runtime", "lib",
+                                    "libcudart.so*"))[0]
+        rt = ctypes.CDLL(so)
+        torch.zeros(1, device="cuda")
+        rc = rt.cudaDeviceSetLimit(5, ctypes.c_size_t(int(l2f)))
+        v = ctypes.c_size_t(0)
+        rt.cudaDeviceGetLimit(ctypes.byref(v), 5)
+        print(json.dumps({"l2_fetch_granularity_set": int(l2f), "rc": rc, "now": v.value}), flush=True)
     cfg = synth.CONFIGS[sys.argv[1]]
     n = int(sys.argv[2])
     src = sys.argv[3]
